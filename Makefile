@@ -29,7 +29,7 @@ oracle/liboracle.so: oracle/fgr_oracle.c oracle/fgr_oracle.h
 
 build/%.o: $(CSRC)/%.cu $(KERN_HDR)
 	@mkdir -p build
-	$(NVCC) $(NVFLAGS) -dc -o $@ $< 2> build/$*.ptxas.txt || (cat build/$*.ptxas.txt; false)
+	$(NVCC) $(NVFLAGS) -c -o $@ $< 2> build/$*.ptxas.txt || (cat build/$*.ptxas.txt; false)
 
 $(PKG)/libfastgr.so: $(KERN_OBJ)
 	$(NVCC) $(ARCH) -shared -o $@ $(KERN_OBJ) -L$(NCCL_LIB) -l:libnccl.so.2 \

@@ -1,0 +1,196 @@
+/*
+ * fastgr.h — C ABI of the B200-native batched 3-D L-shape pattern router
+ * (FastGR pattern-routing stage: PAPER.md §III-C/§III-D).
+ *
+ * Plain C: pointers and sizes only, no exceptions and no torch types cross this
+ * boundary.  Every entry point returns an fgr_status; on non-OK, fgr_last_error()
+ * returns a thread-local message.  A non-OK status from validation leaves the
+ * grid's demand untouched.  A CUDA or NCCL failure moves the handle to
+ * FGR_ERR_STATE (every later call on it returns FGR_ERR_STATE).
+ *
+ * Streams: every call enqueues on the caller's stream (cudaStream_t passed as
+ * void*, e.g. torch.cuda.current_stream().cuda_stream; NULL = legacy default).
+ * Only fgr_plan, fgr_route_batch and fgr_run_host synchronise that stream
+ * (plan returns num_batches to the host; route_batch sizes its launch).
+ *
+ * Problem statement (§II-A): a grid graph of G-cells with L
+ * metal layers, each with one preferred direction (L203-206); wire edges join
+ * adjacent G-cells on one layer and carry capacity (tracks) and demand; via
+ * edges join layers at one G-cell.  A multipin net is a set of pin points on
+ * the grid (L226-227) given as a tree of two-pin nets (L227-233).
+ */
+#ifndef FASTGR_H
+#define FASTGR_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#if defined(__GNUC__)
+#define FGR_API __attribute__((visibility("default")))
+#else
+#define FGR_API
+#endif
+
+typedef enum {
+    FGR_OK = 0,
+    FGR_ERR_INVALID = 1,   /* malformed input (see each call)                           */
+    FGR_ERR_RANGE = 2,     /* a cost could overflow the integer ranges (R19)   */
+    FGR_ERR_OOM = 3,       /* device allocation failed                                   */
+    FGR_ERR_CUDA = 4,      /* CUDA runtime error                                         */
+    FGR_ERR_NCCL = 5,      /* NCCL error                                                 */
+    FGR_ERR_STATE = 6      /* handle unusable after an earlier CUDA/NCCL failure, or a
+                              call made in the wrong state (e.g. comm not initialised)   */
+} fgr_status;
+
+/* Message for the last non-OK status returned on this thread ("" if none). */
+FGR_API const char* fgr_last_error(void);
+FGR_API const char* fgr_version(void);
+
+typedef struct fgr_grid fgr_grid;
+
+/*
+ * Grid description (cost scheme L556-563 = DESIGN.md
+ * readings R1/R2).  All integer costs:
+ *   edge cost   ec_l(e) = len_cost + T_l[clamp(cap_l(e) - dem_l(e), -S, S)]
+ *   T_l[s]      = round_half_away(ovf_weight[l] / (1 + exp(logistic_slope * s)))
+ *   via stack   V(lo,hi) = sum_{k=lo}^{hi-1} via_cost[k]
+ * Host pointers are read during fgr_grid_create only.
+ */
+typedef struct {
+    int32_t nx, ny, nlayers;           /* G-cell dims 2..32767; 2 <= nlayers <= 16            */
+    const uint8_t* dir;                /* host [nlayers]: 0 = horizontal, 1 = vertical; needs
+                                          at least one H and one V layer                       */
+    const int32_t* layer_capacity;     /* host [nlayers]: tracks per wire edge, 0..255         */
+    const uint8_t* edge_capacity;      /* DEVICE [nlayers][ny][nx] per-edge override or NULL;
+                                          copied at create.  Entry (l,y,x) is edge (x,y)-(x+1,y)
+                                          on an H layer, (x,y)-(x,y+1) on a V layer.           */
+    int32_t len_cost;                  /* per unit wire edge, >= 0 (default 64)                */
+    const int32_t* via_cost;           /* host [nlayers-1], >= 0 (default 32)                  */
+    const int32_t* ovf_weight;         /* host [nlayers], >= 0 (default 4096)                  */
+    double logistic_slope;             /* per track of slack (default 1.0)                     */
+    int32_t slack_clamp;               /* S, 0..1024 (default 64)                              */
+} fgr_grid_desc;
+
+/* Host-only: the integer logistic table T as the library builds it,
+ * table[l*(2S+1) + (s+S)] for s in [-S,S].  Needs no GPU. */
+FGR_API fgr_status fgr_cost_table(const fgr_grid_desc* desc, int64_t* table);
+
+/* Allocates the grid on `device` (demand = 0).  Errors: INVALID (desc), RANGE
+ * ((len_cost + max W) * max(nx,ny) >= 2^32), OOM, CUDA.  Caller owns *out. */
+FGR_API fgr_status fgr_grid_create(const fgr_grid_desc* desc, int device, void* stream, fgr_grid** out);
+FGR_API fgr_status fgr_grid_destroy(fgr_grid* grid);
+
+/* Demand in the dense layout int32 [nlayers][ny][nx] (same entry convention as
+ * edge_capacity; unused entries (x = nx-1 on H, y = ny-1 on V) are ignored on set
+ * and returned as 0).  DEVICE pointers.  set(NULL) zeroes the demand.  Setting the
+ * demand marks every cost stale (the next route does a full refresh). */
+FGR_API fgr_status fgr_grid_set_demand(fgr_grid* grid, const int32_t* demand, void* stream);
+FGR_API fgr_status fgr_grid_get_demand(fgr_grid* grid, int32_t* demand, void* stream);
+
+/*
+ * Nets: DEVICE pointers owned by the caller, valid for the duration of the call.
+ * CSR over nets: net i has nodes node_offset[i] .. node_offset[i+1]-1 (>= 1 node).
+ * Local node 0 is the root; parent[] is net-local with parent[j] in [0, j-1] for
+ * j >= 1 (so any descending index order is children-first) and -1 at j = 0.
+ * x,y are G-cell coordinates; [pin_lo, pin_hi] is the node's pin layer span
+ * (-1,-1 = Steiner node, or paper-literal 2-D pin).  A node and its parent must
+ * lie in different G-cells (merge coincident nodes, union their spans).
+ * Single-node nets are trivial: never batched, no demand, cost 0.
+ */
+typedef struct {
+    int32_t num_nets, num_nodes;
+    const int32_t* node_offset;        /* [num_nets+1], node_offset[0] = 0                     */
+    const int16_t* x;                  /* [num_nodes]                                           */
+    const int16_t* y;                  /* [num_nodes]                                           */
+    const int8_t* pin_lo;              /* [num_nodes]                                           */
+    const int8_t* pin_hi;              /* [num_nodes]                                           */
+    const int32_t* parent;             /* [num_nodes]                                           */
+} fgr_nets;
+
+/*
+ * fgr_plan — conflict-free batching (Algorithm 1, §III-C
+ * L468-504): non-trivial nets sorted by ascending bounding-box half-perimeter
+ * (over all tree nodes), ties by net id (L1305-1308; R12); a net
+ * joins the first batch holding no net whose closed bounding box touches its
+ * own (R13).  Computed on the device as first-fit colouring, identical to the
+ * literal repeated passes of Algorithm 1 (proof).
+ *   batch_of_net [num_nets]   DEVICE out: batch id, -1 for trivial nets
+ *   order        [num_nets]   DEVICE out: net ids grouped by batch (batch 0 first);
+ *                             trivial nets last; order inside a batch is unspecified
+ *   batch_offset [num_nets+1] DEVICE out: batch b = order[batch_offset[b] .. batch_offset[b+1])
+ *   num_batches               HOST out
+ * Errors: INVALID (malformed nets: the message names the first bad net), RANGE
+ * (a net's worst-case cost could reach 2^31, or a net too large for the
+ * on-chip DP tables), OOM, CUDA.  Synchronises `stream`.
+ */
+FGR_API fgr_status fgr_plan(fgr_grid* grid, const fgr_nets* nets, int32_t* batch_of_net, int32_t* order,
+                            int32_t* batch_offset, int32_t* num_batches, void* stream);
+
+/*
+ * fgr_route_batch — route one conflict-free batch on the current demand:
+ * cost refresh of stale rows/columns, the per-net tree DP (Eqs. (1)-(7),
+ * PAPER.md L582-756), backtrack, and the +1 demand commit of every chosen leg.
+ *   net_ids [count] DEVICE: nets of the batch (their bounding boxes must be
+ *                   pairwise disjoint — not checked; overlapping boxes give a
+ *                   result that depends on scheduling)
+ *   seg_out [num_nodes] DEVICE out: for each non-root node v (edge v -> parent u):
+ *           bend | ls<<8 | lt<<16 | straight<<24.  bend 0: bend point (x_u, y_v),
+ *           leg 1 horizontal on layer ls, leg 2 vertical on lt; bend 1: bend point
+ *           (x_v, y_u), leg 1 vertical on ls, leg 2 horizontal on lt; straight:
+ *           one leg on ls = lt.  Roots get 0xFFFFFFFF.  Other nodes untouched.
+ *   net_cost [num_nets] DEVICE out: routed cost of each listed net.
+ * Synchronises `stream` once (launch sizing).  Ignores any communicator.
+ */
+FGR_API fgr_status fgr_route_batch(fgr_grid* grid, const fgr_nets* nets, const int32_t* net_ids, int32_t count,
+                                   uint32_t* seg_out, uint32_t* net_cost, void* stream);
+
+/*
+ * fgr_route_all — the pattern-routing stage: batches in sequence (PAPER.md
+ * L504-512, Fig. 7), each routed on the demand left by all earlier batches.
+ * order/batch_offset/num_batches as returned by fgr_plan for the same nets.
+ * seg_out [num_nodes] and net_cost [num_nets] are fully written (trivial nets:
+ * seg 0xFFFFFFFF, cost 0).  With a communicator (fgr_comm_init, world > 1),
+ * each batch's nets are split across ranks and the routes are exchanged with
+ * one NCCL all-reduce per batch; every rank ends with identical outputs and
+ * demand, bitwise equal to world = 1.  No host synchronisation when the
+ * arguments are those of the grid's last fgr_plan call.
+ */
+FGR_API fgr_status fgr_route_all(fgr_grid* grid, const fgr_nets* nets, const int32_t* order,
+                                 const int32_t* batch_offset, int32_t num_batches, uint32_t* seg_out,
+                                 uint32_t* net_cost, void* stream);
+
+/* Multi-GPU (one process per GPU).  fgr_comm_unique_id fills 128 bytes on the
+ * root rank; broadcast them (e.g. torch.distributed) and call fgr_comm_init on
+ * every rank with the grid already created on that rank's device. */
+FGR_API fgr_status fgr_comm_unique_id(void* out128);
+FGR_API fgr_status fgr_comm_init(fgr_grid* grid, const void* nccl_unique_id, int rank, int world);
+
+/*
+ * fgr_run_host — end-to-end convenience over HOST buffers: copies the nets to
+ * the device, resets the demand to zero, plans, routes all batches, and copies
+ * the per-node segments and per-net costs back.  Host arrays as in fgr_nets;
+ * seg_out [num_nodes], net_cost [num_nets], num_batches may be NULL.
+ * Synchronises `stream`.
+ */
+FGR_API fgr_status fgr_run_host(fgr_grid* grid, int32_t num_nets, int32_t num_nodes, const int32_t* node_offset,
+                                const int16_t* x, const int16_t* y, const int8_t* pin_lo, const int8_t* pin_hi,
+                                const int32_t* parent, uint32_t* seg_out, uint32_t* net_cost,
+                                int32_t* num_batches, void* stream);
+
+/* Counters of the last fgr_route_all (for the byte model in DESIGN.md §5). */
+typedef struct {
+    int64_t refresh_segments;          /* 32-position row/column segments rescanned            */
+    int64_t refresh_bytes;             /* algorithmic refresh bytes (D read + cap read + P write) */
+    int64_t dp_nets, dp_edges;         /* nets and tree edges routed                            */
+    int64_t kernel_launches;           /* kernels launched by the library                       */
+    int32_t num_batches, world, rank;
+} fgr_stats;
+FGR_API fgr_status fgr_get_stats(fgr_grid* grid, fgr_stats* out);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* FASTGR_H */

@@ -1,0 +1,166 @@
+// fgr_internal.cuh — internal state and device helpers of libfastgr (not part of the ABI).
+//
+// HBM layout.  For each direction d in {H, V} the wire edges of
+// the d-layers are stored "sector-major": one line (a row for H, a column for
+// V) is a run of `len` positions, each position holding W_d words, one per
+// d-layer slot (W_d = number of d-layers rounded up to a power of two >= 4):
+//     H:  element (y, x, slot) at ((y*nx + x)*WH + slot)   edge (x,y)-(x+1,y)
+//     V:  element (x, y, slot) at ((x*ny + y)*WV + slot)   edge (x,y)-(x,y+1)
+// so all H layers of one G-cell edge sit in one 32-byte sector (L = 9: 5 H
+// layers -> WH = 8) and a tree-DP gather of a prefix position is one sector.
+// Arrays per direction: D (int32 demand), C (uint8 capacity), P (uint32
+// segment-local exclusive prefix of the edge cost), ST (uint32 per-segment
+// totals), SB (uint32 exclusive prefix of segment totals).  A segment is 32
+// consecutive positions of one line; the global prefix of position p is
+// SB[seg(p)] + P[p], so a leg cost is a difference of two such sums (exact in
+// uint32 modular arithmetic because every true prefix is < 2^32, R19).
+#pragma once
+
+#include <cuda_runtime.h>
+#include <nccl.h>
+#include <stdint.h>
+
+#include <string>
+
+#include "fastgr.h"
+
+#define FGR_SEG 32          // positions per scan segment (one warp)
+#define FGR_SEG_SHIFT 5
+#define FGR_INF 0x7FFFFFFFu // "impossible" cost; finite costs are < FGR_INF (R19)
+#define FGR_MAXL 16
+#define FGR_SMALL_NET 32    // nets with <= this many nodes take the warp path
+#define FGR_CTA_THREADS 256
+#define FGR_WARPS_PER_CTA (FGR_CTA_THREADS / 32)
+
+// ------------------------------------------------------------------ device views
+struct DirView {            // one direction's arrays
+    int32_t* D;
+    const uint8_t* C;
+    uint32_t* P;
+    uint32_t* ST;
+    uint32_t* SB;
+    int len;                // positions per line (nx for H, ny for V)
+    int lines;              // ny for H, nx for V
+    int W;                  // words per position
+    int cnt;                // layers of this direction
+    int nseg;               // segments per line
+    int seg_base;           // global segment index of this direction's first segment
+    int line_base;          // index of this direction's first line in the line counters
+};
+
+struct GridView {
+    DirView h, v;
+    int nx, ny, L, S, len_cost;
+    const int32_t* table;   // [L][2S+1]
+    uint32_t* dseg;         // [total segments] dirty flag
+    uint32_t* linecnt;      // [ny + nx] dirty segments per line
+    uint32_t* linedone;     // [ny + nx] refreshed segments per line (this launch)
+    int32_t* seglist;       // list the DP appends to (dirty segments)
+    int32_t* segcount;      // its length
+    unsigned long long* stats;  // [4] device counters (refresh segments, ...)
+    uint8_t dir[FGR_MAXL];
+    uint8_t slot[FGR_MAXL]; // index of layer l among the layers of its direction
+    uint8_t layer_of_slot[2][FGR_MAXL];
+    uint32_t viapre[FGR_MAXL + 1];  // V(lo,hi) = viapre[hi] - viapre[lo]
+};
+
+struct NetsView {
+    const int32_t* off;
+    const int16_t* x;
+    const int16_t* y;
+    const int8_t* plo;
+    const int8_t* phi;
+    const int32_t* par;
+};
+
+// ------------------------------------------------------------------ host state
+struct PlanCache {
+    bool valid = false;
+    fgr_nets nets{};
+    const int32_t* order = nullptr;
+    const int32_t* batch_offset = nullptr;
+    int num_batches = 0;
+    // host mirrors, per batch
+    int* h_off = nullptr;      // [B+1]
+    int* h_nlarge = nullptr;   // [B]
+    int* h_maxm = nullptr;     // [B] max nodes of a large net in the batch
+    long long* h_segb = nullptr;  // [B] upper bound on segments the batch can dirty
+    int cap = 0;
+};
+
+struct Scratch {            // grow-only device scratch
+    void* p = nullptr;
+    size_t bytes = 0;
+};
+
+struct fgr_grid {
+    int device = 0;
+    int nx = 0, ny = 0, L = 0, S = 0, len_cost = 0;
+    uint8_t dir[FGR_MAXL];
+    int32_t layer_capacity[FGR_MAXL];
+    int32_t via_cost[FGR_MAXL];
+    int32_t ovf_weight[FGR_MAXL];
+    double slope = 1.0;
+    int nH = 0, nV = 0, WH = 0, WV = 0;
+    GridView view{};
+    // device allocations
+    void* mem = nullptr;        // one slab for the grid arrays
+    size_t mem_bytes = 0;
+    int32_t* d_table = nullptr;
+    int32_t* d_list[2] = {nullptr, nullptr};
+    int32_t* d_count = nullptr; // [2]
+    unsigned long long* d_stats = nullptr;
+    int parity = 0;             // list the next DP appends to
+    bool full_dirty = true;     // next refresh must rescan everything
+    bool broken = false;
+    int total_segs = 0;
+    // plan scratch
+    Scratch s_plan[12];
+    PlanCache cache;
+    // multi-GPU
+    ncclComm_t comm = nullptr;
+    int rank = 0, world = 1;
+    Scratch s_rec[4];
+    fgr_stats stats{};
+    int max_smem = 0;
+    int num_sms = 0;
+};
+
+// ------------------------------------------------------------------ host helpers
+fgr_status fgr_set_error(fgr_status s, const char* fmt, ...);
+fgr_status fgr_cuda_fail(fgr_grid* g, cudaError_t e, const char* where);
+void* fgr_scratch(Scratch& s, size_t bytes, cudaError_t* err);
+
+#define FGR_CHECK_CUDA(g, expr)                                        \
+    do {                                                               \
+        cudaError_t _e = (expr);                                       \
+        if (_e != cudaSuccess) return fgr_cuda_fail((g), _e, #expr);   \
+    } while (0)
+
+// launchers (defined in the .cu files)
+cudaError_t fgr_launch_refresh(fgr_grid* g, cudaStream_t st, bool full);
+cudaError_t fgr_launch_refresh_sized(fgr_grid* g, cudaStream_t st, bool full, long long max_tasks);
+cudaError_t fgr_launch_dp(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int count,
+                          int nlarge, int maxm_large, uint32_t* seg_out, uint32_t* cost_out,
+                          uint32_t* rec_seg, const int32_t* rec_off, uint32_t* rec_cost, int list_base,
+                          bool commit);
+cudaError_t fgr_launch_commit(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int count,
+                              const uint32_t* rec_seg, const int32_t* rec_off, int list_base);
+size_t fgr_dp_smem_small(const fgr_grid* g);
+size_t fgr_dp_smem_large(const fgr_grid* g, int m);
+void fgr_flip_lists(fgr_grid* g);   // after each DP launch: the refresh consumes what the DP produced
+
+static inline NetsView fgr_nets_view(const fgr_nets* n) {
+    NetsView v;
+    v.off = n->node_offset; v.x = n->x; v.y = n->y; v.plo = n->pin_lo; v.phi = n->pin_hi; v.par = n->parent;
+    return v;
+}
+
+// ------------------------------------------------------------------ device helpers
+// min(a + b, INF) for a, b <= INF: one DPX VIADDMNMX on sm_100a.
+__device__ __forceinline__ uint32_t sat_add(uint32_t a, uint32_t b) { return __viaddmin_u32(a, b, FGR_INF); }
+
+__device__ __forceinline__ int lane_id() { return threadIdx.x & 31; }
+
+template <int N>
+struct U32Vec { uint32_t v[N]; };

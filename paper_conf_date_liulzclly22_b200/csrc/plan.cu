@@ -1,0 +1,436 @@
+// plan.cu — S0 preprocess, S1 sort, S2 conflict-free batching.
+//
+// Algorithm 1 repeated until no nets remain (L487-494), over
+// nets sorted by ascending bounding-box half-perimeter (L1305-1308, reading R12),
+// with "conflict" = the closed bounding boxes share a G-cell (L504, reading R13).
+// The repeated greedy passes assign net i (in sorted order) to
+//     batch(i) = mex { batch(j) : j before i, box(j) touches box(i) }
+// (first fit; proof in DESIGN.md §2).  On the device:
+//   1. warp per net: validation, bbox over all nodes (R14), HPWL key, range bound;
+//   2. CUB radix sort of (HPWL << 32 | id);
+//   3. spatial binning of the sorted boxes into 8x8-cell tiles, (tile, rank) pairs
+//      sorted so each tile lists its nets in rank order;
+//   4. a persistent ticketed colouring kernel: warps take nets in rank order, scan
+//      the tile lists for earlier touching boxes (each pair counted once, in the
+//      tile holding the lower-left corner of the intersection), wait for those
+//      neighbours' batch ids to be published and take the smallest free id;
+//   5. CUB radix sort of (batch << 32 | small-net flag | rank) -> batch CSR.
+#include <cub/cub.cuh>
+
+#include "fgr_internal.cuh"
+
+#define TILE_SHIFT 3
+
+namespace {
+
+struct PlanParams {
+    int N, nx, ny, L;
+    unsigned long long max_ec;   // len_cost + max W
+    unsigned long long vmax;     // V(0, L-1)
+    int max_nodes_large;         // largest net the CTA path can hold in shared memory
+};
+
+__device__ __forceinline__ unsigned long long pack_box(int x0, int y0, int x1, int y1) {
+    return (unsigned long long)(uint16_t)x0 | ((unsigned long long)(uint16_t)y0 << 16) |
+           ((unsigned long long)(uint16_t)x1 << 32) | ((unsigned long long)(uint16_t)y1 << 48);
+}
+__device__ __forceinline__ void unpack_box(unsigned long long b, int& x0, int& y0, int& x1, int& y1) {
+    x0 = (int)(b & 0xFFFF); y0 = (int)((b >> 16) & 0xFFFF); x1 = (int)((b >> 32) & 0xFFFF); y1 = (int)(b >> 48);
+}
+
+// S0: one warp per net.
+__global__ void k_preprocess(PlanParams p, NetsView nv, unsigned long long* __restrict__ keys,
+                             unsigned long long* __restrict__ box, int* __restrict__ msize, int* __restrict__ segb,
+                             int* __restrict__ counters /* [0] trivial, [1] err invalid net, [2] err range net */) {
+    const int warp = (int)((blockIdx.x * (size_t)blockDim.x + threadIdx.x) >> 5);
+    const int lane = lane_id();
+    if (warp >= p.N) return;
+    const int net = warp;
+    const int a0 = nv.off[net], a1 = nv.off[net + 1];
+    const int m = a1 - a0;
+    int bad = (m <= 0);
+    int x0 = 0x7FFF, y0 = 0x7FFF, x1 = -1, y1 = -1;
+    unsigned long long wl = 0;
+    int sb = 0;
+    for (int i = lane; i < m; i += 32) {
+        const int v = a0 + i;
+        const int x = nv.x[v], y = nv.y[v];
+        const int lo = nv.plo[v], hi = nv.phi[v];
+        if (x < 0 || x >= p.nx || y < 0 || y >= p.ny) bad = 1;
+        if (!((lo == -1 && hi == -1) || (lo >= 0 && lo <= hi && hi < p.L))) bad = 1;
+        x0 = min(x0, x); y0 = min(y0, y); x1 = max(x1, x); y1 = max(y1, y);
+        const int par = nv.par[v];
+        if (i == 0) { if (par != -1) bad = 1; }
+        else if (par < 0 || par >= i) bad = 1;
+        else {
+            const int xu = nv.x[a0 + par], yu = nv.y[a0 + par];
+            const int dx = abs(x - xu), dy = abs(y - yu);
+            if (dx == 0 && dy == 0) bad = 1;   // zero-length tree edge (R8)
+            wl += (unsigned long long)(dx + dy);
+            sb += (dx >> 5) + (dy >> 5) + 4;
+        }
+    }
+#pragma unroll
+    for (int off = 16; off; off >>= 1) {
+        bad |= __shfl_xor_sync(0xffffffffu, bad, off);
+        x0 = min(x0, __shfl_xor_sync(0xffffffffu, x0, off));
+        y0 = min(y0, __shfl_xor_sync(0xffffffffu, y0, off));
+        x1 = max(x1, __shfl_xor_sync(0xffffffffu, x1, off));
+        y1 = max(y1, __shfl_xor_sync(0xffffffffu, y1, off));
+        wl += __shfl_xor_sync(0xffffffffu, wl, off);
+        sb += __shfl_xor_sync(0xffffffffu, sb, off);
+    }
+    if (lane) return;
+    if (bad) {
+        atomicMin(&counters[1], net);
+        x0 = y0 = x1 = y1 = 0;
+    }
+    const bool trivial = (m == 1);
+    if (trivial) atomicAdd(&counters[0], 1);
+    if (!bad && !trivial) {
+        // R19: worst case of any route = every unit edge at max cost + every via stack at max
+        const unsigned long long bound = wl * p.max_ec + (unsigned long long)(2 * m) * p.vmax;
+        if (bound >= (unsigned long long)FGR_INF || m > p.max_nodes_large) atomicMin(&counters[2], net);
+    }
+    const unsigned hpwl = trivial ? 0xFFFFu : (unsigned)((x1 - x0) + (y1 - y0));
+    keys[net] = ((unsigned long long)hpwl << 32) | (unsigned)net;
+    box[net] = pack_box(x0, y0, x1, y1);
+    msize[net] = m;
+    segb[net] = sb;
+}
+
+__global__ void k_rank_boxes(int N, const int* __restrict__ counters, const unsigned long long* __restrict__ keys,
+                             const unsigned long long* __restrict__ box, unsigned long long* __restrict__ box_r,
+                             int* __restrict__ tcount, int tiles_x) {
+    const int r = blockIdx.x * blockDim.x + threadIdx.x;
+    if (r > N) return;
+    const int R = N - counters[0];
+    if (r >= R) { tcount[r] = 0; return; }
+    const unsigned long long b = box[(unsigned)(keys[r] & 0xFFFFFFFFu)];
+    box_r[r] = b;
+    int x0, y0, x1, y1;
+    unpack_box(b, x0, y0, x1, y1);
+    tcount[r] = ((x1 >> TILE_SHIFT) - (x0 >> TILE_SHIFT) + 1) * ((y1 >> TILE_SHIFT) - (y0 >> TILE_SHIFT) + 1);
+}
+
+__global__ void k_tile_emit(int R, const unsigned long long* __restrict__ box_r, const int* __restrict__ toff,
+                            unsigned long long* __restrict__ tkeys, int tiles_x) {
+    const int r = blockIdx.x * blockDim.x + threadIdx.x;
+    if (r >= R) return;
+    int x0, y0, x1, y1;
+    unpack_box(box_r[r], x0, y0, x1, y1);
+    int k = toff[r];
+    for (int ty = y0 >> TILE_SHIFT; ty <= (y1 >> TILE_SHIFT); ty++)
+        for (int tx = x0 >> TILE_SHIFT; tx <= (x1 >> TILE_SHIFT); tx++)
+            tkeys[k++] = ((unsigned long long)(ty * tiles_x + tx) << 32) | (unsigned)r;
+}
+
+__global__ void k_tile_bounds(int T, const unsigned long long* __restrict__ tkeys, int* __restrict__ tstart,
+                              int* __restrict__ tend, int* __restrict__ entries) {
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= T) return;
+    const unsigned long long k = tkeys[i];
+    const int t = (int)(k >> 32);
+    entries[i] = (int)(k & 0xFFFFFFFFu);
+    if (i == 0 || (int)(tkeys[i - 1] >> 32) != t) tstart[t] = i;
+    if (i == T - 1 || (int)(tkeys[i + 1] >> 32) != t) tend[t] = i + 1;
+}
+
+// S2 core: first-fit colouring in rank order, dataflow over published colours.
+#define COLOR_BITS 1024
+__global__ void __launch_bounds__(256) k_color(int R, const unsigned long long* __restrict__ box_r,
+                                               const int* __restrict__ tstart, const int* __restrict__ tend,
+                                               const int* __restrict__ entries, int tiles_x, int* color,
+                                               int* __restrict__ ticket, int* __restrict__ nbatches,
+                                               int* __restrict__ bcount) {
+    __shared__ uint32_t bits[8][COLOR_BITS / 32];
+    const int w = threadIdx.x >> 5, lane = lane_id();
+    uint32_t* bw = bits[w];
+    volatile int* vcolor = color;
+    for (;;) {
+        int r = 0;
+        if (lane == 0) r = atomicAdd(ticket, 1);
+        r = __shfl_sync(0xffffffffu, r, 0);
+        if (r >= R) return;
+        int x0, y0, x1, y1;
+        unpack_box(box_r[r], x0, y0, x1, y1);
+        int result = -1;
+        for (int wb = 0; result < 0; wb += COLOR_BITS) {
+            for (int q = lane; q < COLOR_BITS / 32; q += 32) bw[q] = 0;
+            __syncwarp();
+            for (int ty = y0 >> TILE_SHIFT; ty <= (y1 >> TILE_SHIFT); ty++)
+                for (int tx = x0 >> TILE_SHIFT; tx <= (x1 >> TILE_SHIFT); tx++) {
+                    const int t = ty * tiles_x + tx;
+                    const int s = tstart[t], e = tend[t];
+                    for (int base = s; base < e; base += 32) {
+                        const int j = base + lane;
+                        const int rr = j < e ? entries[j] : 0x7FFFFFFF;
+                        if (rr < r) {
+                            int a0, b0, a1, b1;
+                            unpack_box(box_r[rr], a0, b0, a1, b1);
+                            if (!(a1 < x0 || x1 < a0 || b1 < y0 || y1 < b0)) {
+                                const int cx = max(a0, x0) >> TILE_SHIFT, cy = max(b0, y0) >> TILE_SHIFT;
+                                if (cx == tx && cy == ty) {           // count each pair once
+                                    int c;
+                                    while ((c = vcolor[rr]) < 0) __nanosleep(64);
+                                    c -= wb;
+                                    if (c >= 0 && c < COLOR_BITS) atomicOr(&bw[c >> 5], 1u << (c & 31));
+                                }
+                            }
+                        }
+                        if (__any_sync(0xffffffffu, j < e && rr >= r)) break;   // lists are rank-sorted
+                    }
+                }
+            __syncwarp();
+            // smallest clear bit in this window
+            int found = -1;
+            for (int q0 = 0; q0 < COLOR_BITS / 32 && found < 0; q0 += 32) {
+                const uint32_t word = bw[q0 + lane];
+                const uint32_t freeb = ~word;
+                const uint32_t any = __ballot_sync(0xffffffffu, freeb != 0);
+                if (any) {
+                    const int ql = __ffs(any) - 1;
+                    const uint32_t fw = __shfl_sync(0xffffffffu, freeb, ql);
+                    found = (q0 + ql) * 32 + __ffs(fw) - 1;
+                }
+            }
+            __syncwarp();
+            if (found >= 0) result = wb + found;
+        }
+        if (lane == 0) {
+            __threadfence();
+            atomicExch(&color[r], result);
+            atomicMax(nbatches, result + 1);
+            atomicAdd(&bcount[result], 1);
+        }
+    }
+}
+
+__global__ void k_batch_keys(int R, const int* __restrict__ color, const unsigned long long* __restrict__ keys,
+                             const int* __restrict__ msize, unsigned long long* __restrict__ bkeys) {
+    const int r = blockIdx.x * blockDim.x + threadIdx.x;
+    if (r >= R) return;
+    const int id = (int)(keys[r] & 0xFFFFFFFFu);
+    const unsigned small = msize[id] > FGR_SMALL_NET ? 0u : 0x80000000u;
+    bkeys[r] = ((unsigned long long)color[r] << 32) | small | (unsigned)r;
+}
+
+__global__ void k_finalize(int N, const int* __restrict__ counters, const unsigned long long* __restrict__ keys,
+                           const unsigned long long* __restrict__ bkeys, const int* __restrict__ msize,
+                           const int* __restrict__ segb, int* __restrict__ order, int* __restrict__ batch_of_net,
+                           int* __restrict__ nlarge, int* __restrict__ maxm, unsigned long long* __restrict__ segsum) {
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= N) return;
+    const int R = N - counters[0];
+    if (i < R) {
+        const unsigned long long bk = bkeys[i];
+        const int r = (int)(bk & 0x7FFFFFFFu);
+        const int c = (int)(bk >> 32);
+        const int id = (int)(keys[r] & 0xFFFFFFFFu);
+        order[i] = id;
+        batch_of_net[id] = c;
+        const int m = msize[id];
+        if (m > FGR_SMALL_NET) { atomicAdd(&nlarge[c], 1); atomicMax(&maxm[c], m); }
+        // per-batch sum of dirty-segment bounds (refresh launch sizing); keys are
+        // batch-sorted, so a warp almost always shares one batch id
+        const unsigned long long v = (unsigned long long)segb[id];
+        const unsigned act = __activemask();
+        const int lead = __ffs(act) - 1;
+        const int c0 = __shfl_sync(act, c, lead);
+        if (__all_sync(act, c == c0)) {
+            const unsigned sum = __reduce_add_sync(act, (unsigned)v);
+            if (lane_id() == lead) atomicAdd(&segsum[c], (unsigned long long)sum);
+        } else {
+            atomicAdd(&segsum[c], v);
+        }
+    } else {
+        const int id = (int)(keys[i] & 0xFFFFFFFFu);
+        order[i] = id;
+        batch_of_net[id] = -1;
+    }
+}
+
+template <typename T>
+T* take(fgr_grid* g, int slot, size_t n, cudaError_t* e) {
+    return (T*)fgr_scratch(g->s_plan[slot], n * sizeof(T), e);
+}
+
+int bits_for(long long v) {
+    int b = 1;
+    while ((1LL << b) <= v) b++;
+    return b;
+}
+
+}  // namespace
+
+// largest net the CTA path can hold (shared memory), capped by its depth arrays
+static int max_large_nodes(const fgr_grid* g) {
+    int m = 2048;
+    while (m > FGR_SMALL_NET && fgr_dp_smem_large(g, m) + 64 > (size_t)g->max_smem) m -= 16;
+    return m;
+}
+
+extern "C" FGR_API fgr_status fgr_plan(fgr_grid* g, const fgr_nets* nets, int32_t* batch_of_net, int32_t* order,
+                                       int32_t* batch_offset, int32_t* num_batches, void* stream) {
+    if (!g || !nets || !num_batches) return fgr_set_error(FGR_ERR_INVALID, "NULL argument");
+    if (g->broken) return fgr_set_error(FGR_ERR_STATE, "grid unusable after an earlier CUDA/NCCL error");
+    const int N = nets->num_nets;
+    if (N < 0 || nets->num_nodes < 0) return fgr_set_error(FGR_ERR_INVALID, "negative sizes");
+    if (N > 0 && (!nets->node_offset || !nets->x || !nets->y || !nets->pin_lo || !nets->pin_hi || !nets->parent ||
+                  !batch_of_net || !order || !batch_offset))
+        return fgr_set_error(FGR_ERR_INVALID, "NULL array");
+    cudaStream_t st = (cudaStream_t)stream;
+    FGR_CHECK_CUDA(g, cudaSetDevice(g->device));
+    g->cache.valid = false;
+    *num_batches = 0;
+    if (N == 0) {
+        FGR_CHECK_CUDA(g, cudaMemsetAsync(batch_offset, 0, sizeof(int32_t), st));
+        FGR_CHECK_CUDA(g, cudaStreamSynchronize(st));
+        g->cache.valid = true;
+        g->cache.nets = *nets; g->cache.order = order; g->cache.batch_offset = batch_offset; g->cache.num_batches = 0;
+        return FGR_OK;
+    }
+    cudaError_t e = cudaSuccess;
+    const NetsView nv = fgr_nets_view(nets);
+    PlanParams p;
+    p.N = N; p.nx = g->nx; p.ny = g->ny; p.L = g->L;
+    int maxw = 0;
+    for (int l = 0; l < g->L; l++) maxw = g->ovf_weight[l] > maxw ? g->ovf_weight[l] : maxw;
+    p.max_ec = (unsigned long long)g->len_cost + (unsigned long long)maxw;
+    p.vmax = g->view.viapre[g->L - 1];
+    p.max_nodes_large = max_large_nodes(g);
+
+    const int tiles_x = ((g->nx - 1) >> TILE_SHIFT) + 1, tiles_y = ((g->ny - 1) >> TILE_SHIFT) + 1;
+    const int ntiles = tiles_x * tiles_y;
+    auto* keys = take<unsigned long long>(g, 0, N, &e);
+    auto* keys_s = take<unsigned long long>(g, 1, N, &e);
+    auto* box = take<unsigned long long>(g, 2, N, &e);
+    auto* box_r = take<unsigned long long>(g, 3, (size_t)N + 1, &e);
+    auto* msize = take<int>(g, 4, N, &e);
+    auto* segb = take<int>(g, 5, N, &e);
+    auto* tcount = take<int>(g, 6, (size_t)N + 1, &e);
+    // counters: [0] trivial [1] err invalid [2] err range [3] ticket [4] nbatches [5..] spare
+    auto* counters = take<int>(g, 7, 16 + 2 * (size_t)ntiles, &e);
+    if (e != cudaSuccess) return fgr_cuda_fail(g, e, "plan scratch");
+    int* tstart = counters + 16;
+    int* tend = tstart + ntiles;
+    int hc[8] = {0, 0x7FFFFFFF, 0x7FFFFFFF, 0, 0, 0, 0, 0};
+    FGR_CHECK_CUDA(g, cudaMemcpyAsync(counters, hc, sizeof(hc), cudaMemcpyHostToDevice, st));
+    FGR_CHECK_CUDA(g, cudaMemsetAsync(tstart, 0, 2 * sizeof(int) * ntiles, st));
+    k_preprocess<<<(unsigned)(((size_t)N * 32 + 255) / 256), 256, 0, st>>>(p, nv, keys, box, msize, segb, counters);
+    FGR_CHECK_CUDA(g, cudaGetLastError());
+    // S1: sort by (HPWL, id)
+    size_t tmp_bytes = 0;
+    cub::DeviceRadixSort::SortKeys(nullptr, tmp_bytes, keys, keys_s, N, 0, 48, st);
+    void* tmp = fgr_scratch(g->s_plan[8], tmp_bytes, &e);
+    if (e != cudaSuccess) return fgr_cuda_fail(g, e, "plan sort scratch");
+    FGR_CHECK_CUDA(g, cub::DeviceRadixSort::SortKeys(tmp, tmp_bytes, keys, keys_s, N, 0, 48, st));
+    k_rank_boxes<<<(N + 1 + 255) / 256, 256, 0, st>>>(N, counters, keys_s, box, box_r, tcount, tiles_x);
+    FGR_CHECK_CUDA(g, cudaGetLastError());
+    // tile offsets
+    int* toff = (int*)keys;   // keys (N x 8 B) are no longer needed: reuse as N+1 ints
+    tmp_bytes = 0;
+    cub::DeviceScan::ExclusiveSum(nullptr, tmp_bytes, tcount, toff, N + 1, st);
+    tmp = fgr_scratch(g->s_plan[8], tmp_bytes, &e);
+    if (e != cudaSuccess) return fgr_cuda_fail(g, e, "plan scan scratch");
+    FGR_CHECK_CUDA(g, cub::DeviceScan::ExclusiveSum(tmp, tmp_bytes, tcount, toff, N + 1, st));
+    int hbuf[4];
+    FGR_CHECK_CUDA(g, cudaMemcpyAsync(hbuf, counters, 3 * sizeof(int), cudaMemcpyDeviceToHost, st));
+    int T = 0;
+    FGR_CHECK_CUDA(g, cudaMemcpyAsync(&T, toff + N, sizeof(int), cudaMemcpyDeviceToHost, st));
+    FGR_CHECK_CUDA(g, cudaStreamSynchronize(st));  // sync 1 of 2
+    if (hbuf[1] != 0x7FFFFFFF)
+        return fgr_set_error(FGR_ERR_INVALID, "net %d is malformed (node count, coordinates, pin span, parent "
+                             "index (must be in [0, j-1]) or a zero-length tree edge)", hbuf[1]);
+    if (hbuf[2] != 0x7FFFFFFF)
+        return fgr_set_error(FGR_ERR_RANGE, "net %d: worst-case cost may reach 2^31 or it has more than %d nodes",
+                             hbuf[2], p.max_nodes_large);
+    const int R = N - hbuf[0];
+    // S2: binning
+    auto* tkeys = take<unsigned long long>(g, 9, (size_t)T + 1, &e);
+    auto* tkeys_s = take<unsigned long long>(g, 10, (size_t)T + 1, &e);
+    if (e != cudaSuccess) return fgr_cuda_fail(g, e, "plan tile scratch");
+    int* entries = (int*)tkeys;   // reused after the sort
+    int* color = tcount;          // N+1 ints, tcount no longer needed after the scan
+    if (R > 0) {
+        k_tile_emit<<<(R + 255) / 256, 256, 0, st>>>(R, box_r, toff, tkeys, tiles_x);
+        FGR_CHECK_CUDA(g, cudaGetLastError());
+        tmp_bytes = 0;
+        const int tb = 32 + bits_for(ntiles);
+        cub::DeviceRadixSort::SortKeys(nullptr, tmp_bytes, tkeys, tkeys_s, T, 0, tb, st);
+        tmp = fgr_scratch(g->s_plan[8], tmp_bytes, &e);
+        if (e != cudaSuccess) return fgr_cuda_fail(g, e, "plan tile sort scratch");
+        FGR_CHECK_CUDA(g, cub::DeviceRadixSort::SortKeys(tmp, tmp_bytes, tkeys, tkeys_s, T, 0, tb, st));
+        k_tile_bounds<<<(T + 255) / 256, 256, 0, st>>>(T, tkeys_s, tstart, tend, entries);
+        FGR_CHECK_CUDA(g, cudaGetLastError());
+    }
+    // colouring
+    auto* bc = take<int>(g, 11, 3 * ((size_t)R + 1), &e);   // bcount | nlarge | maxm
+    if (e != cudaSuccess) return fgr_cuda_fail(g, e, "plan batch scratch");
+    int* d_bcount = bc;
+    int* d_nlarge = bc + (R + 1);
+    int* d_maxm = bc + 2 * (R + 1);
+    FGR_CHECK_CUDA(g, cudaMemsetAsync(bc, 0, 3 * sizeof(int) * ((size_t)R + 1), st));
+    FGR_CHECK_CUDA(g, cudaMemsetAsync(color, 0xFF, sizeof(int) * ((size_t)N + 1), st));
+    FGR_CHECK_CUDA(g, cudaMemsetAsync(batch_of_net, 0xFF, sizeof(int) * (size_t)N, st));
+    if (R > 0) {
+        int occ = 1;
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_color, 256, 0);
+        int blocks = g->num_sms * (occ > 0 ? occ : 1);
+        int need = (R + 7) / 8;
+        if (blocks > need) blocks = need;
+        k_color<<<blocks, 256, 0, st>>>(R, box_r, tstart, tend, entries, tiles_x, color, counters + 3, counters + 4,
+                                        d_bcount);
+        FGR_CHECK_CUDA(g, cudaGetLastError());
+        g->stats.kernel_launches++;
+    }
+    // batch CSR
+    auto* bkeys = (unsigned long long*)box;      // box (N x 8 B) no longer needed
+    auto* bkeys_s = keys;                        // keys region (toff) no longer needed after emit
+    if (R > 0) {
+        k_batch_keys<<<(R + 255) / 256, 256, 0, st>>>(R, color, keys_s, msize, bkeys);
+        FGR_CHECK_CUDA(g, cudaGetLastError());
+        tmp_bytes = 0;
+        const int bb = 32 + bits_for(R);
+        cub::DeviceRadixSort::SortKeys(nullptr, tmp_bytes, bkeys, bkeys_s, R, 0, bb, st);
+        tmp = fgr_scratch(g->s_plan[8], tmp_bytes, &e);
+        if (e != cudaSuccess) return fgr_cuda_fail(g, e, "plan batch sort scratch");
+        FGR_CHECK_CUDA(g, cub::DeviceRadixSort::SortKeys(tmp, tmp_bytes, bkeys, bkeys_s, R, 0, bb, st));
+    }
+    tmp_bytes = 0;
+    cub::DeviceScan::ExclusiveSum(nullptr, tmp_bytes, d_bcount, batch_offset, R + 1, st);
+    tmp = fgr_scratch(g->s_plan[8], tmp_bytes, &e);
+    if (e != cudaSuccess) return fgr_cuda_fail(g, e, "plan offset scratch");
+    FGR_CHECK_CUDA(g, cub::DeviceScan::ExclusiveSum(tmp, tmp_bytes, d_bcount, batch_offset, R + 1, st));
+    auto* segsum = (unsigned long long*)box_r;   // box_r no longer needed after colouring
+    FGR_CHECK_CUDA(g, cudaMemsetAsync(segsum, 0, sizeof(unsigned long long) * ((size_t)R + 1), st));
+    k_finalize<<<(N + 255) / 256, 256, 0, st>>>(N, counters, keys_s, bkeys_s, msize, segb, order, batch_of_net,
+                                                d_nlarge, d_maxm, segsum);
+    FGR_CHECK_CUDA(g, cudaGetLastError());
+    g->stats.kernel_launches += 6;
+    int B = 0;
+    FGR_CHECK_CUDA(g, cudaMemcpyAsync(&B, counters + 4, sizeof(int), cudaMemcpyDeviceToHost, st));
+    FGR_CHECK_CUDA(g, cudaStreamSynchronize(st));  // sync 2 of 2
+    PlanCache& c = g->cache;
+    if (c.cap < B + 1) {
+        free(c.h_off); free(c.h_nlarge); free(c.h_maxm);
+        c.cap = B + 1;
+        c.h_off = (int*)malloc(sizeof(int) * c.cap);
+        c.h_nlarge = (int*)malloc(sizeof(int) * c.cap);
+        c.h_maxm = (int*)malloc(sizeof(int) * c.cap);
+        c.h_segb = (long long*)malloc(sizeof(long long) * c.cap);
+    }
+    if (B > 0) {
+        FGR_CHECK_CUDA(g, cudaMemcpy(c.h_off, batch_offset, sizeof(int) * (B + 1), cudaMemcpyDeviceToHost));
+        FGR_CHECK_CUDA(g, cudaMemcpy(c.h_nlarge, d_nlarge, sizeof(int) * B, cudaMemcpyDeviceToHost));
+        FGR_CHECK_CUDA(g, cudaMemcpy(c.h_maxm, d_maxm, sizeof(int) * B, cudaMemcpyDeviceToHost));
+        FGR_CHECK_CUDA(g, cudaMemcpy(c.h_segb, segsum, sizeof(long long) * B, cudaMemcpyDeviceToHost));
+    }
+    c.valid = true;
+    c.nets = *nets;
+    c.order = order;
+    c.batch_offset = batch_offset;
+    c.num_batches = B;
+    *num_batches = B;
+    return FGR_OK;
+}

@@ -1,0 +1,197 @@
+// refresh.cu — S3 cost refresh (north_star "logistic congestion
+// cost, then a warp-shuffle segmented scan into per-layer prefix sums").
+//
+// The paper only says the wire cost considers wirelength and congestion and defers
+// the formula to [3]; our integer reading is R1.
+//
+// One warp refreshes one 32-position segment of one row (H layers) or column (V
+// layers): lane j owns position 32*s + j and all W layer slots of it (one
+// 16/32/64-byte sector), computes ec = len + T[clamp(cap - dem)] per slot, runs a
+// 5-step __shfl_up_sync inclusive scan per slot, and writes the exclusive
+// segment-local prefix P and the segment total ST.  The warp that finishes the
+// last dirty segment of a line (per-line atomic counter) rescans that line's
+// segment totals into the segment bases SB.  Only segments the previous batch
+// committed to are rescanned (dirty list built by the DP's commit), so the bytes
+// moved per batch follow the demand that changed, not the grid size.
+#include "fgr_internal.cuh"
+
+template <int W>
+struct Vec {
+    static __device__ __forceinline__ void load_i32(const int32_t* p, int32_t (&o)[W]) {
+#pragma unroll
+        for (int q = 0; q < W / 4; q++) {
+            int4 t = reinterpret_cast<const int4*>(p)[q];
+            o[4 * q] = t.x; o[4 * q + 1] = t.y; o[4 * q + 2] = t.z; o[4 * q + 3] = t.w;
+        }
+    }
+    static __device__ __forceinline__ void load_u32_cg(const uint32_t* p, uint32_t (&o)[W]) {
+#pragma unroll
+        for (int q = 0; q < W / 4; q++) {
+            uint4 t = __ldcg(reinterpret_cast<const uint4*>(p) + q);
+            o[4 * q] = t.x; o[4 * q + 1] = t.y; o[4 * q + 2] = t.z; o[4 * q + 3] = t.w;
+        }
+    }
+    static __device__ __forceinline__ void store_u32(uint32_t* p, const uint32_t (&o)[W]) {
+#pragma unroll
+        for (int q = 0; q < W / 4; q++)
+            reinterpret_cast<uint4*>(p)[q] = make_uint4(o[4 * q], o[4 * q + 1], o[4 * q + 2], o[4 * q + 3]);
+    }
+    static __device__ __forceinline__ void load_u8(const uint8_t* p, uint8_t (&o)[W]) {
+        if constexpr (W == 4) {
+            uint32_t t = *reinterpret_cast<const uint32_t*>(p);
+#pragma unroll
+            for (int k = 0; k < 4; k++) o[k] = (uint8_t)(t >> (8 * k));
+        } else if constexpr (W == 8) {
+            uint2 t = *reinterpret_cast<const uint2*>(p);
+#pragma unroll
+            for (int k = 0; k < 4; k++) { o[k] = (uint8_t)(t.x >> (8 * k)); o[4 + k] = (uint8_t)(t.y >> (8 * k)); }
+        } else {
+            uint4 t = *reinterpret_cast<const uint4*>(p);
+            uint32_t w4[4] = {t.x, t.y, t.z, t.w};
+#pragma unroll
+            for (int k = 0; k < 16; k++) o[k] = (uint8_t)(w4[k >> 2] >> (8 * (k & 3)));
+        }
+    }
+};
+
+template <int W>
+__device__ __forceinline__ void warp_incl_scan(uint32_t (&x)[W]) {
+    const int lane = lane_id();
+#pragma unroll
+    for (int off = 1; off < 32; off <<= 1) {
+#pragma unroll
+        for (int k = 0; k < W; k++) {
+            uint32_t t = __shfl_up_sync(0xffffffffu, x[k], off);
+            if (lane >= off) x[k] += t;
+        }
+    }
+}
+
+template <int W>
+__device__ __forceinline__ void refresh_segment(const GridView& g, const DirView& d, int dsel, int line, int s,
+                                                int gs, bool full) {
+    const int lane = lane_id();
+    const int pos = s * FGR_SEG + lane;
+    const bool inb = pos < d.len;
+    const bool edge = pos < d.len - 1;
+    const size_t base = ((size_t)line * d.len + pos) * W;
+    int32_t dem[W];
+    uint8_t cap[W];
+    uint32_t ec[W], incl[W];
+    if (inb) {
+        Vec<W>::load_i32(d.D + base, dem);
+        Vec<W>::load_u8(d.C + base, cap);
+    }
+    const int span = 2 * g.S + 1;
+#pragma unroll
+    for (int k = 0; k < W; k++) {
+        uint32_t c = 0;
+        if (edge && k < d.cnt) {
+            int sl = (int)cap[k] - dem[k];
+            sl = sl < -g.S ? -g.S : (sl > g.S ? g.S : sl);
+            c = (uint32_t)g.len_cost + (uint32_t)__ldg(g.table + g.layer_of_slot[dsel][k] * span + sl + g.S);
+        }
+        ec[k] = c;
+        incl[k] = c;
+    }
+    warp_incl_scan<W>(incl);
+    if (inb) {
+        uint32_t p[W];
+#pragma unroll
+        for (int k = 0; k < W; k++) p[k] = incl[k] - ec[k];
+        Vec<W>::store_u32(d.P + base, p);
+    }
+    if (lane == 31) Vec<W>::store_u32(d.ST + ((size_t)line * d.nseg + s) * W, incl);
+    const int lidx = d.line_base + line;
+    int last = 0;
+    if (lane == 0) {
+        g.dseg[gs] = 0;
+        __threadfence();
+        unsigned need = full ? (unsigned)d.nseg : g.linecnt[lidx];
+        unsigned old = atomicAdd(&g.linedone[lidx], 1u);
+        last = (old + 1 == need);
+    }
+    last = __shfl_sync(0xffffffffu, last, 0);
+    if (!last) return;
+    __threadfence();
+    // Segment bases of this line: exclusive scan of all segment totals.
+    uint32_t carry[W];
+#pragma unroll
+    for (int k = 0; k < W; k++) carry[k] = 0;
+    for (int c0 = 0; c0 < d.nseg; c0 += 32) {
+        const int s2 = c0 + lane;
+        uint32_t v[W], inc[W];
+        if (s2 < d.nseg) Vec<W>::load_u32_cg(d.ST + ((size_t)line * d.nseg + s2) * W, v);
+        else {
+#pragma unroll
+            for (int k = 0; k < W; k++) v[k] = 0;
+        }
+#pragma unroll
+        for (int k = 0; k < W; k++) inc[k] = v[k];
+        warp_incl_scan<W>(inc);
+        if (s2 < d.nseg) {
+            uint32_t o[W];
+#pragma unroll
+            for (int k = 0; k < W; k++) o[k] = carry[k] + inc[k] - v[k];
+            Vec<W>::store_u32(d.SB + ((size_t)line * d.nseg + s2) * W, o);
+        }
+#pragma unroll
+        for (int k = 0; k < W; k++) carry[k] += __shfl_sync(0xffffffffu, inc[k], 31);
+    }
+    if (lane == 0) { g.linedone[lidx] = 0; g.linecnt[lidx] = 0; }
+}
+
+template <int WH, int WV>
+__global__ void __launch_bounds__(256) k_refresh(GridView g, const int32_t* __restrict__ list,
+                                                 const int32_t* __restrict__ count, int full) {
+    const int hsegs = g.h.lines * g.h.nseg;
+    const int ntasks = full ? hsegs + g.v.lines * g.v.nseg : *count;
+    const int warp = (int)((blockIdx.x * (size_t)blockDim.x + threadIdx.x) >> 5);
+    const int nwarps = (int)((gridDim.x * (size_t)blockDim.x) >> 5);
+    unsigned nh = 0, nv = 0;
+    for (int t = warp; t < ntasks; t += nwarps) {
+        const int gs = full ? t : list[t];
+        if (gs < hsegs) {
+            const int line = gs / g.h.nseg;
+            refresh_segment<WH>(g, g.h, 0, line, gs - line * g.h.nseg, gs, full);
+            nh++;
+        } else {
+            const int r = gs - hsegs;
+            const int line = r / g.v.nseg;
+            refresh_segment<WV>(g, g.v, 1, line, r - line * g.v.nseg, gs, full);
+            nv++;
+        }
+    }
+    if (lane_id() == 0 && (nh | nv)) {
+        atomicAdd(&g.stats[0], (unsigned long long)nh);
+        atomicAdd(&g.stats[1], (unsigned long long)nv);
+    }
+}
+
+template <int WH, int WV>
+static cudaError_t launch_t(fgr_grid* g, cudaStream_t st, bool full, int blocks) {
+    const int consume = g->parity ^ 1;   // the list the last DP filled
+    k_refresh<WH, WV><<<blocks, 256, 0, st>>>(g->view, g->d_list[consume], g->d_count + consume, full ? 1 : 0);
+    return cudaGetLastError();
+}
+
+// Upper bound on tasks is passed through g->stats.kernel_launches bookkeeping by the caller.
+cudaError_t fgr_launch_refresh_sized(fgr_grid* g, cudaStream_t st, bool full, long long max_tasks) {
+    int cap_blocks = g->num_sms * 8;
+    long long tasks = full ? (long long)g->total_segs : max_tasks;
+    if (tasks <= 0) return cudaSuccess;
+    int blocks = (int)((tasks + 7) / 8);
+    if (blocks > cap_blocks) blocks = cap_blocks;
+    if (blocks < 1) blocks = 1;
+    g->stats.kernel_launches++;
+    const int wh = g->WH, wv = g->WV;
+#define FGR_RL(A, B) if (wh == A && wv == B) return launch_t<A, B>(g, st, full, blocks);
+    FGR_RL(4, 4) FGR_RL(4, 8) FGR_RL(4, 16) FGR_RL(8, 4) FGR_RL(8, 8) FGR_RL(8, 16) FGR_RL(16, 4) FGR_RL(16, 8)
+    FGR_RL(16, 16)
+#undef FGR_RL
+    return cudaErrorInvalidValue;
+}
+
+cudaError_t fgr_launch_refresh(fgr_grid* g, cudaStream_t st, bool full) {
+    return fgr_launch_refresh_sized(g, st, full, (long long)g->total_segs);
+}

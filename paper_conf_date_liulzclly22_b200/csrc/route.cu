@@ -1,0 +1,340 @@
+// route.cu — the pattern-routing stage driver: batches in sequence (PAPER.md
+// L504-512, Fig. 7 "kernels invoked sequentially, each processing one batch"),
+// each batch = [cost refresh of the segments the previous batch dirtied] ->
+// [tree DP + backtrack + commit].  Multi-GPU (not in the paper; north_star): the
+// grid is replicated, each batch's nets are split across ranks, the per-node
+// route records of the batch are exchanged with one NCCL all-reduce (records of
+// other ranks' nets are zero), and every rank commits every net of the batch, so
+// all replicas stay bitwise identical to the 1-GPU result (nets of one batch are
+// independent: reading R13).
+#include <cub/cub.cuh>
+
+#include <cstdlib>
+#include <cstring>
+
+#include "fgr_internal.cuh"
+
+namespace {
+
+__global__ void k_classify(int count, const int32_t* __restrict__ ids, const int32_t* __restrict__ off,
+                           int32_t* __restrict__ out, int* __restrict__ ctr /* [0] large, [1] small, [2] maxm */) {
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= count) return;
+    const int id = ids[i];
+    const int m = off[id + 1] - off[id];
+    if (m > FGR_SMALL_NET) {
+        out[atomicAdd(&ctr[0], 1)] = id;
+        atomicMax(&ctr[2], m);
+    } else {
+        out[count - 1 - atomicAdd(&ctr[1], 1)] = id;
+    }
+}
+
+__global__ void k_net_sizes(int n, const int32_t* __restrict__ order, const int32_t* __restrict__ off,
+                            int32_t* __restrict__ sizes) {
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i < n) sizes[i] = off[order[i] + 1] - off[order[i]];
+}
+
+__global__ void k_batch_info(int B, const int32_t* __restrict__ boff, const int32_t* __restrict__ order,
+                             const int32_t* __restrict__ off, const int16_t* __restrict__ x,
+                             const int16_t* __restrict__ y, const int32_t* __restrict__ par,
+                             int* __restrict__ nlarge, int* __restrict__ maxm, unsigned long long* __restrict__ segb) {
+    // one block per batch
+    const int b = blockIdx.x;
+    if (b >= B) return;
+    int nl = 0, mm = 0;
+    unsigned long long sb = 0;
+    for (int i = boff[b] + threadIdx.x; i < boff[b + 1]; i += blockDim.x) {
+        const int id = order[i];
+        const int a0 = off[id], m = off[id + 1] - a0;
+        if (m > FGR_SMALL_NET) { nl++; mm = max(mm, m); }
+        for (int j = 1; j < m; j++) {
+            const int u = a0 + par[a0 + j];
+            sb += (unsigned)((abs(x[a0 + j] - x[u]) >> 5) + (abs(y[a0 + j] - y[u]) >> 5) + 4);
+        }
+    }
+    atomicAdd(&nlarge[b], nl);
+    atomicMax(&maxm[b], mm);
+    atomicAdd(&segb[b], sb);
+}
+
+__global__ void k_scatter_records(int n, const int32_t* __restrict__ order, const int32_t* __restrict__ off,
+                                  const int32_t* __restrict__ rec_off, const uint32_t* __restrict__ rec_seg,
+                                  const uint32_t* __restrict__ rec_cost, uint32_t* __restrict__ seg_out,
+                                  uint32_t* __restrict__ cost_out) {
+    const int warp = (int)((blockIdx.x * (size_t)blockDim.x + threadIdx.x) >> 5);
+    if (warp >= n) return;
+    const int id = order[warp];
+    const int a0 = off[id], m = off[id + 1] - a0;
+    for (int j = lane_id(); j < m; j += 32) seg_out[a0 + j] = rec_seg[rec_off[warp] + j];
+    if (lane_id() == 0) cost_out[id] = rec_cost[warp];
+}
+
+bool nets_equal(const fgr_nets& a, const fgr_nets& b) {
+    return a.num_nets == b.num_nets && a.num_nodes == b.num_nodes && a.node_offset == b.node_offset && a.x == b.x &&
+           a.y == b.y && a.pin_lo == b.pin_lo && a.pin_hi == b.pin_hi && a.parent == b.parent;
+}
+
+}  // namespace
+
+// Refresh before a DP launch: a full rescan after set_demand/creation, else only
+// the segments the last commit dirtied (bounded by `max_tasks`).
+static cudaError_t refresh_before_dp(fgr_grid* g, cudaStream_t st, long long max_tasks) {
+    if (g->full_dirty) {
+        cudaError_t e = cudaMemsetAsync(g->d_count, 0, 2 * sizeof(int32_t), st);
+        if (e != cudaSuccess) return e;
+        g->full_dirty = false;
+        return fgr_launch_refresh_sized(g, st, true, 0);
+    }
+    return fgr_launch_refresh_sized(g, st, false, max_tasks);
+}
+
+extern "C" FGR_API fgr_status fgr_route_batch(fgr_grid* g, const fgr_nets* nets, const int32_t* net_ids, int32_t count,
+                                              uint32_t* seg_out, uint32_t* net_cost, void* stream) {
+    if (!g || !nets) return fgr_set_error(FGR_ERR_INVALID, "NULL argument");
+    if (g->broken) return fgr_set_error(FGR_ERR_STATE, "grid unusable after an earlier CUDA/NCCL error");
+    if (count < 0) return fgr_set_error(FGR_ERR_INVALID, "count < 0");
+    if (count == 0) return FGR_OK;
+    if (!net_ids || !seg_out || !net_cost) return fgr_set_error(FGR_ERR_INVALID, "NULL array");
+    cudaStream_t st = (cudaStream_t)stream;
+    FGR_CHECK_CUDA(g, cudaSetDevice(g->device));
+    cudaError_t e;
+    int32_t* list = (int32_t*)fgr_scratch(g->s_rec[0], sizeof(int32_t) * (size_t)count + 64, &e);
+    if (e != cudaSuccess) return fgr_cuda_fail(g, e, "route_batch scratch");
+    int* ctr = (int*)(list + count);
+    FGR_CHECK_CUDA(g, cudaMemsetAsync(ctr, 0, 4 * sizeof(int), st));
+    k_classify<<<(count + 255) / 256, 256, 0, st>>>(count, net_ids, nets->node_offset, list, ctr);
+    FGR_CHECK_CUDA(g, cudaGetLastError());
+    int hc[4];
+    FGR_CHECK_CUDA(g, cudaMemcpyAsync(hc, ctr, sizeof(hc), cudaMemcpyDeviceToHost, st));
+    FGR_CHECK_CUDA(g, cudaStreamSynchronize(st));
+    FGR_CHECK_CUDA(g, refresh_before_dp(g, st, g->total_segs));
+    const NetsView nv = fgr_nets_view(nets);
+    FGR_CHECK_CUDA(g, fgr_launch_dp(g, st, nv, list, count, hc[0], hc[2], seg_out, net_cost, nullptr, nullptr,
+                                    nullptr, 0, true));
+    fgr_flip_lists(g);
+    return FGR_OK;
+}
+
+// Host mirrors of per-batch launch sizes: from fgr_plan's cache, or rebuilt (one sync).
+static fgr_status batch_info(fgr_grid* g, const fgr_nets* nets, const int32_t* order, const int32_t* batch_offset,
+                             int B, cudaStream_t st) {
+    PlanCache& c = g->cache;
+    if (c.valid && c.num_batches == B && c.order == order && c.batch_offset == batch_offset &&
+        nets_equal(c.nets, *nets))
+        return FGR_OK;
+    cudaError_t e;
+    void* p = fgr_scratch(g->s_rec[1], (size_t)B * 16 + 64, &e);
+    if (e != cudaSuccess) return fgr_cuda_fail(g, e, "batch info scratch");
+    unsigned long long* d_segb = (unsigned long long*)p;
+    int* d_nl = (int*)(d_segb + B);
+    int* d_mm = d_nl + B;
+    FGR_CHECK_CUDA(g, cudaMemsetAsync(p, 0, (size_t)B * 16, st));
+    if (B > 0) {
+        k_batch_info<<<B, 256, 0, st>>>(B, batch_offset, order, nets->node_offset, nets->x, nets->y, nets->parent,
+                                        d_nl, d_mm, d_segb);
+        FGR_CHECK_CUDA(g, cudaGetLastError());
+    }
+    if (c.cap < B + 1) {
+        free(c.h_off); free(c.h_nlarge); free(c.h_maxm); free(c.h_segb);
+        c.cap = B + 1;
+        c.h_off = (int*)malloc(sizeof(int) * c.cap);
+        c.h_nlarge = (int*)malloc(sizeof(int) * c.cap);
+        c.h_maxm = (int*)malloc(sizeof(int) * c.cap);
+        c.h_segb = (long long*)malloc(sizeof(long long) * c.cap);
+    }
+    FGR_CHECK_CUDA(g, cudaMemcpyAsync(c.h_off, batch_offset, sizeof(int) * (B + 1), cudaMemcpyDeviceToHost, st));
+    if (B > 0) {
+        FGR_CHECK_CUDA(g, cudaMemcpyAsync(c.h_nlarge, d_nl, sizeof(int) * B, cudaMemcpyDeviceToHost, st));
+        FGR_CHECK_CUDA(g, cudaMemcpyAsync(c.h_maxm, d_mm, sizeof(int) * B, cudaMemcpyDeviceToHost, st));
+        FGR_CHECK_CUDA(g, cudaMemcpyAsync(c.h_segb, d_segb, sizeof(long long) * B, cudaMemcpyDeviceToHost, st));
+    }
+    FGR_CHECK_CUDA(g, cudaStreamSynchronize(st));
+    c.valid = true;
+    c.nets = *nets;
+    c.order = order;
+    c.batch_offset = batch_offset;
+    c.num_batches = B;
+    return FGR_OK;
+}
+
+extern "C" FGR_API fgr_status fgr_route_all(fgr_grid* g, const fgr_nets* nets, const int32_t* order,
+                                            const int32_t* batch_offset, int32_t num_batches, uint32_t* seg_out,
+                                            uint32_t* net_cost, void* stream) {
+    if (!g || !nets) return fgr_set_error(FGR_ERR_INVALID, "NULL argument");
+    if (g->broken) return fgr_set_error(FGR_ERR_STATE, "grid unusable after an earlier CUDA/NCCL error");
+    const int B = num_batches, N = nets->num_nets, M = nets->num_nodes;
+    if (B < 0 || N < 0 || M < 0) return fgr_set_error(FGR_ERR_INVALID, "negative sizes");
+    if (N > 0 && (!order || !batch_offset || !seg_out || !net_cost))
+        return fgr_set_error(FGR_ERR_INVALID, "NULL array");
+    cudaStream_t st = (cudaStream_t)stream;
+    FGR_CHECK_CUDA(g, cudaSetDevice(g->device));
+    fgr_status s = batch_info(g, nets, order, batch_offset, B, st);
+    if (s != FGR_OK) return s;
+    const PlanCache& c = g->cache;
+    if (M > 0) FGR_CHECK_CUDA(g, cudaMemsetAsync(seg_out, 0xFF, sizeof(uint32_t) * (size_t)M, st));
+    if (N > 0) FGR_CHECK_CUDA(g, cudaMemsetAsync(net_cost, 0, sizeof(uint32_t) * (size_t)N, st));
+    const NetsView nv = fgr_nets_view(nets);
+    g->stats.num_batches = B;
+    g->stats.world = g->world;
+    g->stats.rank = g->rank;
+    g->stats.dp_nets = B > 0 ? c.h_off[B] : 0;
+    g->stats.kernel_launches = 0;
+    FGR_CHECK_CUDA(g, cudaMemsetAsync(g->d_stats, 0, 4 * sizeof(unsigned long long), st));
+    if (g->world <= 1) {
+        for (int b = 0; b < B; b++) {
+            const long long bound = b > 0 ? c.h_segb[b - 1] : (long long)g->total_segs;
+            FGR_CHECK_CUDA(g, refresh_before_dp(g, st, bound));
+            const int o0 = c.h_off[b], cnt = c.h_off[b + 1] - o0;
+            FGR_CHECK_CUDA(g, fgr_launch_dp(g, st, nv, order + o0, cnt, c.h_nlarge[b], c.h_maxm[b], seg_out,
+                                            net_cost, nullptr, nullptr, nullptr, 0, true));
+            fgr_flip_lists(g);
+        }
+        return FGR_OK;
+    }
+    // ---- multi-GPU: split each batch, exchange route records, commit everywhere
+    if (!g->comm) return fgr_set_error(FGR_ERR_STATE, "world > 1 without a communicator");
+    cudaError_t e;
+    const int R = B > 0 ? c.h_off[B] : 0;
+    int32_t* rec_off = (int32_t*)fgr_scratch(g->s_rec[2], sizeof(int32_t) * ((size_t)R + 1) * 2 + 64, &e);
+    if (e != cudaSuccess) return fgr_cuda_fail(g, e, "record offsets");
+    int32_t* sizes = rec_off + R + 1;
+    if (R > 0) {
+        k_net_sizes<<<(R + 255) / 256, 256, 0, st>>>(R, order, nets->node_offset, sizes);
+        FGR_CHECK_CUDA(g, cudaGetLastError());
+    }
+    FGR_CHECK_CUDA(g, cudaMemsetAsync(sizes + R, 0, sizeof(int32_t), st));
+    size_t tb = 0;
+    cub::DeviceScan::ExclusiveSum(nullptr, tb, sizes, rec_off, R + 1, st);
+    void* tmp = fgr_scratch(g->s_plan[8], tb, &e);
+    if (e != cudaSuccess) return fgr_cuda_fail(g, e, "scan scratch");
+    FGR_CHECK_CUDA(g, cub::DeviceScan::ExclusiveSum(tmp, tb, sizes, rec_off, R + 1, st));
+    int* h_roff = (int*)malloc(sizeof(int) * (B + 1));
+    for (int b = 0; b <= B; b++)
+        FGR_CHECK_CUDA(g, cudaMemcpyAsync(h_roff + b, rec_off + c.h_off[b], sizeof(int), cudaMemcpyDeviceToHost, st));
+    FGR_CHECK_CUDA(g, cudaStreamSynchronize(st));
+    const size_t nrec = (size_t)h_roff[B];
+    uint32_t* rec = (uint32_t*)fgr_scratch(g->s_rec[3], sizeof(uint32_t) * (nrec + (size_t)R + 1), &e);
+    if (e != cudaSuccess) { free(h_roff); return fgr_cuda_fail(g, e, "records"); }
+    uint32_t* rec_cost = rec + nrec;
+    FGR_CHECK_CUDA(g, cudaMemsetAsync(rec, 0, sizeof(uint32_t) * (nrec + (size_t)R + 1), st));
+    fgr_status rs = FGR_OK;
+    for (int b = 0; b < B && rs == FGR_OK; b++) {
+        const long long bound = b > 0 ? c.h_segb[b - 1] : (long long)g->total_segs;
+        cudaError_t ce = refresh_before_dp(g, st, bound);
+        if (ce != cudaSuccess) { rs = fgr_cuda_fail(g, ce, "refresh"); break; }
+        const int o0 = c.h_off[b], cnt = c.h_off[b + 1] - o0, nl = c.h_nlarge[b], ns = cnt - nl;
+        // contiguous chunks of the large and of the small nets per rank
+        const int l0 = (int)((long long)nl * g->rank / g->world), l1 = (int)((long long)nl * (g->rank + 1) / g->world);
+        const int s0 = (int)((long long)ns * g->rank / g->world), s1 = (int)((long long)ns * (g->rank + 1) / g->world);
+        if (l1 > l0)
+            ce = fgr_launch_dp(g, st, nv, order + o0 + l0, l1 - l0, l1 - l0, c.h_maxm[b], nullptr, nullptr, rec,
+                               rec_off, rec_cost, o0 + l0, false);
+        if (ce == cudaSuccess && s1 > s0)
+            ce = fgr_launch_dp(g, st, nv, order + o0 + nl + s0, s1 - s0, 0, 0, nullptr, nullptr, rec, rec_off,
+                               rec_cost, o0 + nl + s0, false);
+        if (ce != cudaSuccess) { rs = fgr_cuda_fail(g, ce, "dp"); break; }
+        ncclResult_t nr = ncclGroupStart();
+        if (nr == ncclSuccess)
+            nr = ncclAllReduce(rec + h_roff[b], rec + h_roff[b], (size_t)(h_roff[b + 1] - h_roff[b]), ncclUint32,
+                               ncclSum, g->comm, st);
+        if (nr == ncclSuccess)
+            nr = ncclAllReduce(rec_cost + o0, rec_cost + o0, (size_t)cnt, ncclUint32, ncclSum, g->comm, st);
+        ncclResult_t ne = ncclGroupEnd();
+        if (nr != ncclSuccess || ne != ncclSuccess) {
+            g->broken = true;
+            rs = fgr_set_error(FGR_ERR_NCCL, "NCCL all-reduce failed: %s", ncclGetErrorString(nr != ncclSuccess ? nr : ne));
+            break;
+        }
+        ce = fgr_launch_commit(g, st, nv, order + o0, cnt, rec, rec_off, o0);
+        if (ce != cudaSuccess) { rs = fgr_cuda_fail(g, ce, "commit"); break; }
+        fgr_flip_lists(g);
+    }
+    free(h_roff);
+    if (rs != FGR_OK) return rs;
+    if (R > 0) {
+        k_scatter_records<<<(unsigned)(((size_t)R * 32 + 255) / 256), 256, 0, st>>>(R, order, nets->node_offset,
+                                                                                     rec_off, rec, rec_cost, seg_out,
+                                                                                     net_cost);
+        FGR_CHECK_CUDA(g, cudaGetLastError());
+    }
+    return FGR_OK;
+}
+
+extern "C" FGR_API fgr_status fgr_comm_unique_id(void* out128) {
+    if (!out128) return fgr_set_error(FGR_ERR_INVALID, "out is NULL");
+    ncclUniqueId id;
+    ncclResult_t r = ncclGetUniqueId(&id);
+    if (r != ncclSuccess) return fgr_set_error(FGR_ERR_NCCL, "ncclGetUniqueId: %s", ncclGetErrorString(r));
+    static_assert(sizeof(ncclUniqueId) == 128, "NCCL unique id is 128 bytes");
+    memcpy(out128, &id, 128);
+    return FGR_OK;
+}
+
+extern "C" FGR_API fgr_status fgr_comm_init(fgr_grid* g, const void* uid, int rank, int world) {
+    if (!g || !uid) return fgr_set_error(FGR_ERR_INVALID, "NULL argument");
+    if (world < 1 || rank < 0 || rank >= world) return fgr_set_error(FGR_ERR_INVALID, "bad rank/world %d/%d", rank, world);
+    if (g->broken) return fgr_set_error(FGR_ERR_STATE, "grid unusable after an earlier CUDA/NCCL error");
+    FGR_CHECK_CUDA(g, cudaSetDevice(g->device));
+    if (g->comm) { ncclCommDestroy(g->comm); g->comm = nullptr; }
+    ncclUniqueId id;
+    memcpy(&id, uid, sizeof(id));
+    ncclResult_t r = ncclCommInitRank(&g->comm, world, id, rank);
+    if (r != ncclSuccess) { g->comm = nullptr; return fgr_set_error(FGR_ERR_NCCL, "ncclCommInitRank: %s", ncclGetErrorString(r)); }
+    g->rank = rank;
+    g->world = world;
+    return FGR_OK;
+}
+
+extern "C" FGR_API fgr_status fgr_run_host(fgr_grid* g, int32_t N, int32_t M, const int32_t* h_off, const int16_t* h_x,
+                                           const int16_t* h_y, const int8_t* h_plo, const int8_t* h_phi,
+                                           const int32_t* h_par, uint32_t* h_seg, uint32_t* h_cost,
+                                           int32_t* h_nb, void* stream) {
+    if (!g) return fgr_set_error(FGR_ERR_INVALID, "grid is NULL");
+    if (g->broken) return fgr_set_error(FGR_ERR_STATE, "grid unusable after an earlier CUDA/NCCL error");
+    if (N < 0 || M < 0 || (N > 0 && (!h_off || !h_x || !h_y || !h_plo || !h_phi || !h_par)))
+        return fgr_set_error(FGR_ERR_INVALID, "bad host arrays");
+    cudaStream_t st = (cudaStream_t)stream;
+    FGR_CHECK_CUDA(g, cudaSetDevice(g->device));
+    // one device slab: off | par | seg | x | y | plo | phi | cost | batch | order | boff
+    const size_t bytes = 4 * ((size_t)N + 1) + 4 * (size_t)M + 4 * (size_t)M + 2 * (size_t)M + 2 * (size_t)M + M + M +
+                         4 * (size_t)N + 4 * (size_t)N + 4 * (size_t)N + 4 * ((size_t)N + 1) + 256;
+    cudaError_t e;
+    char* p = (char*)fgr_scratch(g->s_rec[0], bytes + 64, &e);
+    if (e != cudaSuccess) return fgr_cuda_fail(g, e, "run_host buffers");
+    int32_t* d_off = (int32_t*)p; p += 4 * ((size_t)N + 1);
+    int32_t* d_par = (int32_t*)p; p += 4 * (size_t)M;
+    uint32_t* d_seg = (uint32_t*)p; p += 4 * (size_t)M;
+    int32_t* d_bat = (int32_t*)p; p += 4 * (size_t)N;
+    int32_t* d_ord = (int32_t*)p; p += 4 * (size_t)N;
+    int32_t* d_boff = (int32_t*)p; p += 4 * ((size_t)N + 1);
+    uint32_t* d_cost = (uint32_t*)p; p += 4 * (size_t)N;
+    int16_t* d_x = (int16_t*)p; p += 2 * (size_t)M;
+    int16_t* d_y = (int16_t*)p; p += 2 * (size_t)M;
+    int8_t* d_plo = (int8_t*)p; p += M;
+    int8_t* d_phi = (int8_t*)p;
+    FGR_CHECK_CUDA(g, cudaMemcpyAsync(d_off, h_off, 4 * ((size_t)N + 1), cudaMemcpyHostToDevice, st));
+    if (M > 0) {
+        FGR_CHECK_CUDA(g, cudaMemcpyAsync(d_par, h_par, 4 * (size_t)M, cudaMemcpyHostToDevice, st));
+        FGR_CHECK_CUDA(g, cudaMemcpyAsync(d_x, h_x, 2 * (size_t)M, cudaMemcpyHostToDevice, st));
+        FGR_CHECK_CUDA(g, cudaMemcpyAsync(d_y, h_y, 2 * (size_t)M, cudaMemcpyHostToDevice, st));
+        FGR_CHECK_CUDA(g, cudaMemcpyAsync(d_plo, h_plo, (size_t)M, cudaMemcpyHostToDevice, st));
+        FGR_CHECK_CUDA(g, cudaMemcpyAsync(d_phi, h_phi, (size_t)M, cudaMemcpyHostToDevice, st));
+    }
+    fgr_nets n;
+    n.num_nets = N; n.num_nodes = M; n.node_offset = d_off; n.x = d_x; n.y = d_y; n.pin_lo = d_plo; n.pin_hi = d_phi;
+    n.parent = d_par;
+    fgr_status s = fgr_grid_set_demand(g, nullptr, stream);
+    if (s != FGR_OK) return s;
+    int32_t B = 0;
+    s = fgr_plan(g, &n, d_bat, d_ord, d_boff, &B, stream);
+    if (s != FGR_OK) return s;
+    s = fgr_route_all(g, &n, d_ord, d_boff, B, d_seg, d_cost, stream);
+    if (s != FGR_OK) return s;
+    if (h_seg && M > 0) FGR_CHECK_CUDA(g, cudaMemcpyAsync(h_seg, d_seg, 4 * (size_t)M, cudaMemcpyDeviceToHost, st));
+    if (h_cost && N > 0) FGR_CHECK_CUDA(g, cudaMemcpyAsync(h_cost, d_cost, 4 * (size_t)N, cudaMemcpyDeviceToHost, st));
+    FGR_CHECK_CUDA(g, cudaStreamSynchronize(st));
+    if (h_nb) *h_nb = B;
+    return FGR_OK;
+}

@@ -1,0 +1,272 @@
+"""Thin ctypes binding of libfastgr (include/fastgr.h): argument marshalling only.
+
+Every step of the path runs in the library's CUDA kernels; this module only
+packs structs, passes device pointers (torch tensors are used for device memory
+and streams) and turns status codes into exceptions.  There is no CPU fallback:
+importing works without a GPU (so the ABI can be checked on CPU), but every
+compute call needs the CUDA library and a device, and fails loudly otherwise.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from typing import Optional
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libfastgr.so")
+_LIB = None
+
+FGR_OK, FGR_ERR_INVALID, FGR_ERR_RANGE, FGR_ERR_OOM, FGR_ERR_CUDA, FGR_ERR_NCCL, FGR_ERR_STATE = range(7)
+STATUS_NAMES = ["OK", "INVALID", "RANGE", "OOM", "CUDA", "NCCL", "STATE"]
+
+# every entry point include/fastgr.h declares
+EXPORTS = ["fgr_last_error", "fgr_version", "fgr_cost_table", "fgr_grid_create", "fgr_grid_destroy",
+           "fgr_grid_set_demand", "fgr_grid_get_demand", "fgr_plan", "fgr_route_batch", "fgr_route_all",
+           "fgr_comm_unique_id", "fgr_comm_init", "fgr_run_host", "fgr_get_stats"]
+
+
+class FgrError(RuntimeError):
+    def __init__(self, status, msg):
+        super().__init__(f"FGR_ERR_{STATUS_NAMES[status] if 0 <= status < 7 else status}: {msg}")
+        self.status = status
+
+
+class fgr_grid_desc(ctypes.Structure):
+    _fields_ = [("nx", ctypes.c_int32), ("ny", ctypes.c_int32), ("nlayers", ctypes.c_int32),
+                ("dir", ctypes.c_void_p), ("layer_capacity", ctypes.c_void_p), ("edge_capacity", ctypes.c_void_p),
+                ("len_cost", ctypes.c_int32), ("via_cost", ctypes.c_void_p), ("ovf_weight", ctypes.c_void_p),
+                ("logistic_slope", ctypes.c_double), ("slack_clamp", ctypes.c_int32)]
+
+
+class fgr_nets(ctypes.Structure):
+    _fields_ = [("num_nets", ctypes.c_int32), ("num_nodes", ctypes.c_int32), ("node_offset", ctypes.c_void_p),
+                ("x", ctypes.c_void_p), ("y", ctypes.c_void_p), ("pin_lo", ctypes.c_void_p),
+                ("pin_hi", ctypes.c_void_p), ("parent", ctypes.c_void_p)]
+
+
+class fgr_stats(ctypes.Structure):
+    _fields_ = [("refresh_segments", ctypes.c_int64), ("refresh_bytes", ctypes.c_int64), ("dp_nets", ctypes.c_int64),
+                ("dp_edges", ctypes.c_int64), ("kernel_launches", ctypes.c_int64), ("num_batches", ctypes.c_int32),
+                ("world", ctypes.c_int32), ("rank", ctypes.c_int32)]
+
+
+def lib():
+    """Load libfastgr.so (built in-tree by `make` / __graft_entry__.build())."""
+    global _LIB
+    if _LIB is None:
+        if not os.path.exists(LIB_PATH):
+            raise RuntimeError(f"{LIB_PATH} is missing: the CUDA extension must be built (make); "
+                               "there is no fallback path")
+        L = ctypes.CDLL(LIB_PATH, mode=ctypes.RTLD_GLOBAL)
+        P, I, S = ctypes.c_void_p, ctypes.c_int32, ctypes.c_int
+        sig = {
+            "fgr_last_error": ([], ctypes.c_char_p),
+            "fgr_version": ([], ctypes.c_char_p),
+            "fgr_cost_table": ([P, P], S),
+            "fgr_grid_create": ([P, S, P, P], S),
+            "fgr_grid_destroy": ([P], S),
+            "fgr_grid_set_demand": ([P, P, P], S),
+            "fgr_grid_get_demand": ([P, P, P], S),
+            "fgr_plan": ([P, P, P, P, P, P, P], S),
+            "fgr_route_batch": ([P, P, P, I, P, P, P], S),
+            "fgr_route_all": ([P, P, P, P, I, P, P, P], S),
+            "fgr_comm_unique_id": ([P], S),
+            "fgr_comm_init": ([P, P, S, S], S),
+            "fgr_run_host": ([P, I, I, P, P, P, P, P, P, P, P, P, P], S),
+            "fgr_get_stats": ([P, P], S),
+        }
+        for name, (args, res) in sig.items():
+            f = getattr(L, name)
+            f.argtypes, f.restype = args, res
+        _LIB = L
+    return _LIB
+
+
+def _check(status):
+    if status != FGR_OK:
+        raise FgrError(status, lib().fgr_last_error().decode())
+
+
+def _ptr(t):
+    """Device/host address of a torch tensor or numpy array (None -> NULL)."""
+    if t is None:
+        return None
+    if isinstance(t, np.ndarray):
+        return t.ctypes.data
+    return t.data_ptr()
+
+
+def _stream(stream):
+    if stream is None:
+        import torch
+        return torch.cuda.current_stream().cuda_stream
+    return stream if isinstance(stream, int) else stream.cuda_stream
+
+
+# ----------------------------------------------------------------- C names
+def fgr_version() -> str:
+    return lib().fgr_version().decode()
+
+
+def make_desc(nx, ny, nlayers, dir, layer_capacity, len_cost, via_cost, ovf_weight, logistic_slope, slack_clamp,
+              edge_capacity_dev=None):
+    keep = [np.ascontiguousarray(dir, np.uint8), np.ascontiguousarray(layer_capacity, np.int32),
+            np.ascontiguousarray(via_cost, np.int32), np.ascontiguousarray(ovf_weight, np.int32)]
+    d = fgr_grid_desc(nx, ny, nlayers, keep[0].ctypes.data, keep[1].ctypes.data, _ptr(edge_capacity_dev), len_cost,
+                      keep[2].ctypes.data, keep[3].ctypes.data, float(logistic_slope), slack_clamp)
+    d._keep = keep
+    return d
+
+
+def fgr_cost_table(desc) -> np.ndarray:
+    t = np.zeros((desc.nlayers, 2 * desc.slack_clamp + 1), np.int64)
+    _check(lib().fgr_cost_table(ctypes.byref(desc), t.ctypes.data))
+    return t
+
+
+def fgr_grid_create(desc, device=0, stream=None):
+    h = ctypes.c_void_p()
+    _check(lib().fgr_grid_create(ctypes.byref(desc), device, _stream(stream), ctypes.byref(h)))
+    return h
+
+
+def fgr_grid_destroy(h):
+    _check(lib().fgr_grid_destroy(h))
+
+
+def fgr_grid_set_demand(h, demand=None, stream=None):
+    _check(lib().fgr_grid_set_demand(h, _ptr(demand), _stream(stream)))
+
+
+def fgr_grid_get_demand(h, out, stream=None):
+    _check(lib().fgr_grid_get_demand(h, _ptr(out), _stream(stream)))
+
+
+def make_nets(num_nets, num_nodes, node_offset, x, y, pin_lo, pin_hi, parent):
+    n = fgr_nets(num_nets, num_nodes, _ptr(node_offset), _ptr(x), _ptr(y), _ptr(pin_lo), _ptr(pin_hi), _ptr(parent))
+    n._keep = (node_offset, x, y, pin_lo, pin_hi, parent)
+    return n
+
+
+def fgr_plan(h, nets, batch_of_net, order, batch_offset, stream=None) -> int:
+    nb = ctypes.c_int32(0)
+    _check(lib().fgr_plan(h, ctypes.byref(nets), _ptr(batch_of_net), _ptr(order), _ptr(batch_offset),
+                          ctypes.byref(nb), _stream(stream)))
+    return nb.value
+
+
+def fgr_route_batch(h, nets, net_ids, count, seg_out, net_cost, stream=None):
+    _check(lib().fgr_route_batch(h, ctypes.byref(nets), _ptr(net_ids), int(count), _ptr(seg_out), _ptr(net_cost),
+                                 _stream(stream)))
+
+
+def fgr_route_all(h, nets, order, batch_offset, num_batches, seg_out, net_cost, stream=None):
+    _check(lib().fgr_route_all(h, ctypes.byref(nets), _ptr(order), _ptr(batch_offset), int(num_batches),
+                               _ptr(seg_out), _ptr(net_cost), _stream(stream)))
+
+
+def fgr_comm_unique_id() -> bytes:
+    buf = ctypes.create_string_buffer(128)
+    _check(lib().fgr_comm_unique_id(buf))
+    return buf.raw
+
+
+def fgr_comm_init(h, unique_id: bytes, rank: int, world: int):
+    buf = ctypes.create_string_buffer(bytes(unique_id), 128)
+    _check(lib().fgr_comm_init(h, buf, rank, world))
+
+
+def fgr_run_host(h, node_offset, x, y, pin_lo, pin_hi, parent, seg_out=None, net_cost=None, stream=None) -> int:
+    """Host-buffer end-to-end call (numpy or pinned CPU torch tensors)."""
+    nb = ctypes.c_int32(0)
+    N = len(node_offset) - 1
+    M = len(x)
+    _check(lib().fgr_run_host(h, N, M, _ptr(node_offset), _ptr(x), _ptr(y), _ptr(pin_lo), _ptr(pin_hi),
+                              _ptr(parent), _ptr(seg_out), _ptr(net_cost), ctypes.byref(nb), _stream(stream)))
+    return nb.value
+
+
+def fgr_get_stats(h) -> dict:
+    s = fgr_stats()
+    _check(lib().fgr_get_stats(h, ctypes.byref(s)))
+    return {k: getattr(s, k) for k, _ in fgr_stats._fields_}
+
+
+# ----------------------------------------------------------------- conveniences (marshalling only)
+class Router:
+    """Owns a grid handle plus device copies of one design's nets (torch tensors)."""
+
+    def __init__(self, design, device: int = 0, stream=None):
+        import torch
+        if not torch.cuda.is_available():
+            raise RuntimeError("fastgr needs a CUDA device (no CPU fallback)")
+        self.torch = torch
+        self.dev = torch.device("cuda", device)
+        self.d = design
+        ecap = None
+        if design.edge_capacity is not None:
+            ecap = torch.from_numpy(np.ascontiguousarray(design.edge_capacity)).to(self.dev)
+        self.desc = make_desc(design.nx, design.ny, design.nlayers, design.dir, design.layer_capacity,
+                              design.len_cost, design.via_cost, design.ovf_weight, design.logistic_slope,
+                              design.slack_clamp, ecap)
+        self.h = fgr_grid_create(self.desc, device, stream)
+        torch.cuda.synchronize(self.dev)
+        self._ecap = ecap
+        t = lambda a: torch.from_numpy(np.ascontiguousarray(a)).to(self.dev)
+        self.t_off, self.t_x, self.t_y = t(design.node_offset), t(design.x), t(design.y)
+        self.t_plo, self.t_phi, self.t_par = t(design.pin_lo), t(design.pin_hi), t(design.parent)
+        self.nets = make_nets(design.num_nets, design.num_nodes, self.t_off, self.t_x, self.t_y, self.t_plo,
+                              self.t_phi, self.t_par)
+        N, M = design.num_nets, design.num_nodes
+        i32 = torch.int32
+        self.batch_of_net = torch.empty(max(N, 1), dtype=i32, device=self.dev)
+        self.order = torch.empty(max(N, 1), dtype=i32, device=self.dev)
+        self.batch_offset = torch.empty(N + 1, dtype=i32, device=self.dev)
+        self.seg = torch.empty(max(M, 1), dtype=i32, device=self.dev)
+        self.cost = torch.empty(max(N, 1), dtype=i32, device=self.dev)
+        self.num_batches = 0
+
+    def close(self):
+        if self.h:
+            fgr_grid_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def reset_demand(self, demand=None, stream=None):
+        fgr_grid_set_demand(self.h, demand, stream)
+
+    def plan(self, stream=None) -> int:
+        self.num_batches = fgr_plan(self.h, self.nets, self.batch_of_net, self.order, self.batch_offset, stream)
+        return self.num_batches
+
+    def route_all(self, stream=None):
+        fgr_route_all(self.h, self.nets, self.order, self.batch_offset, self.num_batches, self.seg, self.cost, stream)
+
+    def route_batch(self, net_ids, stream=None):
+        fgr_route_batch(self.h, self.nets, net_ids, int(net_ids.numel()), self.seg, self.cost, stream)
+
+    def demand(self, stream=None):
+        out = self.torch.empty((self.d.nlayers, self.d.ny, self.d.nx), dtype=self.torch.int32, device=self.dev)
+        fgr_grid_get_demand(self.h, out, stream)
+        return out
+
+    def run(self, stream=None):
+        """Whole stage from zero demand: set_demand(NULL) -> plan -> route_all."""
+        self.reset_demand(None, stream)
+        self.plan(stream)
+        self.route_all(stream)
+
+    def results(self):
+        """(batch_of_net, num_batches, seg uint32, cost uint32, demand) as host numpy arrays."""
+        self.torch.cuda.synchronize(self.dev)
+        N, M = self.d.num_nets, self.d.num_nodes
+        return (self.batch_of_net[:N].cpu().numpy(), self.num_batches,
+                self.seg[:M].cpu().numpy().view(np.uint32), self.cost[:N].cpu().numpy().view(np.uint32),
+                self.demand().cpu().numpy())
