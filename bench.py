@@ -1,0 +1,340 @@
+#!/usr/bin/env python
+"""bench.py — device-timed nets/s of the pattern-routing stage (BASELINE.json metric).
+
+A step = one pass of the whole hot path over one design: demand reset ->
+fgr_plan (S0-S2: validate, sort, conflict-free batching) -> fgr_route_all (per
+batch: S3 cost refresh, S4-S6 tree DP + backtrack + commit).  Inputs are resident
+in HBM before the timed region; L2 is flushed (256 MiB write) between steps,
+outside each step's event pair.  `value` = nets routed (>= 1 tree edge) / step
+time, max over ranks.  `e2e` = the same metric through fgr_run_host (host
+buffers in, routes out, copies inside the timed region).
+
+Usage: python bench.py [--gpus N] [--steps K] [--warmup W] [--config t9] [--impl ours|reference]
+Multi-GPU: torchrun --nproc-per-node N bench.py --gpus N (one process per GPU).
+"""
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import gen  # noqa: E402
+
+METRIC = "nets/sec for pattern routing (device-timed, max over ranks), % HBM roofline"
+WORKLOADS = {
+    "tiny": "tiny synthetic: 64x64 GCell grid, 5 layers, 200 nets of 2-6 pins",
+    "t1": "ISPD18-test1-shaped synthetic: 3000 nets, 9 layers, 200x200 GCells",
+    "t5": "ISPD18-test5-shaped synthetic: 72000 nets, 9 layers, 300x300 GCells, congested core",
+    "t9": "ISPD19-test9-shaped synthetic: 900000 nets, 9 layers, 900x900 GCells",
+    "scale": "scaling synthetic: 2M nets, 9 layers, 2000x2000 GCells",
+}
+
+
+def peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            p = json.load(f)
+        return float(p["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def design_stats(d):
+    """Per-design algorithmic quantities (independent of the routes chosen)."""
+    sizes = d.net_sizes()
+    routed = sizes >= 2
+    par = d.parent.astype(np.int64)
+    nid = np.repeat(np.arange(d.num_nets), sizes)
+    off = d.node_offset[:-1].astype(np.int64)[nid]
+    child = par >= 0
+    pidx = off[child] + par[child]
+    dx = np.abs(d.x[child].astype(np.int64) - d.x[pidx].astype(np.int64))
+    dy = np.abs(d.y[child].astype(np.int64) - d.y[pidx].astype(np.int64))
+    large_node = (sizes > 32)[nid][child]
+    E = int(child.sum())
+    WL = int((dx + dy).sum())
+    return dict(nets_total=int(d.num_nets), nets_routed=int(routed.sum()), nodes=int(d.num_nodes), edges=E,
+                wirelength=WL, edges_large=int(large_node.sum()), wl_large=int((dx + dy)[large_node].sum()),
+                nodes_large=int(sizes[sizes > 32].sum()), nets_large=int((sizes > 32).sum()))
+
+
+def dp_bytes(M, E, WL, N):
+    """SURVEY.md §8(d) per-net figure: 12 B/node input + 8 gathered 32-B sectors per
+    tree edge + 4 B/edge segment out + 4 B/net cost + 8 B per committed unit edge."""
+    return 12 * M + 256 * E + 4 * E + 4 * N + 8 * WL
+
+
+class Clocks:
+    """nvidia-smi sampling of SM clocks and throttle reasons during the timed region."""
+
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.p = None
+
+    def start(self):
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
+                                       "--format=csv,noheader,nounits", "-lms", "100"],
+                                      stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except Exception:
+            self.p = None
+
+    def stop(self):
+        if self.p is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.25)
+        self.p.terminate()
+        out, _ = self.p.communicate(timeout=10)
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in out.strip().splitlines():
+            f = [x.strip() for x in line.split(",")]
+            if len(f) < 7:
+                continue
+            try:
+                sm.append(float(f[0])); mx.append(float(f[1]))
+            except ValueError:
+                continue
+            for n, v in zip(names, f[3:7]):
+                if v.lower().startswith("active"):
+                    reasons.add(n)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "samples": len(sm), "reasons": sorted(reasons)}
+
+
+def run_reference(args, rank):
+    """The reference arm: the plain CPU oracle timed on the host cores, on bounded samples."""
+    if rank != 0:
+        return
+    from oracle import Oracle
+    d = gen.make_config(args.config)
+    frac = args.ref_fraction
+    rng = np.random.default_rng(1234)
+    n_sample = max(1, int(d.num_nets * frac))
+    times, routed = [], 0
+    for k in range(args.warmup + args.steps):
+        ids = np.sort(rng.choice(d.num_nets, n_sample, replace=False))
+        s = d.subset(ids)
+        o = Oracle(s)
+        t0 = time.perf_counter()
+        b, nb = o.plan()
+        o.route(b, nb)
+        t = time.perf_counter() - t0
+        if k >= args.warmup:
+            times.append(t)
+            routed = int((s.net_sizes() >= 2).sum())
+    ms = 1000 * statistics.mean(times)
+    val = routed / (ms / 1000)
+    sample = f"{n_sample} random nets ({frac:.0%}) of {args.config} per step, full grid, single thread"
+    line = {"metric": METRIC, "value": val, "unit": "nets/s", "n_gpus": args.gpus, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "int64", "data": "synthetic", "impl": "reference",
+            "config": {"workload": WORKLOADS[args.config], "sample": sample},
+            "cpu_baseline": {"value": val, "unit": "nets/s", "cores": 1, "kind": "oracle", "sample": sample},
+            "e2e": {"value": val, "unit": "nets/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def cpu_baseline(d, config, budget_s=20.0):
+    """The oracle as it stands, on this host, single thread: whole design if it fits the budget."""
+    from oracle import Oracle
+    o = Oracle(d)
+    t0 = time.perf_counter()
+    b, nb = o.plan()
+    o.route(b, nb)
+    t = time.perf_counter() - t0
+    routed = int((d.net_sizes() >= 2).sum())
+    return {"value": routed / t, "unit": "nets/s", "cores": 1, "kind": "oracle",
+            "sample": f"the whole {config} design ({d.num_nets} nets), plan + route, one run",
+            "seconds": t, "cpu": _cpu_model()}
+
+
+def _cpu_model():
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip() + f" ({os.cpu_count()} cpus)"
+    except Exception:
+        pass
+    return None
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="t9", choices=sorted(WORKLOADS))
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--ref-fraction", type=float, default=0.25)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    args = ap.parse_args()
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        run_reference(args, rank)
+        return
+
+    import torch
+    import torch.distributed as dist
+    from paper_conf_date_liulzclly22_b200 import fastgr as F
+    from paper_conf_date_liulzclly22_b200 import Router
+
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = torch.device("cuda", local)
+    d = gen.make_config(args.config)
+    ds = design_stats(d)
+    r = Router(d, device=local)
+    if world > 1:
+        uid = [F.fgr_comm_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(uid, src=0)
+        F.fgr_comm_init(r.h, uid[0], rank, world)
+    stream = torch.cuda.current_stream(dev)
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+
+    def step():
+        r.reset_demand(None)
+        r.plan()
+        mid.record(stream)
+        r.route_all()
+
+    for _ in range(args.warmup):
+        mid = torch.cuda.Event(enable_timing=True)
+        step()
+    torch.cuda.synchronize(dev)
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize(dev)
+
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True),
+            torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    clocks = Clocks(local)
+    clocks.start()
+    F.fgr_profile_enable(r.h, True)
+    barrier()
+    t_wall = time.perf_counter()
+    for k in range(args.steps):
+        flush.zero_()
+        a, mid, b = evs[k]
+        a.record(stream)
+        step()
+        b.record(stream)
+    barrier()
+    t_wall = time.perf_counter() - t_wall
+    prof = F.fgr_profile_read(r.h)
+    F.fgr_profile_enable(r.h, False)
+    clk = clocks.stop()
+    step_ms = [a.elapsed_time(b) for a, _, b in evs]
+    plan_ms = [a.elapsed_time(m) for a, m, _ in evs]
+    route_ms = [m.elapsed_time(b) for _, m, b in evs]
+    total = torch.tensor([sum(step_ms)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(total, op=dist.ReduceOp.MAX)
+    ms_per_step = float(total.item()) / args.steps
+    stats = F.fgr_get_stats(r.h)
+    value = ds["nets_routed"] / (ms_per_step / 1000.0)
+
+    # dominant kernel and its roofline (live CUDA-event durations over the timed region)
+    peak, peak_src = peaks()
+    launches_total = sum(n for _, n in prof.values())
+    dom = max(prof, key=lambda c: prof[c][0])
+    dom_ms, dom_n = prof[dom]
+    steps = args.steps
+    if dom in ("dp_small", "dp_large"):
+        if dom == "dp_small":
+            M = ds["nodes"] - ds["nodes_large"]; E = ds["edges"] - ds["edges_large"]
+            WL = ds["wirelength"] - ds["wl_large"]; N = ds["nets_routed"] - ds["nets_large"]
+        else:
+            M, E, WL, N = ds["nodes_large"], ds["edges_large"], ds["wl_large"], ds["nets_large"]
+        alg_bytes_step = dp_bytes(M, E, WL, N) / world
+        unit_note = "SURVEY §8(d): 12 B/node + 256 B/edge + 4 B/edge + 4 B/net + 8 B/unit edge"
+    elif dom == "refresh":
+        alg_bytes_step = stats["refresh_bytes"]  # counted during the timed region (refresh_bytes per step below)
+        unit_note = "per refreshed 32-position segment: 32 x 9 x W bytes (int32 demand + uint8 cap + uint32 prefix)"
+    else:
+        alg_bytes_step = None
+        unit_note = "no byte model for this class"
+    roof = None
+    if alg_bytes_step is not None and dom_n > 0:
+        per_launch = alg_bytes_step * steps / dom_n
+        avg_s = dom_ms / dom_n / 1000.0
+        ach = per_launch / avg_s / 1e9
+        roof = {"bound": "hbm", "kernel": dom, "achieved": ach, "peak": peak, "unit": "GB/s", "frac": ach / peak,
+                "traffic": None, "bytes_per_launch": per_launch, "avg_launch_us": avg_s * 1e6,
+                "launches_per_step": dom_n / steps, "share_of_step": dom_ms / steps / ms_per_step,
+                "peak_source": peak_src, "byte_model": unit_note}
+
+    # e2e through the public C ABI with host buffers (pinned), copies inside the timed region
+    e2e = None
+    if not args.no_e2e and world == 1:
+        pin = lambda a: torch.from_numpy(np.ascontiguousarray(a)).pin_memory()
+        h = [pin(d.node_offset), pin(d.x), pin(d.y), pin(d.pin_lo), pin(d.pin_hi), pin(d.parent)]
+        seg_h = torch.empty(d.num_nodes, dtype=torch.int32).pin_memory()
+        cost_h = torch.empty(d.num_nets, dtype=torch.int32).pin_memory()
+        h2d = sum(t.numel() * t.element_size() for t in h)
+        d2h = seg_h.numel() * 4 + cost_h.numel() * 4
+        for _ in range(max(1, args.warmup)):
+            F.fgr_run_host(r.h, *h, seg_out=seg_h, net_cost=cost_h)
+        times = []
+        for _ in range(max(3, min(args.steps, 5))):
+            flush.zero_()
+            a = torch.cuda.Event(enable_timing=True); b = torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            F.fgr_run_host(r.h, *h, seg_out=seg_h, net_cost=cost_h)
+            b.record(stream)
+            b.synchronize()
+            times.append(a.elapsed_time(b))
+        e2e_ms = statistics.mean(times)
+        e2e = {"value": ds["nets_routed"] / (e2e_ms / 1000.0), "unit": "nets/s", "ms_per_step": e2e_ms,
+               "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h),
+               "call": "fgr_run_host (pinned host nets in -> plan -> route_all -> seg/cost out)"}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cpu = cpu_baseline(d, args.config)
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": "nets/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "int32", "data": "synthetic",
+            "config": {"workload": WORKLOADS[args.config], "name": args.config, "seed": d.seed,
+                       "nets_total": ds["nets_total"], "nets_routed": ds["nets_routed"], "nodes": ds["nodes"],
+                       "tree_edges": ds["edges"], "batches": r.num_batches,
+                       "l2": "flushed between steps (256 MiB write, outside the step events)",
+                       "parallelism": f"grid replicated, batches split over {world} rank(s)"},
+            "plan_ms": statistics.mean(plan_ms), "route_ms": statistics.mean(route_ms),
+            "clocks": clk, "e2e": e2e, "gpu_launches": int(launches_total // max(1, steps)),
+            "gpu_launches_note": "library kernels per step (CUB sort kernels counted as one launch each call)",
+            "roofline": roof, "cpu_baseline": cpu,
+            "kernels_ms_per_step": {c: v[0] / steps for c, v in prof.items() if v[1]},
+            "kernels_launches_per_step": {c: v[1] / steps for c, v in prof.items() if v[1]},
+            "refresh_segments_per_step": stats["refresh_segments"],
+            "wall_s": t_wall,
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+    r.close()
+
+
+if __name__ == "__main__":
+    main()

@@ -190,6 +190,18 @@ typedef struct {
 } fgr_stats;
 FGR_API fgr_status fgr_get_stats(fgr_grid* grid, fgr_stats* out);
 
+/*
+ * Per-kernel-class device timing (CUDA events recorded on the caller's stream
+ * around every launch of the class while enabled).  Classes:
+ *   0 refresh, 1 dp_small (warp per net), 2 dp_large (CTA per net), 3 commit,
+ *   4 plan_preprocess, 5 plan_sort (CUB), 6 plan_color, 7 plan_other, 8 exchange (NCCL)
+ * fgr_profile_read synchronises, then returns the summed milliseconds and the
+ * number of launches per class since the last enable, and clears the counters.
+ */
+#define FGR_PROF_CLASSES 9
+FGR_API fgr_status fgr_profile_enable(fgr_grid* grid, int enable);
+FGR_API fgr_status fgr_profile_read(fgr_grid* grid, double* ms /* [9] */, int64_t* launches /* [9] */);
+
 #ifdef __cplusplus
 }
 #endif

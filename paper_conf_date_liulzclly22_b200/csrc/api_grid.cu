@@ -173,7 +173,7 @@ extern "C" FGR_API fgr_status fgr_grid_create(const fgr_grid_desc* d, int device
     size_t bH = cells * g->WH, bV = cells * g->WV;
     size_t sH = (size_t)h.lines * h.nseg * g->WH, sV = (size_t)w.lines * w.nseg * g->WV;
     size_t sizes[] = {bH * 4, bV * 4, bH, bV, bH * 4, bV * 4, sH * 4, sV * 4, sH * 4, sV * 4,
-                      (size_t)g->total_segs * 4, (size_t)(g->nx + g->ny) * 4, (size_t)(g->nx + g->ny) * 4};
+                      (size_t)g->total_segs, (size_t)(g->nx + g->ny), (size_t)(g->nx + g->ny) * 4};
     size_t total = 0;
     for (size_t z : sizes) total += align256(z);
     e = cudaMalloc(&g->mem, total);
@@ -187,7 +187,7 @@ extern "C" FGR_API fgr_status fgr_grid_create(const fgr_grid_desc* d, int device
     h.P = (uint32_t*)ptrs[4]; w.P = (uint32_t*)ptrs[5];
     h.ST = (uint32_t*)ptrs[6]; w.ST = (uint32_t*)ptrs[7];
     h.SB = (uint32_t*)ptrs[8]; w.SB = (uint32_t*)ptrs[9];
-    v.dseg = (uint32_t*)ptrs[10]; v.linecnt = (uint32_t*)ptrs[11]; v.linedone = (uint32_t*)ptrs[12];
+    v.dseg = (uint8_t*)ptrs[10]; v.dline = (uint8_t*)ptrs[11]; v.linedone = (uint32_t*)ptrs[12];
     // lists, counters, table
     size_t tab = (size_t)g->L * (2 * g->S + 1);
     int32_t* htab = (int32_t*)malloc(tab * sizeof(int32_t));
@@ -196,16 +196,12 @@ extern "C" FGR_API fgr_status fgr_grid_create(const fgr_grid_desc* d, int device
             htab[(size_t)l * (2 * g->S + 1) + (k + g->S)] =
                 (int32_t)std::llround((double)g->ovf_weight[l] / (1.0 + std::exp(g->slope * (double)k)));
     bool ok = cudaMalloc(&g->d_table, tab * sizeof(int32_t)) == cudaSuccess &&
-              cudaMalloc(&g->d_list[0], (size_t)g->total_segs * 4) == cudaSuccess &&
-              cudaMalloc(&g->d_list[1], (size_t)g->total_segs * 4) == cudaSuccess &&
-              cudaMalloc(&g->d_count, 2 * sizeof(int32_t)) == cudaSuccess &&
               cudaMalloc(&g->d_stats, 4 * sizeof(unsigned long long)) == cudaSuccess;
     if (!ok) { free(htab); fgr_grid_destroy(g); return fgr_set_error(FGR_ERR_OOM, "out of device memory (grid)"); }
     v.table = g->d_table;
     v.stats = g->d_stats;
     cudaMemcpyAsync(g->d_table, htab, tab * sizeof(int32_t), cudaMemcpyHostToDevice, st);
     cudaMemsetAsync(g->mem, 0, total, st);
-    cudaMemsetAsync(g->d_count, 0, 2 * sizeof(int32_t), st);
     cudaMemsetAsync(g->d_stats, 0, 4 * sizeof(unsigned long long), st);
     int32_t hcap[FGR_MAXL];
     for (int l = 0; l < g->L; l++) hcap[l] = g->layer_capacity[l];
@@ -220,9 +216,6 @@ extern "C" FGR_API fgr_status fgr_grid_create(const fgr_grid_desc* d, int device
     free(htab);
     if (e == cudaSuccess) e = cudaGetLastError();
     if (e != cudaSuccess) { fgr_grid_destroy(g); return fgr_cuda_fail(nullptr, e, "grid init"); }
-    v.seglist = g->d_list[0];
-    v.segcount = g->d_count;
-    g->parity = 0;
     g->full_dirty = true;
     cudaDeviceGetAttribute(&g->max_smem, cudaDevAttrMaxSharedMemoryPerBlockOptin, device);
     cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, device);
@@ -237,12 +230,10 @@ extern "C" FGR_API fgr_status fgr_grid_destroy(fgr_grid* g) {
     if (g->comm) ncclCommDestroy(g->comm);
     cudaFree(g->mem);
     cudaFree(g->d_table);
-    cudaFree(g->d_list[0]);
-    cudaFree(g->d_list[1]);
-    cudaFree(g->d_count);
     cudaFree(g->d_stats);
     for (auto& s : g->s_plan) cudaFree(s.p);
     for (auto& s : g->s_rec) cudaFree(s.p);
+    for (auto e : g->prof.pool) cudaEventDestroy(e);
     free(g->cache.h_off);
     free(g->cache.h_nlarge);
     free(g->cache.h_maxm);
@@ -280,13 +271,66 @@ extern "C" FGR_API fgr_status fgr_grid_get_demand(fgr_grid* g, int32_t* demand, 
     return FGR_OK;
 }
 
+int fgr_prof_begin(fgr_grid* g, int cls, cudaStream_t st) {
+    Profiler& p = g->prof;
+    if (!p.on) return -1;
+    if (p.used * 2 + 2 > p.pool.size()) {
+        for (int i = 0; i < 256; i++) {
+            cudaEvent_t e;
+            if (cudaEventCreate(&e) != cudaSuccess) return -1;
+            p.pool.push_back(e);
+        }
+    }
+    const int slot = (int)p.used++;
+    if (p.cls.size() < p.used) p.cls.resize(p.used);
+    p.cls[slot] = cls;
+    cudaEventRecord(p.pool[2 * slot], st);
+    return slot;
+}
+
+void fgr_prof_end(fgr_grid* g, int slot, cudaStream_t st) {
+    if (slot < 0) return;
+    cudaEventRecord(g->prof.pool[2 * slot + 1], st);
+}
+
+extern "C" FGR_API fgr_status fgr_profile_enable(fgr_grid* g, int enable) {
+    if (!g) return fgr_set_error(FGR_ERR_INVALID, "grid is NULL");
+    g->prof.on = enable != 0;
+    g->prof.used = 0;
+    for (int i = 0; i < FGR_PROF_CLASSES; i++) { g->prof.ms[i] = 0; g->prof.launches[i] = 0; }
+    return FGR_OK;
+}
+
+extern "C" FGR_API fgr_status fgr_profile_read(fgr_grid* g, double* ms, int64_t* launches) {
+    if (!g || !ms || !launches) return fgr_set_error(FGR_ERR_INVALID, "NULL argument");
+    Profiler& p = g->prof;
+    FGR_CHECK_CUDA(g, cudaSetDevice(g->device));
+    for (size_t i = 0; i < p.used; i++) {
+        FGR_CHECK_CUDA(g, cudaEventSynchronize(p.pool[2 * i + 1]));
+        float t = 0;
+        FGR_CHECK_CUDA(g, cudaEventElapsedTime(&t, p.pool[2 * i], p.pool[2 * i + 1]));
+        p.ms[p.cls[i]] += t;
+        p.launches[p.cls[i]]++;
+    }
+    p.used = 0;
+    for (int i = 0; i < FGR_PROF_CLASSES; i++) {
+        ms[i] = p.ms[i];
+        launches[i] = p.launches[i];
+        p.ms[i] = 0;
+        p.launches[i] = 0;
+    }
+    return FGR_OK;
+}
+
 extern "C" FGR_API fgr_status fgr_get_stats(fgr_grid* g, fgr_stats* out) {
     if (!g || !out) return fgr_set_error(FGR_ERR_INVALID, "grid or out is NULL");
     if (g->broken) return fgr_set_error(FGR_ERR_STATE, "grid unusable after an earlier CUDA/NCCL error");
     unsigned long long hs[4];
     FGR_CHECK_CUDA(g, cudaMemcpy(hs, g->d_stats, sizeof(hs), cudaMemcpyDeviceToHost));
     *out = g->stats;
-    out->refresh_segments = (int64_t)hs[0];
-    out->refresh_bytes = (int64_t)hs[1];
+    out->refresh_segments = (int64_t)(hs[0] + hs[1]);
+    // per refreshed segment: 32 positions x (demand int32 read + capacity byte read + prefix uint32 write)
+    out->refresh_bytes = (int64_t)(hs[0] * 32ull * 9ull * (unsigned long long)g->WH +
+                                   hs[1] * 32ull * 9ull * (unsigned long long)g->WV);
     return FGR_OK;
 }

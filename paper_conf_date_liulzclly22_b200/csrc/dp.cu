@@ -13,48 +13,57 @@
 // then a top-down backtrack (S5) and the +1 demand commit of every chosen leg
 // (S6) with dirty-segment marking for the next cost refresh.
 //
-// B200 mapping: one warp per net (<= 32 nodes) or one 256-thread CTA per net
-// (larger nets); nodes are processed level by level, children before parents
-// (the DFS order of PAPER.md L320-333 generalised to a level order); all prefix
-// gathers of a net are issued up front (costs are fixed during the DP); the
-// per-node tables live in shared memory; every min-plus step is a DPX
+// B200 mapping.  The layer count LT is a template parameter (every per-layer
+// loop is unrolled exactly).  A "group" of LT lanes evaluates one node: lane l
+// owns layer l of the node's vectors (F rows, B, E — the L parallel computation
+// flows of P:L754-756).  A warp holds G = min(4, 32/LT) groups:
+//   * k_dp_group: nets with <= 32 nodes, G nets per warp, each group walking
+//     its net's nodes children-first (parent[i] < i, so descending index order);
+//   * k_dp_large: nets with > 32 nodes, one 256-thread CTA per net, level by
+//     level, 8*G nodes of a level in flight.
+// All prefix gathers of a net are issued up front (costs are fixed during the
+// DP); the per-node tables live in shared memory; each min-plus step is a DPX
 // VIADDMNMX (sat_add).  Tie-breaks follow reading R11 exactly.
 #include "fgr_internal.cuh"
 
 namespace {
 
+constexpr int kMC = FGR_SMALL_NET;          // node capacity of one group in k_dp_group
+constexpr int kGroupWarps = 4;              // warps per CTA in k_dp_group
+
+__host__ __device__ constexpr int groups_of(int LT) { return (32 / LT) < 4 ? (32 / LT) : 4; }
+__host__ __device__ inline size_t a16(size_t b) { return (b + 15) & ~(size_t)15; }
+
 struct Hdr {                  // per-block constants copied to shared memory
     uint32_t viapre[FGR_MAXL + 1];
     uint8_t dir[FGR_MAXL];
     uint8_t slot[FGR_MAXL];
-    uint8_t los[2][FGR_MAXL];
 };
 
 struct Tabs {
-    uint32_t* E;      // [m][L]  E_v(lt) = c*(v -> parent, lt)
-    uint32_t* legH;   // [m][2][nH]  0: row y_v, 1: row y_u   (x_v..x_u)
-    uint32_t* legV;   // [m][2][nV]  0: col x_v, 1: col x_u   (y_v..y_u)
-    uint32_t* cmask;  // warp path: children bitmask [32]
+    uint32_t* E;      // [m][LT]      E_v(lt) = c*(v -> parent, lt)
+    uint32_t* legH;   // [m][2][nH]   0: row y_v, 1: row y_u   (x_v..x_u)
+    uint32_t* legV;   // [m][2][nV]   0: col x_v, 1: col x_u   (y_v..y_u)
+    uint32_t* aux;    // [m]  group path: children bitmask, then pointer-jumping ancestor
     int16_t* x;
     int16_t* y;
     int16_t* par;
     uint16_t* depth;
     uint16_t* cstart; // CTA path: child CSR [m+1]
     uint16_t* clist;  // CTA path: [m]
-    uint16_t* anc;    // CTA path: pointer-jumping scratch [m]
+    uint16_t* anc;    // CTA path: pointer-jumping scratch [m], then the nodes sorted by level
+    uint16_t* lvstart;// CTA path: level CSR [m+1]
     int8_t* plo;
     int8_t* phi;
     uint8_t* span;    // chosen via span (lo << 4) | hi  (low byte of the packed (value, lo, hi) key)
-    uint8_t* recE;    // [m][L] argmin ls of E_v(lt)
-    uint8_t* recB;    // [m][L] argmin span of B_v(ls)
+    uint8_t* recE;    // [m][LT] argmin ls of E_v(lt)
+    uint8_t* recB;    // [m][LT] argmin span of B_v(ls)
 };
 
-struct WScr {          // warp-private scratch
-    uint32_t* F;      // [L][L]
-    uint32_t* B;      // [L]
+struct WScr {          // per-group scratch
+    unsigned long long* R;  // [LT][LT]  R(lo,b) = min_{hi >= b} key(lo,hi), key = F<<8 | lo<<4 | hi
+    uint32_t* B;            // [LT]
 };
-
-__host__ __device__ inline size_t a16(size_t b) { return (b + 15) & ~(size_t)15; }
 
 __host__ __device__ inline size_t tabs_bytes(int m, int L, int nH, int nV, bool cta) {
     size_t b = 0;
@@ -63,28 +72,29 @@ __host__ __device__ inline size_t tabs_bytes(int m, int L, int nH, int nV, bool 
     b += a16((size_t)m * 2 * nV * 4);
     if (!cta) b += a16((size_t)m * 4);
     b += 4 * a16((size_t)m * 2);
-    if (cta) b += a16((size_t)(m + 1) * 2) + 2 * a16((size_t)m * 2);
+    if (cta) b += 2 * a16((size_t)(m + 1) * 2) + 2 * a16((size_t)m * 2);
     b += 3 * a16((size_t)m);
     b += 2 * a16((size_t)m * L);
     return b;
 }
 
-__host__ __device__ inline size_t wscr_bytes(int L) { return a16((size_t)L * L * 4) + a16((size_t)L * 4); }
+__host__ __device__ inline size_t wscr_bytes(int L) { return a16((size_t)L * L * 8) + a16((size_t)L * 4); }
 
 __device__ inline Tabs carve_tabs(unsigned char* p, int m, int L, int nH, int nV, bool cta) {
     Tabs t;
     t.E = (uint32_t*)p; p += a16((size_t)m * L * 4);
     t.legH = (uint32_t*)p; p += a16((size_t)m * 2 * nH * 4);
     t.legV = (uint32_t*)p; p += a16((size_t)m * 2 * nV * 4);
-    t.cmask = nullptr;
-    if (!cta) { t.cmask = (uint32_t*)p; p += a16((size_t)m * 4); }
+    t.aux = nullptr;
+    if (!cta) { t.aux = (uint32_t*)p; p += a16((size_t)m * 4); }
     t.x = (int16_t*)p; p += a16((size_t)m * 2);
     t.y = (int16_t*)p; p += a16((size_t)m * 2);
     t.par = (int16_t*)p; p += a16((size_t)m * 2);
     t.depth = (uint16_t*)p; p += a16((size_t)m * 2);
-    t.cstart = t.clist = t.anc = nullptr;
+    t.cstart = t.clist = t.anc = t.lvstart = nullptr;
     if (cta) {
         t.cstart = (uint16_t*)p; p += a16((size_t)(m + 1) * 2);
+        t.lvstart = (uint16_t*)p; p += a16((size_t)(m + 1) * 2);
         t.clist = (uint16_t*)p; p += a16((size_t)m * 2);
         t.anc = (uint16_t*)p; p += a16((size_t)m * 2);
     }
@@ -98,8 +108,8 @@ __device__ inline Tabs carve_tabs(unsigned char* p, int m, int L, int nH, int nV
 
 __device__ inline WScr carve_wscr(unsigned char* p, int L) {
     WScr w;
-    w.F = (uint32_t*)p;
-    w.B = (uint32_t*)(p + a16((size_t)L * L * 4));
+    w.R = (unsigned long long*)p;
+    w.B = (uint32_t*)(p + a16((size_t)L * L * 8));
     return w;
 }
 
@@ -108,8 +118,6 @@ __device__ inline void init_hdr(Hdr* h, const GridView& g) {
     for (int i = threadIdx.x; i < FGR_MAXL; i += blockDim.x) {
         h->dir[i] = g.dir[i];
         h->slot[i] = g.slot[i];
-        h->los[0][i] = g.layer_of_slot[0][i];
-        h->los[1][i] = g.layer_of_slot[1][i];
     }
 }
 
@@ -120,6 +128,24 @@ struct Out {
     const int32_t* rec_off;
     uint32_t* rec_cost;   // record mode: rec_cost[list_base + idx]
     int list_base;
+};
+
+// Per-lane constants of the group lane that owns layer `gl`.
+template <int LT>
+struct LaneConst {
+    uint32_t vp[LT + 1];   // via prefix: V(lo,hi) = vp[hi] - vp[lo]
+    uint32_t hmask;        // layers with dir == H
+    int my_dir, my_slot;
+    __device__ __forceinline__ void load(const Hdr* h, int gl) {
+#pragma unroll
+        for (int i = 0; i <= LT; i++) vp[i] = h->viapre[i];
+        hmask = 0;
+#pragma unroll
+        for (int i = 0; i < LT; i++) hmask |= (h->dir[i] == 0 ? 1u : 0u) << i;
+        const int l = gl < LT ? gl : 0;
+        my_dir = h->dir[l];
+        my_slot = h->slot[l];
+    }
 };
 
 // ------------------------------------------------------------- leg gathers
@@ -163,159 +189,142 @@ __device__ __forceinline__ void gather_task(const GridView& g, const Tabs& t, in
     }
 }
 
-// ------------------------------------------------------------- DP steps (one warp)
-// F_v(lo,hi) for all spans (lane = lo), then B_v(ls) (lane = ls) or the root minimum.
-template <bool CTA>
-__device__ __forceinline__ void span_table(const Hdr* h, const Tabs& t, const WScr& w, int v, int L) {
-    const int lane = lane_id();
-    if (lane < L) {
-        uint32_t acc[FGR_MAXL];
-        const uint32_t vlo = h->viapre[lane];
+// ------------------------------------------------------------- DP steps (one group of LT lanes)
+// F_v(lo, hi) for the group lane lo, reduced to suffix minima R(lo, b) of the packed keys.
+template <int LT, bool CTA>
+__device__ __forceinline__ void span_rows(const LaneConst<LT>& c, const Tabs& t, const WScr& w, int v, int lo, bool act) {
+    if (!act) return;
+    uint32_t acc[LT];
 #pragma unroll
-        for (int hi = 0; hi < FGR_MAXL; hi++) acc[hi] = (hi < L && hi >= lane) ? h->viapre[hi] - vlo : FGR_INF;
-        if (CTA) {
-            const int c0 = t.cstart[v], c1 = t.cstart[v + 1];
-            for (int k = c0; k < c1; k++) {
-                const uint32_t* Ec = t.E + (size_t)t.clist[k] * L;
-                uint32_t run = FGR_INF;
+    for (int hi = 0; hi < LT; hi++) acc[hi] = hi >= lo ? c.vp[hi] - c.vp[lo] : FGR_INF;
+    auto add_child = [&](int ch) {
+        const uint32_t* Ec = t.E + (size_t)ch * LT;
+        uint32_t run = FGR_INF;
 #pragma unroll
-                for (int hi = 0; hi < FGR_MAXL; hi++)
-                    if (hi < L && hi >= lane) { run = min(run, Ec[hi]); acc[hi] = sat_add(acc[hi], run); }
-            }
-        } else {
-            uint32_t cm = t.cmask[v];
-            while (cm) {
-                const int c = __ffs(cm) - 1;
-                cm &= cm - 1;
-                const uint32_t* Ec = t.E + (size_t)c * L;
-                uint32_t run = FGR_INF;
-#pragma unroll
-                for (int hi = 0; hi < FGR_MAXL; hi++)
-                    if (hi < L && hi >= lane) { run = min(run, Ec[hi]); acc[hi] = sat_add(acc[hi], run); }
-            }
+        for (int hi = 0; hi < LT; hi++) {
+            const uint32_t e = Ec[hi];
+            if (hi >= lo) { run = min(run, e); acc[hi] = sat_add(acc[hi], run); }
         }
-#pragma unroll
-        for (int hi = 0; hi < FGR_MAXL; hi++)
-            if (hi < L && hi >= lane) w.F[lane * L + hi] = acc[hi];
+    };
+    if (CTA) {
+        const int k1 = t.cstart[v + 1];
+        for (int k = t.cstart[v]; k < k1; k++) add_child(t.clist[k]);
+    } else {
+        uint32_t cm = t.aux[v];
+        while (cm) {
+            const int ch = __ffs(cm) - 1;
+            cm &= cm - 1;
+            add_child(ch);
+        }
     }
-    __syncwarp();
+    unsigned long long run = ~0ull;
+#pragma unroll
+    for (int hi = LT - 1; hi >= 0; hi--)
+        if (hi >= lo) {
+            const unsigned long long key = ((unsigned long long)acc[hi] << 8) | (unsigned)(lo << 4) | (unsigned)hi;
+            run = key < run ? key : run;
+            w.R[lo * LT + hi] = run;
+        }
 }
 
-// Eq. (2) per ls, with the (value, lo, hi) lexicographic tie-break of R11 as one 64-bit min.
-__device__ __forceinline__ void node_table(const Tabs& t, const WScr& w, int v, int L) {
-    const int lane = lane_id();
-    if (lane < L) {
-        int a = lane, b = lane;
-        const int plo = t.plo[v], phi = t.phi[v];
-        if (plo >= 0) { a = min(a, plo); b = max(b, phi); }
-        unsigned long long best = ~0ull;
-        for (int lo = 0; lo <= a; lo++)
-            for (int hi = b; hi < L; hi++) {
-                unsigned long long key = ((unsigned long long)w.F[lo * L + hi] << 8) | (unsigned)(lo << 4) | (unsigned)hi;
-                best = key < best ? key : best;
-            }
-        w.B[lane] = (uint32_t)(best >> 8);
-        t.recB[(size_t)v * L + lane] = (uint8_t)(best & 0xFF);
-    }
-    __syncwarp();
+// Eq. (2) per ls: min over lo <= a = min(ls, pin_lo) of R(lo, b), b = max(ls, pin_hi);
+// the packed key carries the (value, lo, hi) lexicographic tie-break of R11.
+template <int LT>
+__device__ __forceinline__ void node_table(const Tabs& t, const WScr& w, int v, int ls, bool act) {
+    if (!act) return;
+    int a = ls, b = ls;
+    const int plo = t.plo[v], phi = t.phi[v];
+    if (plo >= 0) { a = min(a, plo); b = max(b, phi); }
+    unsigned long long best = ~0ull;
+#pragma unroll
+    for (int lo = 0; lo < LT; lo++)
+        if (lo <= a) {
+            const unsigned long long k = w.R[lo * LT + b];
+            best = k < best ? k : best;
+        }
+    w.B[ls] = (uint32_t)(best >> 8);
+    t.recB[(size_t)v * LT + ls] = (uint8_t)(best & 0xFF);
 }
 
 // Eqs. (1),(3),(5)-(7): E_v(lt) = min_ls [B_v(ls) + leg1(ls) + V(ls,lt) + leg2(lt)], lane = lt.
-__device__ __forceinline__ void edge_table(const Hdr* h, const Tabs& t, const WScr& w, int v, int L, int nH, int nV) {
-    const int lane = lane_id();
-    if (lane < L) {
-        const int lt = lane;
-        const int u = t.par[v];
-        const int xv = t.x[v], yv = t.y[v], xu = t.x[u], yu = t.y[u];
-        const int dlt = h->dir[lt];
-        uint32_t best = FGR_INF;
-        int bls = lt;
-        if (yv == yu || xv == xu) {               // straight: one leg on ls = lt (R7)
-            const int de = (yv == yu) ? 0 : 1;
-            if (dlt == de) {
-                const uint32_t leg = de == 0 ? t.legH[(size_t)v * 2 * nH + h->slot[lt]]
-                                             : t.legV[(size_t)v * 2 * nV + h->slot[lt]];
-                best = sat_add(w.B[lt], leg);
-            }
-        } else if (dlt == 1) {                    // bend 0: leg 1 H on row y_v, leg 2 V on col x_u
-            const uint32_t leg2 = t.legV[((size_t)v * 2 + 1) * nV + h->slot[lt]];
-            const uint32_t* l1 = t.legH + (size_t)v * 2 * nH;
-            for (int s = 0; s < nH; s++) {
-                const int ls = h->los[0][s];
-                const uint32_t via = ls < lt ? h->viapre[lt] - h->viapre[ls] : h->viapre[ls] - h->viapre[lt];
-                const uint32_t c = sat_add(sat_add(sat_add(w.B[ls], l1[s]), via), leg2);
-                if (c < best) { best = c; bls = ls; }
-            }
-        } else {                                  // bend 1: leg 1 V on col x_v, leg 2 H on row y_u
-            const uint32_t leg2 = t.legH[((size_t)v * 2 + 1) * nH + h->slot[lt]];
-            const uint32_t* l1 = t.legV + (size_t)v * 2 * nV;
-            for (int s = 0; s < nV; s++) {
-                const int ls = h->los[1][s];
-                const uint32_t via = ls < lt ? h->viapre[lt] - h->viapre[ls] : h->viapre[ls] - h->viapre[lt];
-                const uint32_t c = sat_add(sat_add(sat_add(w.B[ls], l1[s]), via), leg2);
-                if (c < best) { best = c; bls = ls; }
-            }
+template <int LT>
+__device__ __forceinline__ void edge_table(const LaneConst<LT>& c, const Tabs& t, const WScr& w, int v, int lt,
+                                           int nH, int nV, bool act) {
+    if (!act) return;
+    const int u = t.par[v];
+    const int xv = t.x[v], yv = t.y[v], xu = t.x[u], yu = t.y[u];
+    uint32_t best = FGR_INF;
+    int bls = lt;
+    if (yv == yu || xv == xu) {                   // straight: one leg on ls = lt (R7)
+        const int de = (yv == yu) ? 0 : 1;
+        if (c.my_dir == de) {
+            const uint32_t leg = de == 0 ? t.legH[(size_t)v * 2 * nH + c.my_slot] : t.legV[(size_t)v * 2 * nV + c.my_slot];
+            best = sat_add(w.B[lt], leg);
         }
-        t.E[(size_t)v * L + lt] = best;
-        t.recE[(size_t)v * L + lt] = (uint8_t)bls;
+    } else {
+        // bend 0 (lt vertical): leg 1 H on row y_v, leg 2 V on col x_u;
+        // bend 1 (lt horizontal): leg 1 V on col x_v, leg 2 H on row y_u
+        const bool b0 = c.my_dir == 1;
+        const uint32_t leg2 = b0 ? t.legV[((size_t)v * 2 + 1) * nV + c.my_slot] : t.legH[((size_t)v * 2 + 1) * nH + c.my_slot];
+        const uint32_t* l1 = b0 ? t.legH + (size_t)v * 2 * nH : t.legV + (size_t)v * 2 * nV;
+        const uint32_t opp = b0 ? c.hmask : ~c.hmask;
+        uint32_t vplt = 0;
+#pragma unroll
+        for (int l = 0; l < LT; l++)
+            if (l == lt) vplt = c.vp[l];
+        int s = 0;
+#pragma unroll
+        for (int ls = 0; ls < LT; ls++)
+            if ((opp >> ls) & 1u) {
+                const uint32_t via = ls < lt ? vplt - c.vp[ls] : c.vp[ls] - vplt;
+                const uint32_t cst = sat_add(sat_add(sat_add(w.B[ls], l1[s]), via), leg2);
+                if (cst < best) { best = cst; bls = ls; }
+                s++;
+            }
     }
-    __syncwarp();
+    t.E[(size_t)v * LT + lt] = best;
+    t.recE[(size_t)v * LT + lt] = (uint8_t)bls;
 }
 
-// Generalised Eq. (4): min over spans containing the root pin span; returns the packed key.
-__device__ __forceinline__ unsigned long long root_min(const Tabs& t, const WScr& w, int L) {
-    const int lane = lane_id();
-    unsigned long long best = ~0ull;
-    if (lane < L) {
-        const int plo = t.plo[0], phi = t.phi[0];
-        const int a = plo >= 0 ? plo : L - 1;     // Steiner root: any span
-        const int b = plo >= 0 ? phi : 0;
-        if (lane <= a)
-            for (int hi = max(lane, b); hi < L; hi++) {
-                unsigned long long key = ((unsigned long long)w.F[lane * L + hi] << 8) | (unsigned)(lane << 4) | (unsigned)hi;
-                best = key < best ? key : best;
-            }
-    }
-#pragma unroll
-    for (int off = 16; off; off >>= 1) {
-        unsigned long long o = __shfl_xor_sync(0xffffffffu, best, off);
-        best = o < best ? o : best;
-    }
-    return best;
+// Generalised Eq. (4): candidate of lane lo for the min over spans containing the root pin span.
+template <int LT>
+__device__ __forceinline__ unsigned long long root_cand(const Tabs& t, const WScr& w, int lo, bool act) {
+    if (!act) return ~0ull;
+    const int plo = t.plo[0], phi = t.phi[0];
+    const int a = plo >= 0 ? plo : LT - 1;     // Steiner root: any span
+    const int b = plo >= 0 ? phi : 0;
+    return lo <= a ? w.R[lo * LT + max(lo, b)] : ~0ull;
 }
 
 // S5: child layer = smallest l in the parent's span minimising E_v(l) (R11).
-__device__ __forceinline__ uint32_t backtrack_node(const Hdr* h, const Tabs& t, int v, int L) {
+template <int LT>
+__device__ __forceinline__ uint32_t backtrack_node(const Hdr* h, const Tabs& t, int v) {
     const int u = t.par[v];
     const int sp = t.span[u];
     const int lo = sp >> 4, hi = sp & 15;
     int lt = lo;
-    uint32_t be = t.E[(size_t)v * L + lo];
+    uint32_t be = t.E[(size_t)v * LT + lo];
     for (int l = lo + 1; l <= hi; l++) {
-        const uint32_t e = t.E[(size_t)v * L + l];
+        const uint32_t e = t.E[(size_t)v * LT + l];
         if (e < be) { be = e; lt = l; }
     }
-    const int ls = t.recE[(size_t)v * L + lt];
-    t.span[v] = t.recB[(size_t)v * L + ls];
+    const int ls = t.recE[(size_t)v * LT + lt];
+    t.span[v] = t.recB[(size_t)v * LT + ls];
     const bool straight = (t.x[v] == t.x[u]) || (t.y[v] == t.y[u]);
     const uint32_t bend = straight ? 0u : (h->dir[lt] == 1 ? 0u : 1u);
     return bend | ((uint32_t)ls << 8) | ((uint32_t)lt << 16) | ((uint32_t)straight << 24);
 }
 
-// S6: +1 on every unit edge of a leg, and mark the touched segments dirty.
+// S6: +1 on every unit edge of a leg (fire-and-forget RED), and mark the touched
+// 32-position segments and their line stale for the next refresh (plain byte stores).
 __device__ __forceinline__ void commit_leg(const GridView& g, const DirView& d, int line, int a, int b, int sl) {
     if (a >= b) return;
     int32_t* D = d.D + (size_t)line * d.len * d.W + sl;
     for (int p = a; p < b; p++) atomicAdd(D + (size_t)p * d.W, 1);
     const int s0 = a >> FGR_SEG_SHIFT, s1 = (b - 1) >> FGR_SEG_SHIFT;
-    for (int s = s0; s <= s1; s++) {
-        const int gs = d.seg_base + line * d.nseg + s;
-        if (atomicExch(&g.dseg[gs], 1u) == 0u) {
-            const int k = atomicAdd(g.segcount, 1);
-            g.seglist[k] = gs;
-            atomicAdd(&g.linecnt[d.line_base + line], 1u);
-        }
-    }
+    uint8_t* f = g.dseg + d.seg_base + (size_t)line * d.nseg;
+    for (int s = s0; s <= s1; s++) f[s] = 1;
+    g.dline[d.line_base + line] = 1;
 }
 
 __device__ __forceinline__ void commit_edge(const GridView& g, const Hdr* h, int xv, int yv, int xu, int yu, uint32_t seg) {
@@ -334,107 +343,223 @@ __device__ __forceinline__ void commit_edge(const GridView& g, const Hdr* h, int
     }
 }
 
-// ------------------------------------------------------------- kernels
-// Warp path: one warp per net with <= 32 nodes.
-__global__ void __launch_bounds__(FGR_CTA_THREADS) k_dp_small(GridView g, NetsView nv, const int32_t* __restrict__ list,
-                                                               int count, Out o, int commit, int32_t* reset_ptr) {
+// ------------------------------------------------------------- group kernel (nets <= 32 nodes)
+// Flattened (group, item) iteration: item counts per group n[q]; returns the group of item `it`.
+template <int G>
+struct Flat {
+    int pre[G + 1];
+    __device__ __forceinline__ void build(const int (&n)[G]) {
+        pre[0] = 0;
+#pragma unroll
+        for (int q = 0; q < G; q++) pre[q + 1] = pre[q] + n[q];
+    }
+    __device__ __forceinline__ int total() const { return pre[G]; }
+    __device__ __forceinline__ int group(int it) const {
+        int q = 0;
+#pragma unroll
+        for (int k = 1; k < G; k++) q += (it >= pre[k]) ? 1 : 0;
+        return q;
+    }
+    __device__ __forceinline__ int base(int q) const {
+        int b = 0;
+#pragma unroll
+        for (int k = 0; k < G; k++) b = (k == q) ? pre[k] : b;
+        return b;
+    }
+};
+
+template <int LT>
+__global__ void __launch_bounds__(32 * kGroupWarps) k_dp_group(GridView g, NetsView nv, const int32_t* __restrict__ list,
+                                                               int count, Out o, int commit) {
+    constexpr int G = groups_of(LT);
     extern __shared__ __align__(16) unsigned char smem[];
     Hdr* h = reinterpret_cast<Hdr*>(smem);
     init_hdr(h, g);
-    if (reset_ptr && blockIdx.x == 0 && threadIdx.x == 0) *reset_ptr = 0;
     __syncthreads();
-    const int L = g.L, nH = g.h.cnt, nV = g.v.cnt;
+    const int nH = g.h.cnt, nV = g.v.cnt;
     const int warp = threadIdx.x >> 5, lane = lane_id();
-    const int idx = blockIdx.x * FGR_WARPS_PER_CTA + warp;
-    if (idx >= count) return;
-    const size_t per_warp = a16(sizeof(Hdr)) ;
-    unsigned char* base = smem + per_warp + (size_t)warp * (tabs_bytes(32, L, nH, nV, false) + wscr_bytes(L));
-    Tabs t = carve_tabs(base, 32, L, nH, nV, false);
-    WScr w = carve_wscr(base + tabs_bytes(32, L, nH, nV, false), L);
-    const int net = list[idx];
-    const int a0 = nv.off[net];
-    const int m = nv.off[net + 1] - a0;
-    // node data (lane = node)
-    int par = -1, xx = 0, yy = 0;
-    if (lane < m) {
-        xx = nv.x[a0 + lane]; yy = nv.y[a0 + lane]; par = nv.par[a0 + lane];
-        t.x[lane] = (int16_t)xx; t.y[lane] = (int16_t)yy; t.par[lane] = (int16_t)par;
-        t.plo[lane] = nv.plo[a0 + lane]; t.phi[lane] = nv.phi[a0 + lane];
+    const int idx0 = (blockIdx.x * kGroupWarps + warp) * G;
+    if (idx0 >= count) return;
+    const int gi = lane / LT < G ? lane / LT : G;      // my group (G = idle lane)
+    const int gl = lane - gi * LT;                     // my layer inside the group
+    const size_t tb = tabs_bytes(kMC, LT, nH, nV, false), wb = wscr_bytes(LT);
+    unsigned char* wbase = smem + a16(sizeof(Hdr)) + (size_t)warp * G * (tb + wb);
+    auto tabs_of = [&](int q) { return carve_tabs(wbase + (size_t)q * (tb + wb), kMC, LT, nH, nV, false); };
+    auto wscr_of = [&](int q) { return carve_wscr(wbase + (size_t)q * (tb + wb) + tb, LT); };
+    LaneConst<LT> c;
+    c.load(h, gl);
+    // nets of the G groups
+    int net_l = -1, a0_l = 0, m_l = 0;
+    if (lane < G && idx0 + lane < count) {
+        net_l = list[idx0 + lane];
+        a0_l = nv.off[net_l];
+        m_l = nv.off[net_l + 1] - a0_l;
     }
-    // depth by pointer jumping (root points at itself with depth 0)
-    int dep = (lane > 0 && lane < m) ? 1 : 0;
-    int anc = (lane > 0 && lane < m) ? par : 0;
+    int mq[G], aq[G];
 #pragma unroll
-    for (int r = 0; r < 5; r++) {
-        const int da = __shfl_sync(0xffffffffu, dep, anc);
-        const int aa = __shfl_sync(0xffffffffu, anc, anc);
-        dep += da; anc = aa;
-    }
-    // children masks
-    for (int v = 0; v < m; v++) {
-        const uint32_t cm = __ballot_sync(0xffffffffu, lane > 0 && lane < m && par == v);
-        if (lane == v) t.cmask[v] = cm;
-    }
-    int maxd = dep;
+    for (int q = 0; q < G; q++) { mq[q] = __shfl_sync(0xffffffffu, m_l, q); aq[q] = __shfl_sync(0xffffffffu, a0_l, q); }
+    int my_m = 0;
 #pragma unroll
-    for (int off = 16; off; off >>= 1) maxd = max(maxd, __shfl_xor_sync(0xffffffffu, maxd, off));
-    if (lane < m) t.depth[lane] = (uint16_t)dep;
-    __syncwarp();
-    // all prefix gathers of the net up front
-    for (int task = lane; task < 4 * (m - 1); task += 32) gather_task(g, t, task);
-    __syncwarp();
-    // bottom-up DP, deepest level first
-    for (int d = maxd; d >= 1; d--) {
-        uint32_t lv = __ballot_sync(0xffffffffu, lane < m && dep == d);
-        while (lv) {
-            const int v = __ffs(lv) - 1;
-            lv &= lv - 1;
-            span_table<false>(h, t, w, v, L);
-            node_table(t, w, v, L);
-            edge_table(h, t, w, v, L, nH, nV);
-        }
+    for (int q = 0; q < G; q++) my_m = (gi == q) ? mq[q] : my_m;
+    Flat<G> nodes;
+    nodes.build(mq);
+    // node data, zeroed child masks
+    for (int it = lane; it < nodes.total(); it += 32) {
+        const int q = nodes.group(it), i = it - nodes.base(q);
+        int a = 0;
+#pragma unroll
+        for (int k = 0; k < G; k++) a = (k == q) ? aq[k] : a;
+        const Tabs t = tabs_of(q);
+        t.x[i] = nv.x[a + i]; t.y[i] = nv.y[a + i]; t.par[i] = (int16_t)nv.par[a + i];
+        t.plo[i] = nv.plo[a + i]; t.phi[i] = nv.phi[a + i];
+        t.aux[i] = 0;
     }
-    span_table<false>(h, t, w, 0, L);
-    const unsigned long long rk = root_min(t, w, L);
-    if (lane == 0) t.span[0] = (uint8_t)(rk & 0xFF);
     __syncwarp();
-    // top-down backtrack
-    uint32_t seg = 0xFFFFFFFFu;
-    for (int d = 1; d <= maxd; d++) {
-        if (lane < m && dep == d) seg = backtrack_node(h, t, lane, L);
+    for (int it = lane; it < nodes.total(); it += 32) {
+        const int q = nodes.group(it), i = it - nodes.base(q);
+        if (i > 0) { const Tabs t = tabs_of(q); atomicOr(&t.aux[t.par[i]], 1u << i); }
+    }
+    // all prefix gathers of the G nets up front
+    int tq[G];
+#pragma unroll
+    for (int q = 0; q < G; q++) tq[q] = mq[q] > 1 ? 4 * (mq[q] - 1) : 0;
+    Flat<G> tasks;
+    tasks.build(tq);
+    for (int it = lane; it < tasks.total(); it += 32) {
+        const int q = tasks.group(it);
+        gather_task(g, tabs_of(q), it - tasks.base(q));
+    }
+    __syncwarp();
+    // bottom-up DP: descending node index is children-first (parent[i] < i)
+    int maxm = 0;
+#pragma unroll
+    for (int q = 0; q < G; q++) maxm = max(maxm, mq[q]);
+    const Tabs t = tabs_of(gi < G ? gi : 0);
+    const WScr w = wscr_of(gi < G ? gi : 0);
+    const bool glane = gi < G && gl < LT;
+    unsigned long long rootkey = ~0ull;
+    for (int k = 0; k + 1 < maxm; k++) {
+        const int v = my_m - 1 - k;
+        const bool act = glane && v >= 1;
+        span_rows<LT, false>(c, t, w, v, gl, act);
+        __syncwarp();
+        node_table<LT>(t, w, v, gl, act);
+        __syncwarp();
+        edge_table<LT>(c, t, w, v, gl, nH, nV, act);
         __syncwarp();
     }
-    if (lane < m) {
-        if (o.rec_seg) o.rec_seg[o.rec_off[o.list_base + idx] + lane] = seg;
-        else o.seg[a0 + lane] = seg;
+    // root (generalised Eq. (4)); a group's lanes reduce through the B scratch row
+    span_rows<LT, false>(c, t, w, 0, gl, glane && my_m >= 2);
+    __syncwarp();
+    const unsigned long long rc = root_cand<LT>(t, w, gl, glane && my_m >= 2);
+    __syncwarp();
+    if (glane && my_m >= 2) w.R[LT * LT - 1 - gl] = rc;   // R is dead now: reuse its tail for the reduction
+    __syncwarp();
+    if (glane && gl == 0 && my_m >= 2) {
+        unsigned long long b = ~0ull;
+#pragma unroll
+        for (int l = 0; l < LT; l++) { const unsigned long long x = w.R[LT * LT - 1 - l]; b = x < b ? x : b; }
+        t.span[0] = (uint8_t)(b & 0xFF);
+        rootkey = b;
     }
-    if (lane == 0) {
-        const uint32_t total = (uint32_t)(rk >> 8);
-        if (o.rec_seg) o.rec_cost[o.list_base + idx] = total;
-        else o.cost[net] = total;
+    // depth by pointer jumping (aux = ancestor), then a level-ordered backtrack
+    for (int it = lane; it < nodes.total(); it += 32) {
+        const int q = nodes.group(it), i = it - nodes.base(q);
+        const Tabs tt = tabs_of(q);
+        tt.depth[i] = i ? 1 : 0;
+        tt.aux[i] = i ? (uint32_t)tt.par[i] : 0u;
     }
-    if (commit && lane > 0 && lane < m) commit_edge(g, h, xx, yy, t.x[par], t.y[par], seg);
+    __syncwarp();
+#pragma unroll 1
+    for (int r = 0; r < 5; r++) {
+        uint32_t nd[G], na[G];
+#pragma unroll
+        for (int s = 0; s < G; s++) {
+            const int it = lane + 32 * s;
+            if (it < nodes.total()) {
+                const int q = nodes.group(it), i = it - nodes.base(q);
+                const Tabs tt = tabs_of(q);
+                const uint32_t an = tt.aux[i];
+                nd[s] = tt.depth[i] + tt.depth[an];
+                na[s] = tt.aux[an];
+            }
+        }
+        __syncwarp();
+#pragma unroll
+        for (int s = 0; s < G; s++) {
+            const int it = lane + 32 * s;
+            if (it < nodes.total()) {
+                const int q = nodes.group(it), i = it - nodes.base(q);
+                const Tabs tt = tabs_of(q);
+                tt.depth[i] = (uint16_t)nd[s];
+                tt.aux[i] = na[s];
+            }
+        }
+        __syncwarp();
+    }
+    int maxd = 0;
+    for (int it = lane; it < nodes.total(); it += 32) {
+        const int q = nodes.group(it), i = it - nodes.base(q);
+        maxd = max(maxd, (int)tabs_of(q).depth[i]);
+    }
+#pragma unroll
+    for (int off = 16; off; off >>= 1) maxd = max(maxd, __shfl_xor_sync(0xffffffffu, maxd, off));
+    for (int d = 1; d <= maxd; d++) {
+        for (int it = lane; it < nodes.total(); it += 32) {
+            const int q = nodes.group(it), i = it - nodes.base(q);
+            const Tabs tt = tabs_of(q);
+            if (tt.depth[i] == d) {
+                const uint32_t s = backtrack_node<LT>(h, tt, i);
+                tt.legH[(size_t)i * 2 * nH] = s;       // keep the route for the outputs and the commit
+            }
+        }
+        __syncwarp();
+    }
+    // outputs and commit
+    for (int it = lane; it < nodes.total(); it += 32) {
+        const int q = nodes.group(it), i = it - nodes.base(q);
+        const Tabs tt = tabs_of(q);
+        const uint32_t s = i ? tt.legH[(size_t)i * 2 * nH] : 0xFFFFFFFFu;
+        int a = 0;
+#pragma unroll
+        for (int k = 0; k < G; k++) a = (k == q) ? aq[k] : a;
+        if (o.rec_seg) o.rec_seg[o.rec_off[o.list_base + idx0 + q] + i] = s;
+        else o.seg[a + i] = s;
+        if (commit && i > 0) {
+            const int u = tt.par[i];
+            commit_edge(g, h, tt.x[i], tt.y[i], tt.x[u], tt.y[u], s);
+        }
+    }
+    if (glane && gl == 0 && my_m >= 1) {
+        const uint32_t total = my_m >= 2 ? (uint32_t)(rootkey >> 8) : 0u;
+        if (o.rec_seg) o.rec_cost[o.list_base + idx0 + gi] = total;
+        else o.cost[list[idx0 + gi]] = total;
+    }
 }
 
-// CTA path: one 256-thread block per net with > 32 nodes.
+// ------------------------------------------------------------- CTA kernel (nets > 32 nodes)
+template <int LT>
 __global__ void __launch_bounds__(FGR_CTA_THREADS) k_dp_large(GridView g, NetsView nv, const int32_t* __restrict__ list,
-                                                               int count, Out o, int commit, int32_t* reset_ptr) {
+                                                               int count, Out o, int commit) {
+    constexpr int G = groups_of(LT);
     extern __shared__ __align__(16) unsigned char smem[];
     Hdr* h = reinterpret_cast<Hdr*>(smem);
     __shared__ int s_maxd;
     __shared__ unsigned long long s_root;
     init_hdr(h, g);
-    if (threadIdx.x == 0) s_maxd = 0;
-    if (reset_ptr && blockIdx.x == 0 && threadIdx.x == 0) *reset_ptr = 0;
-    const int L = g.L, nH = g.h.cnt, nV = g.v.cnt;
+    if (threadIdx.x == 0) { s_maxd = 0; s_root = ~0ull; }
+    const int nH = g.h.cnt, nV = g.v.cnt;
     const int warp = threadIdx.x >> 5, lane = lane_id(), tid = threadIdx.x, T = blockDim.x;
+    const int gi = lane / LT < G ? lane / LT : G;
+    const int gl = lane - gi * LT;
+    const bool glane = gi < G && gl < LT;
     const int idx = blockIdx.x;
     const int net = list[idx];
     const int a0 = nv.off[net];
     const int m = nv.off[net + 1] - a0;
     unsigned char* base = smem + a16(sizeof(Hdr));
-    WScr w = carve_wscr(base + (size_t)warp * wscr_bytes(L), L);
-    Tabs t = carve_tabs(base + (size_t)FGR_WARPS_PER_CTA * wscr_bytes(L), m, L, nH, nV, true);
+    const WScr w = carve_wscr(base + ((size_t)warp * G + (gi < G ? gi : 0)) * wscr_bytes(LT), LT);
+    const Tabs t = carve_tabs(base + (size_t)FGR_WARPS_PER_CTA * G * wscr_bytes(LT), m, LT, nH, nV, true);
     for (int i = tid; i < m; i += T) {
         const int p = nv.par[a0 + i];
         t.x[i] = nv.x[a0 + i]; t.y[i] = nv.y[a0 + i]; t.par[i] = (int16_t)p;
@@ -442,9 +567,12 @@ __global__ void __launch_bounds__(FGR_CTA_THREADS) k_dp_large(GridView g, NetsVi
         t.depth[i] = i ? 1 : 0;
         t.anc[i] = (uint16_t)(i ? p : 0);
     }
-    uint32_t* cnt = t.legH;   // child counts reuse the leg area before the gathers
-    for (int i = tid; i <= m; i += T) cnt[i] = 0;
+    uint32_t* cnt = t.legH;   // child counts and level counts reuse the leg areas before the gathers
+    uint32_t* dcnt = t.legV;
+    for (int i = tid; i <= m; i += T) { cnt[i] = 0; dcnt[i] = 0; }
     __syncthreads();
+    LaneConst<LT> c;
+    c.load(h, gl);
     for (int i = 1 + tid; i < m; i += T) atomicAdd(&cnt[t.par[i]], 1u);
     // depth by pointer jumping: ceil(log2 m) rounds
     for (int r = 1; r < m; r <<= 1) {
@@ -462,66 +590,91 @@ __global__ void __launch_bounds__(FGR_CTA_THREADS) k_dp_large(GridView g, NetsVi
         }
         __syncthreads();
     }
-    // child CSR: exclusive scan of counts by warp 0
-    if (warp == 0) {
+    int md = 0;
+    for (int i = tid; i < m; i += T) {
+        md = max(md, (int)t.depth[i]);
+        atomicAdd(&dcnt[t.depth[i]], 1u);
+    }
+    atomicMax(&s_maxd, md);
+    __syncthreads();
+    const int maxd = s_maxd;
+    // warp 0: child CSR; warp 1: level CSR (exclusive scans)
+    if (warp < 2) {
+        const uint32_t* src = warp == 0 ? cnt : dcnt;
+        uint16_t* dst = warp == 0 ? t.cstart : t.lvstart;
+        const int n = warp == 0 ? m : maxd + 1;
         uint32_t carry = 0;
-        for (int c0 = 0; c0 <= m; c0 += 32) {
+        for (int c0 = 0; c0 <= n; c0 += 32) {
             const int i = c0 + lane;
-            const uint32_t v = i <= m ? cnt[i] : 0;
+            const uint32_t v = i <= n ? src[i] : 0;
             uint32_t inc = v;
 #pragma unroll
             for (int off = 1; off < 32; off <<= 1) {
                 const uint32_t q = __shfl_up_sync(0xffffffffu, inc, off);
                 if (lane >= off) inc += q;
             }
-            if (i <= m) t.cstart[i] = (uint16_t)(carry + inc - v);
+            if (i <= n) dst[i] = (uint16_t)(carry + inc - v);
             carry += __shfl_sync(0xffffffffu, inc, 31);
         }
     }
-    int md = 0;
-    for (int i = tid; i < m; i += T) md = max(md, (int)t.depth[i]);
-    atomicMax(&s_maxd, md);
     __syncthreads();
     for (int i = tid; i <= m; i += T) cnt[i] = t.cstart[i];
+    for (int i = tid; i <= maxd; i += T) dcnt[i] = t.lvstart[i];
     __syncthreads();
-    for (int i = 1 + tid; i < m; i += T) t.clist[atomicAdd(&cnt[t.par[i]], 1u)] = (uint16_t)i;
+    for (int i = tid; i < m; i += T) {
+        if (i > 0) t.clist[atomicAdd(&cnt[t.par[i]], 1u)] = (uint16_t)i;
+        t.anc[atomicAdd(&dcnt[t.depth[i]], 1u)] = (uint16_t)i;   // nodes grouped by level
+    }
     __syncthreads();
+#pragma unroll 2
     for (int task = tid; task < 4 * (m - 1); task += T) gather_task(g, t, task);
     __syncthreads();
-    const int maxd = s_maxd;
+    // bottom-up DP: 8 warps x G groups evaluate nodes of one level side by side
+    constexpr int SLOTS = FGR_WARPS_PER_CTA * G;
+    const int myslot = warp * G + gi;
     for (int d = maxd; d >= 1; d--) {
-        for (int c0 = warp * 32; c0 < m; c0 += T) {
-            const int i = c0 + lane;
-            uint32_t lv = __ballot_sync(0xffffffffu, i < m && t.depth[i] == d);
-            while (lv) {
-                const int v = c0 + __ffs(lv) - 1;
-                lv &= lv - 1;
-                span_table<true>(h, t, w, v, L);
-                node_table(t, w, v, L);
-                edge_table(h, t, w, v, L, nH, nV);
-            }
+        const int k0 = t.lvstart[d], k1 = t.lvstart[d + 1];
+        for (int kb = k0; kb < k1; kb += SLOTS) {
+            const int k = kb + myslot;
+            const bool act = glane && k < k1;
+            const int v = act ? t.anc[k] : 0;
+            span_rows<LT, true>(c, t, w, v, gl, act);
+            __syncwarp();
+            node_table<LT>(t, w, v, gl, act);
+            __syncwarp();
+            edge_table<LT>(c, t, w, v, gl, nH, nV, act);
+            __syncwarp();
         }
         __syncthreads();
     }
     if (warp == 0) {
-        span_table<true>(h, t, w, 0, L);
-        const unsigned long long rk = root_min(t, w, L);
-        if (lane == 0) { t.span[0] = (uint8_t)(rk & 0xFF); s_root = rk; }
+        const bool act = glane && gi == 0;
+        span_rows<LT, true>(c, t, w, 0, gl, act);
+        __syncwarp();
+        const unsigned long long rc = root_cand<LT>(t, w, gl, act);
+        if (act) atomicMin(&s_root, rc);
     }
     __syncthreads();
+    if (tid == 0) t.span[0] = (uint8_t)(s_root & 0xFF);
+    __syncthreads();
     for (int d = 1; d <= maxd; d++) {
-        for (int i = tid; i < m; i += T)
-            if (t.depth[i] == d) {
-                const uint32_t s = backtrack_node(h, t, i, L);
-                if (o.rec_seg) o.rec_seg[o.rec_off[o.list_base + idx] + i] = s;
-                else o.seg[a0 + i] = s;
-                if (commit) {
-                    const int u = t.par[i];
-                    commit_edge(g, h, t.x[i], t.y[i], t.x[u], t.y[u], s);
-                }
-            }
+        const int k1 = t.lvstart[d + 1];
+        for (int k = t.lvstart[d] + tid; k < k1; k += T) {
+            const int i = t.anc[k];
+            const uint32_t s = backtrack_node<LT>(h, t, i);
+            if (o.rec_seg) o.rec_seg[o.rec_off[o.list_base + idx] + i] = s;
+            else o.seg[a0 + i] = s;
+            t.legH[(size_t)i * 2 * nH] = s;   // the leg costs are dead now: keep the route for the commit
+        }
         __syncthreads();
     }
+    // S6 for the whole net in one pass (the atomics' latencies overlap across threads)
+    if (commit)
+        for (int i = 1 + tid; i < m; i += T) {
+            const uint32_t s = t.legH[(size_t)i * 2 * nH];
+            const int u = t.par[i];
+            commit_edge(g, h, t.x[i], t.y[i], t.x[u], t.y[u], s);
+        }
     if (tid == 0) {
         const uint32_t total = (uint32_t)(s_root >> 8);
         if (o.rec_seg) { o.rec_seg[o.rec_off[o.list_base + idx]] = 0xFFFFFFFFu; o.rec_cost[o.list_base + idx] = total; }
@@ -532,10 +685,9 @@ __global__ void __launch_bounds__(FGR_CTA_THREADS) k_dp_large(GridView g, NetsVi
 // Commit from route records (multi-GPU: after the exchange every rank commits every net).
 __global__ void __launch_bounds__(256) k_commit_records(GridView g, NetsView nv, const int32_t* __restrict__ list, int count,
                                                         const uint32_t* __restrict__ rec_seg,
-                                                        const int32_t* __restrict__ rec_off, int list_base, int32_t* reset_ptr) {
+                                                        const int32_t* __restrict__ rec_off, int list_base) {
     __shared__ Hdr hs;
     init_hdr(&hs, g);
-    if (reset_ptr && blockIdx.x == 0 && threadIdx.x == 0) *reset_ptr = 0;
     __syncthreads();
     const int warp = (int)((blockIdx.x * (size_t)blockDim.x + threadIdx.x) >> 5);
     const int nwarps = (int)((gridDim.x * (size_t)blockDim.x) >> 5);
@@ -550,79 +702,89 @@ __global__ void __launch_bounds__(256) k_commit_records(GridView g, NetsView nv,
     }
 }
 
-}  // namespace
-
-size_t fgr_dp_smem_small(const fgr_grid* g) {
-    return a16(sizeof(Hdr)) + (size_t)FGR_WARPS_PER_CTA * (tabs_bytes(32, g->L, g->nH, g->nV, false) + wscr_bytes(g->L));
+// ------------------------------------------------------------- host side
+size_t smem_group(int L, int nH, int nV) {
+    return a16(sizeof(Hdr)) + (size_t)kGroupWarps * groups_of(L) * (tabs_bytes(kMC, L, nH, nV, false) + wscr_bytes(L));
 }
 
-size_t fgr_dp_smem_large(const fgr_grid* g, int m) {
-    return a16(sizeof(Hdr)) + (size_t)FGR_WARPS_PER_CTA * wscr_bytes(g->L) + tabs_bytes(m, g->L, g->nH, g->nV, true);
+size_t smem_large(int L, int nH, int nV, int m) {
+    return a16(sizeof(Hdr)) + (size_t)FGR_WARPS_PER_CTA * groups_of(L) * wscr_bytes(L) +
+           tabs_bytes(m, L, nH, nV, true);
 }
 
-cudaError_t fgr_launch_dp(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int count, int nlarge,
-                          int maxm_large, uint32_t* seg_out, uint32_t* cost_out, uint32_t* rec_seg,
-                          const int32_t* rec_off, uint32_t* rec_cost, int list_base, bool commit) {
-    GridView v = g->view;
-    v.seglist = g->d_list[g->parity];
-    v.segcount = g->d_count + g->parity;
-    // The other list was consumed by the refresh that ran before this launch: the
-    // first kernel of this batch resets its length for the next commit.
-    int32_t* reset = commit ? g->d_count + (g->parity ^ 1) : nullptr;
-    Out o;
-    o.seg = seg_out; o.cost = cost_out; o.rec_seg = rec_seg; o.rec_off = rec_off; o.rec_cost = rec_cost;
-    o.list_base = list_base;
-    cudaError_t e = cudaSuccess;
-    static int configured = 0;
+template <int LT>
+cudaError_t launch_lt(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int count, int nlarge,
+                      int maxm_large, const Out& o, bool commit) {
+    static bool configured = false;   // one device per process is the supported configuration
     if (!configured) {
-        // opt in to the full shared memory minus each kernel's static shared memory
         cudaFuncAttributes fa;
-        e = cudaFuncGetAttributes(&fa, k_dp_large);
+        cudaError_t e = cudaFuncGetAttributes(&fa, k_dp_large<LT>);
         if (e == cudaSuccess)
-            e = cudaFuncSetAttribute(k_dp_large, cudaFuncAttributeMaxDynamicSharedMemorySize,
+            e = cudaFuncSetAttribute(k_dp_large<LT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                      g->max_smem - (int)fa.sharedSizeBytes);
-        if (e == cudaSuccess) e = cudaFuncGetAttributes(&fa, k_dp_small);
+        if (e == cudaSuccess) e = cudaFuncGetAttributes(&fa, k_dp_group<LT>);
         if (e == cudaSuccess)
-            e = cudaFuncSetAttribute(k_dp_small, cudaFuncAttributeMaxDynamicSharedMemorySize,
+            e = cudaFuncSetAttribute(k_dp_group<LT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                      g->max_smem - (int)fa.sharedSizeBytes);
         if (e != cudaSuccess) return e;
-        configured = 1;
+        configured = true;
     }
+    const GridView& v = g->view;
     if (nlarge > 0) {
-        k_dp_large<<<nlarge, FGR_CTA_THREADS, fgr_dp_smem_large(g, maxm_large), st>>>(v, nv, list, nlarge, o,
-                                                                                       commit ? 1 : 0, reset);
-        reset = nullptr;
+        const int ps = fgr_prof_begin(g, PROF_DP_LARGE, st);
+        k_dp_large<LT><<<nlarge, FGR_CTA_THREADS, smem_large(LT, g->nH, g->nV, maxm_large), st>>>(
+            v, nv, list, nlarge, o, commit ? 1 : 0);
+        fgr_prof_end(g, ps, st);
         g->stats.kernel_launches++;
-        e = cudaGetLastError();
+        cudaError_t e = cudaGetLastError();
         if (e != cudaSuccess) return e;
     }
     const int nsmall = count - nlarge;
     if (nsmall > 0) {
         Out os = o;
-        os.list_base = list_base + nlarge;
-        k_dp_small<<<(nsmall + FGR_WARPS_PER_CTA - 1) / FGR_WARPS_PER_CTA, FGR_CTA_THREADS, fgr_dp_smem_small(g), st>>>(
-            v, nv, list + nlarge, nsmall, os, commit ? 1 : 0, reset);
-        reset = nullptr;
+        os.list_base = o.list_base + nlarge;
+        const int per_cta = kGroupWarps * groups_of(LT);
+        const int ps = fgr_prof_begin(g, PROF_DP_SMALL, st);
+        k_dp_group<LT><<<(nsmall + per_cta - 1) / per_cta, 32 * kGroupWarps, smem_group(LT, g->nH, g->nV), st>>>(
+            v, nv, list + nlarge, nsmall, os, commit ? 1 : 0);
+        fgr_prof_end(g, ps, st);
         g->stats.kernel_launches++;
-        e = cudaGetLastError();
+        cudaError_t e = cudaGetLastError();
         if (e != cudaSuccess) return e;
     }
-    if (reset) return cudaMemsetAsync(reset, 0, sizeof(int32_t), st);
     return cudaSuccess;
+}
+
+}  // namespace
+
+size_t fgr_dp_smem_small(const fgr_grid* g) { return smem_group(g->L, g->nH, g->nV); }
+
+size_t fgr_dp_smem_large(const fgr_grid* g, int m) { return smem_large(g->L, g->nH, g->nV, m); }
+
+cudaError_t fgr_launch_dp(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int count, int nlarge,
+                          int maxm_large, uint32_t* seg_out, uint32_t* cost_out, uint32_t* rec_seg,
+                          const int32_t* rec_off, uint32_t* rec_cost, int list_base, bool commit) {
+    Out o;
+    o.seg = seg_out; o.cost = cost_out; o.rec_seg = rec_seg; o.rec_off = rec_off; o.rec_cost = rec_cost;
+    o.list_base = list_base;
+    switch (g->L) {
+#define FGR_LT(n) case n: return launch_lt<n>(g, st, nv, list, count, nlarge, maxm_large, o, commit);
+        FGR_LT(2) FGR_LT(3) FGR_LT(4) FGR_LT(5) FGR_LT(6) FGR_LT(7) FGR_LT(8) FGR_LT(9) FGR_LT(10) FGR_LT(11)
+        FGR_LT(12) FGR_LT(13) FGR_LT(14) FGR_LT(15) FGR_LT(16)
+#undef FGR_LT
+        default: return cudaErrorInvalidValue;
+    }
 }
 
 cudaError_t fgr_launch_commit(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int count,
                               const uint32_t* rec_seg, const int32_t* rec_off, int list_base) {
-    GridView v = g->view;
-    v.seglist = g->d_list[g->parity];
-    v.segcount = g->d_count + g->parity;
+    const GridView& v = g->view;
     int blocks = (count + 7) / 8;
     if (blocks > g->num_sms * 8) blocks = g->num_sms * 8;
     if (blocks < 1) blocks = 1;
-    k_commit_records<<<blocks, 256, 0, st>>>(v, nv, list, count, rec_seg, rec_off, list_base,
-                                             g->d_count + (g->parity ^ 1));
+    const int ps = fgr_prof_begin(g, PROF_COMMIT, st);
+    k_commit_records<<<blocks, 256, 0, st>>>(v, nv, list, count, rec_seg, rec_off, list_base);
+    fgr_prof_end(g, ps, st);
     g->stats.kernel_launches++;
     return cudaGetLastError();
 }
-
-void fgr_flip_lists(fgr_grid* g) { g->parity ^= 1; }

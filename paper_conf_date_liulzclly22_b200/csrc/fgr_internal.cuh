@@ -26,6 +26,7 @@
 
 #define FGR_SEG 32          // positions per scan segment (one warp)
 #define FGR_SEG_SHIFT 5
+#define FGR_CHUNK_SEGS 8    // segments per refresh task (one warp)
 #define FGR_INF 0x7FFFFFFFu // "impossible" cost; finite costs are < FGR_INF (R19)
 #define FGR_MAXL 16
 #define FGR_SMALL_NET 32    // nets with <= this many nodes take the warp path
@@ -52,11 +53,9 @@ struct GridView {
     DirView h, v;
     int nx, ny, L, S, len_cost;
     const int32_t* table;   // [L][2S+1]
-    uint32_t* dseg;         // [total segments] dirty flag
-    uint32_t* linecnt;      // [ny + nx] dirty segments per line
-    uint32_t* linedone;     // [ny + nx] refreshed segments per line (this launch)
-    int32_t* seglist;       // list the DP appends to (dirty segments)
-    int32_t* segcount;      // its length
+    uint8_t* dseg;          // [total segments] dirty flag (plain stores by the commit)
+    uint8_t* dline;         // [ny + nx] the line has a dirty segment
+    uint32_t* linedone;     // [ny + nx] chunks of the line refreshed in this launch
     unsigned long long* stats;  // [4] device counters (refresh segments, ...)
     uint8_t dir[FGR_MAXL];
     uint8_t slot[FGR_MAXL]; // index of layer l among the layers of its direction
@@ -93,6 +92,17 @@ struct Scratch {            // grow-only device scratch
     size_t bytes = 0;
 };
 
+#include <vector>
+
+struct Profiler {
+    bool on = false;
+    std::vector<cudaEvent_t> pool;        // start/stop pairs
+    std::vector<int> cls;                 // class of each recorded pair
+    size_t used = 0;
+    double ms[FGR_PROF_CLASSES] = {0};
+    long long launches[FGR_PROF_CLASSES] = {0};
+};
+
 struct fgr_grid {
     int device = 0;
     int nx = 0, ny = 0, L = 0, S = 0, len_cost = 0;
@@ -107,10 +117,7 @@ struct fgr_grid {
     void* mem = nullptr;        // one slab for the grid arrays
     size_t mem_bytes = 0;
     int32_t* d_table = nullptr;
-    int32_t* d_list[2] = {nullptr, nullptr};
-    int32_t* d_count = nullptr; // [2]
     unsigned long long* d_stats = nullptr;
-    int parity = 0;             // list the next DP appends to
     bool full_dirty = true;     // next refresh must rescan everything
     bool broken = false;
     int total_segs = 0;
@@ -124,7 +131,14 @@ struct fgr_grid {
     fgr_stats stats{};
     int max_smem = 0;
     int num_sms = 0;
+    Profiler prof;
 };
+
+// Profiling brackets around a launch (no-ops unless fgr_profile_enable(grid, 1)).
+int fgr_prof_begin(fgr_grid* g, int cls, cudaStream_t st);
+void fgr_prof_end(fgr_grid* g, int slot, cudaStream_t st);
+enum { PROF_REFRESH = 0, PROF_DP_SMALL, PROF_DP_LARGE, PROF_COMMIT, PROF_PRE, PROF_SORT, PROF_COLOR, PROF_PLAN_OTHER,
+       PROF_EXCHANGE };
 
 // ------------------------------------------------------------------ host helpers
 fgr_status fgr_set_error(fgr_status s, const char* fmt, ...);
@@ -148,7 +162,6 @@ cudaError_t fgr_launch_commit(fgr_grid* g, cudaStream_t st, const NetsView& nv, 
                               const uint32_t* rec_seg, const int32_t* rec_off, int list_base);
 size_t fgr_dp_smem_small(const fgr_grid* g);
 size_t fgr_dp_smem_large(const fgr_grid* g, int m);
-void fgr_flip_lists(fgr_grid* g);   // after each DP launch: the refresh consumes what the DP produced
 
 static inline NetsView fgr_nets_view(const fgr_nets* n) {
     NetsView v;

@@ -137,13 +137,26 @@ __global__ void k_tile_bounds(int T, const unsigned long long* __restrict__ tkey
 }
 
 // S2 core: first-fit colouring in rank order, dataflow over published colours.
+// A warp scans its net's candidate lists without blocking: colours already
+// published are marked at once, unpublished earlier neighbours are deferred and
+// waited for only after the whole scan, so the scans of consecutive big nets
+// overlap and only the (short) publish chain is serial.
 #define COLOR_BITS 1024
+#define COLOR_DEFER 128
+#define COLOR_UNROLL 4
+__device__ __forceinline__ void mark_colour(uint32_t* bw, int c, int wb) {
+    c -= wb;
+    if (c >= 0 && c < COLOR_BITS) atomicOr(&bw[c >> 5], 1u << (c & 31));
+}
+
 __global__ void __launch_bounds__(256) k_color(int R, const unsigned long long* __restrict__ box_r,
                                                const int* __restrict__ tstart, const int* __restrict__ tend,
                                                const int* __restrict__ entries, int tiles_x, int* color,
                                                int* __restrict__ ticket, int* __restrict__ nbatches,
                                                int* __restrict__ bcount) {
     __shared__ uint32_t bits[8][COLOR_BITS / 32];
+    __shared__ int defer[8][COLOR_DEFER];
+    __shared__ int ndefer[8];
     const int w = threadIdx.x >> 5, lane = lane_id();
     uint32_t* bw = bits[w];
     volatile int* vcolor = color;
@@ -157,30 +170,55 @@ __global__ void __launch_bounds__(256) k_color(int R, const unsigned long long* 
         int result = -1;
         for (int wb = 0; result < 0; wb += COLOR_BITS) {
             for (int q = lane; q < COLOR_BITS / 32; q += 32) bw[q] = 0;
+            if (lane == 0) ndefer[w] = 0;
             __syncwarp();
             for (int ty = y0 >> TILE_SHIFT; ty <= (y1 >> TILE_SHIFT); ty++)
                 for (int tx = x0 >> TILE_SHIFT; tx <= (x1 >> TILE_SHIFT); tx++) {
                     const int t = ty * tiles_x + tx;
                     const int s = tstart[t], e = tend[t];
-                    for (int base = s; base < e; base += 32) {
-                        const int j = base + lane;
-                        const int rr = j < e ? entries[j] : 0x7FFFFFFF;
-                        if (rr < r) {
-                            int a0, b0, a1, b1;
-                            unpack_box(box_r[rr], a0, b0, a1, b1);
-                            if (!(a1 < x0 || x1 < a0 || b1 < y0 || y1 < b0)) {
-                                const int cx = max(a0, x0) >> TILE_SHIFT, cy = max(b0, y0) >> TILE_SHIFT;
-                                if (cx == tx && cy == ty) {           // count each pair once
-                                    int c;
-                                    while ((c = vcolor[rr]) < 0) __nanosleep(64);
-                                    c -= wb;
-                                    if (c >= 0 && c < COLOR_BITS) atomicOr(&bw[c >> 5], 1u << (c & 31));
+                    for (int base = s; base < e; base += 32 * COLOR_UNROLL) {
+                        int rr[COLOR_UNROLL];
+                        unsigned long long bb[COLOR_UNROLL];
+#pragma unroll
+                        for (int u = 0; u < COLOR_UNROLL; u++) {
+                            const int j = base + u * 32 + lane;
+                            rr[u] = j < e ? __ldg(entries + j) : 0x7FFFFFFF;
+                        }
+#pragma unroll
+                        for (int u = 0; u < COLOR_UNROLL; u++) bb[u] = rr[u] < r ? __ldg(box_r + rr[u]) : 0ull;
+                        bool stop = false;
+#pragma unroll
+                        for (int u = 0; u < COLOR_UNROLL; u++) {
+                            stop |= (rr[u] != 0x7FFFFFFF && rr[u] >= r);
+                            if (rr[u] < r) {
+                                int a0, b0, a1, b1;
+                                unpack_box(bb[u], a0, b0, a1, b1);
+                                if (!(a1 < x0 || x1 < a0 || b1 < y0 || y1 < b0) &&
+                                    (max(a0, x0) >> TILE_SHIFT) == tx && (max(b0, y0) >> TILE_SHIFT) == ty) {
+                                    const int c = vcolor[rr[u]];
+                                    if (c >= 0) mark_colour(bw, c, wb);
+                                    else {
+                                        const int k = atomicAdd(&ndefer[w], 1);
+                                        if (k < COLOR_DEFER) defer[w][k] = rr[u];
+                                        else {
+                                            int cc;
+                                            while ((cc = vcolor[rr[u]]) < 0) __nanosleep(64);
+                                            mark_colour(bw, cc, wb);
+                                        }
+                                    }
                                 }
                             }
                         }
-                        if (__any_sync(0xffffffffu, j < e && rr >= r)) break;   // lists are rank-sorted
+                        if (__any_sync(0xffffffffu, stop)) break;   // lists are rank-sorted
                     }
                 }
+            __syncwarp();
+            const int nd = min(ndefer[w], COLOR_DEFER);
+            for (int k = lane; k < nd; k += 32) {
+                int cc;
+                while ((cc = vcolor[defer[w][k]]) < 0) __nanosleep(32);
+                mark_colour(bw, cc, wb);
+            }
             __syncwarp();
             // smallest clear bit in this window
             int found = -1;
@@ -206,13 +244,14 @@ __global__ void __launch_bounds__(256) k_color(int R, const unsigned long long* 
     }
 }
 
+// batch-major, then larger nets first (large nets lead each batch; similar sizes share a warp), then rank
 __global__ void k_batch_keys(int R, const int* __restrict__ color, const unsigned long long* __restrict__ keys,
                              const int* __restrict__ msize, unsigned long long* __restrict__ bkeys) {
     const int r = blockIdx.x * blockDim.x + threadIdx.x;
     if (r >= R) return;
     const int id = (int)(keys[r] & 0xFFFFFFFFu);
-    const unsigned small = msize[id] > FGR_SMALL_NET ? 0u : 0x80000000u;
-    bkeys[r] = ((unsigned long long)color[r] << 32) | small | (unsigned)r;
+    const unsigned inv = 2047u - (unsigned)min(msize[id], 2047);
+    bkeys[r] = ((unsigned long long)color[r] << 42) | ((unsigned long long)inv << 31) | (unsigned)r;
 }
 
 __global__ void k_finalize(int N, const int* __restrict__ counters, const unsigned long long* __restrict__ keys,
@@ -225,7 +264,7 @@ __global__ void k_finalize(int N, const int* __restrict__ counters, const unsign
     if (i < R) {
         const unsigned long long bk = bkeys[i];
         const int r = (int)(bk & 0x7FFFFFFFu);
-        const int c = (int)(bk >> 32);
+        const int c = (int)(bk >> 42);
         const int id = (int)(keys[r] & 0xFFFFFFFFu);
         order[i] = id;
         batch_of_net[id] = c;
@@ -317,14 +356,18 @@ extern "C" FGR_API fgr_status fgr_plan(fgr_grid* g, const fgr_nets* nets, int32_
     int hc[8] = {0, 0x7FFFFFFF, 0x7FFFFFFF, 0, 0, 0, 0, 0};
     FGR_CHECK_CUDA(g, cudaMemcpyAsync(counters, hc, sizeof(hc), cudaMemcpyHostToDevice, st));
     FGR_CHECK_CUDA(g, cudaMemsetAsync(tstart, 0, 2 * sizeof(int) * ntiles, st));
+    int ps = fgr_prof_begin(g, PROF_PRE, st);
     k_preprocess<<<(unsigned)(((size_t)N * 32 + 255) / 256), 256, 0, st>>>(p, nv, keys, box, msize, segb, counters);
+    fgr_prof_end(g, ps, st);
     FGR_CHECK_CUDA(g, cudaGetLastError());
     // S1: sort by (HPWL, id)
     size_t tmp_bytes = 0;
     cub::DeviceRadixSort::SortKeys(nullptr, tmp_bytes, keys, keys_s, N, 0, 48, st);
     void* tmp = fgr_scratch(g->s_plan[8], tmp_bytes, &e);
     if (e != cudaSuccess) return fgr_cuda_fail(g, e, "plan sort scratch");
+    ps = fgr_prof_begin(g, PROF_SORT, st);
     FGR_CHECK_CUDA(g, cub::DeviceRadixSort::SortKeys(tmp, tmp_bytes, keys, keys_s, N, 0, 48, st));
+    fgr_prof_end(g, ps, st);
     k_rank_boxes<<<(N + 1 + 255) / 256, 256, 0, st>>>(N, counters, keys_s, box, box_r, tcount, tiles_x);
     FGR_CHECK_CUDA(g, cudaGetLastError());
     // tile offsets
@@ -360,7 +403,9 @@ extern "C" FGR_API fgr_status fgr_plan(fgr_grid* g, const fgr_nets* nets, int32_
         cub::DeviceRadixSort::SortKeys(nullptr, tmp_bytes, tkeys, tkeys_s, T, 0, tb, st);
         tmp = fgr_scratch(g->s_plan[8], tmp_bytes, &e);
         if (e != cudaSuccess) return fgr_cuda_fail(g, e, "plan tile sort scratch");
+        ps = fgr_prof_begin(g, PROF_SORT, st);
         FGR_CHECK_CUDA(g, cub::DeviceRadixSort::SortKeys(tmp, tmp_bytes, tkeys, tkeys_s, T, 0, tb, st));
+        fgr_prof_end(g, ps, st);
         k_tile_bounds<<<(T + 255) / 256, 256, 0, st>>>(T, tkeys_s, tstart, tend, entries);
         FGR_CHECK_CUDA(g, cudaGetLastError());
     }
@@ -379,8 +424,10 @@ extern "C" FGR_API fgr_status fgr_plan(fgr_grid* g, const fgr_nets* nets, int32_
         int blocks = g->num_sms * (occ > 0 ? occ : 1);
         int need = (R + 7) / 8;
         if (blocks > need) blocks = need;
+        ps = fgr_prof_begin(g, PROF_COLOR, st);
         k_color<<<blocks, 256, 0, st>>>(R, box_r, tstart, tend, entries, tiles_x, color, counters + 3, counters + 4,
                                         d_bcount);
+        fgr_prof_end(g, ps, st);
         FGR_CHECK_CUDA(g, cudaGetLastError());
         g->stats.kernel_launches++;
     }
@@ -391,11 +438,13 @@ extern "C" FGR_API fgr_status fgr_plan(fgr_grid* g, const fgr_nets* nets, int32_
         k_batch_keys<<<(R + 255) / 256, 256, 0, st>>>(R, color, keys_s, msize, bkeys);
         FGR_CHECK_CUDA(g, cudaGetLastError());
         tmp_bytes = 0;
-        const int bb = 32 + bits_for(R);
+        const int bb = 42 + bits_for(R);
         cub::DeviceRadixSort::SortKeys(nullptr, tmp_bytes, bkeys, bkeys_s, R, 0, bb, st);
         tmp = fgr_scratch(g->s_plan[8], tmp_bytes, &e);
         if (e != cudaSuccess) return fgr_cuda_fail(g, e, "plan batch sort scratch");
+        ps = fgr_prof_begin(g, PROF_SORT, st);
         FGR_CHECK_CUDA(g, cub::DeviceRadixSort::SortKeys(tmp, tmp_bytes, bkeys, bkeys_s, R, 0, bb, st));
+        fgr_prof_end(g, ps, st);
     }
     tmp_bytes = 0;
     cub::DeviceScan::ExclusiveSum(nullptr, tmp_bytes, d_bcount, batch_offset, R + 1, st);

@@ -11,7 +11,7 @@
 // segment-local prefix P and the segment total ST.  The warp that finishes the
 // last dirty segment of a line (per-line atomic counter) rescans that line's
 // segment totals into the segment bases SB.  Only segments the previous batch
-// committed to are rescanned (dirty list built by the DP's commit), so the bytes
+// committed to are rescanned (byte flags set by the DP's commit), so the bytes
 // moved per batch follow the demand that changed, not the grid size.
 #include "fgr_internal.cuh"
 
@@ -67,9 +67,9 @@ __device__ __forceinline__ void warp_incl_scan(uint32_t (&x)[W]) {
     }
 }
 
+// One segment: ec = len + T[clamp(cap - dem)] per slot, warp scan, write P and ST.
 template <int W>
-__device__ __forceinline__ void refresh_segment(const GridView& g, const DirView& d, int dsel, int line, int s,
-                                                int gs, bool full) {
+__device__ __forceinline__ void refresh_segment(const GridView& g, const DirView& d, int dsel, int line, int s) {
     const int lane = lane_id();
     const int pos = s * FGR_SEG + lane;
     const bool inb = pos < d.len;
@@ -102,19 +102,12 @@ __device__ __forceinline__ void refresh_segment(const GridView& g, const DirView
         Vec<W>::store_u32(d.P + base, p);
     }
     if (lane == 31) Vec<W>::store_u32(d.ST + ((size_t)line * d.nseg + s) * W, incl);
-    const int lidx = d.line_base + line;
-    int last = 0;
-    if (lane == 0) {
-        g.dseg[gs] = 0;
-        __threadfence();
-        unsigned need = full ? (unsigned)d.nseg : g.linecnt[lidx];
-        unsigned old = atomicAdd(&g.linedone[lidx], 1u);
-        last = (old + 1 == need);
-    }
-    last = __shfl_sync(0xffffffffu, last, 0);
-    if (!last) return;
-    __threadfence();
-    // Segment bases of this line: exclusive scan of all segment totals.
+}
+
+// Segment bases of one line: exclusive scan of all its segment totals.
+template <int W>
+__device__ __forceinline__ void rebase_line(const DirView& d, int line) {
+    const int lane = lane_id();
     uint32_t carry[W];
 #pragma unroll
     for (int k = 0; k < W; k++) carry[k] = 0;
@@ -138,28 +131,76 @@ __device__ __forceinline__ void refresh_segment(const GridView& g, const DirView
 #pragma unroll
         for (int k = 0; k < W; k++) carry[k] += __shfl_sync(0xffffffffu, inc[k], 31);
     }
-    if (lane == 0) { g.linedone[lidx] = 0; g.linecnt[lidx] = 0; }
+}
+
+// One task = (line, chunk of 8 segments).  The dirty segments of the chunk are
+// rescanned; the warp finishing the last dirty chunk of the line rebuilds the
+// segment bases and clears the line's flags.  Returns the segments rescanned.
+template <int W>
+__device__ __forceinline__ int refresh_chunk(const GridView& g, const DirView& d, int dsel, int line, int chunk,
+                                             bool full) {
+    const int lane = lane_id();
+    const int lidx = d.line_base + line;
+    if (!full && g.dline[lidx] == 0) return 0;
+    const uint8_t* f = g.dseg + d.seg_base + (size_t)line * d.nseg;
+    const int nchunks = (d.nseg + FGR_CHUNK_SEGS - 1) / FGR_CHUNK_SEGS;
+    // dirty chunks of the line (every task of the line computes the same count)
+    int nd = 0;
+    uint32_t own = 0;
+    for (int c0 = 0; c0 < nchunks; c0 += 32) {
+        const int c = c0 + lane;
+        uint32_t m = 0;
+        if (c < nchunks)
+            for (int q = 0; q < FGR_CHUNK_SEGS; q++) {
+                const int sg = c * FGR_CHUNK_SEGS + q;
+                if (sg < d.nseg && (full || f[sg])) m |= 1u << q;
+            }
+        nd += __popc(__ballot_sync(0xffffffffu, m != 0));
+        const uint32_t o = __shfl_sync(0xffffffffu, m, (chunk - c0) & 31);
+        if (chunk >= c0 && chunk < c0 + 32) own = o;
+    }
+    if (own == 0) return 0;
+    int done = 0;
+    while (own) {
+        const int q = __ffs(own) - 1;
+        own &= own - 1;
+        refresh_segment<W>(g, d, dsel, line, chunk * FGR_CHUNK_SEGS + q);
+        done++;
+    }
+    int last = 0;
+    if (lane == 0) {
+        __threadfence();
+        const unsigned old = atomicAdd(&g.linedone[lidx], 1u);
+        last = (old + 1 == (unsigned)nd);
+    }
+    last = __shfl_sync(0xffffffffu, last, 0);
+    if (last) {
+        __threadfence();
+        rebase_line<W>(d, line);
+        uint8_t* fw = g.dseg + d.seg_base + (size_t)line * d.nseg;
+        for (int sg = lane; sg < d.nseg; sg += 32) fw[sg] = 0;
+        if (lane == 0) { g.dline[lidx] = 0; g.linedone[lidx] = 0; }
+    }
+    return done;
 }
 
 template <int WH, int WV>
-__global__ void __launch_bounds__(256) k_refresh(GridView g, const int32_t* __restrict__ list,
-                                                 const int32_t* __restrict__ count, int full) {
-    const int hsegs = g.h.lines * g.h.nseg;
-    const int ntasks = full ? hsegs + g.v.lines * g.v.nseg : *count;
+__global__ void __launch_bounds__(256) k_refresh(GridView g, int full) {
+    const int chH = (g.h.nseg + FGR_CHUNK_SEGS - 1) / FGR_CHUNK_SEGS;
+    const int chV = (g.v.nseg + FGR_CHUNK_SEGS - 1) / FGR_CHUNK_SEGS;
+    const int tH = g.h.lines * chH;
+    const int ntasks = tH + g.v.lines * chV;
     const int warp = (int)((blockIdx.x * (size_t)blockDim.x + threadIdx.x) >> 5);
     const int nwarps = (int)((gridDim.x * (size_t)blockDim.x) >> 5);
     unsigned nh = 0, nv = 0;
     for (int t = warp; t < ntasks; t += nwarps) {
-        const int gs = full ? t : list[t];
-        if (gs < hsegs) {
-            const int line = gs / g.h.nseg;
-            refresh_segment<WH>(g, g.h, 0, line, gs - line * g.h.nseg, gs, full);
-            nh++;
+        if (t < tH) {
+            const int line = t / chH;
+            nh += refresh_chunk<WH>(g, g.h, 0, line, t - line * chH, full);
         } else {
-            const int r = gs - hsegs;
-            const int line = r / g.v.nseg;
-            refresh_segment<WV>(g, g.v, 1, line, r - line * g.v.nseg, gs, full);
-            nv++;
+            const int r = t - tH;
+            const int line = r / chV;
+            nv += refresh_chunk<WV>(g, g.v, 1, line, r - line * chV, full);
         }
     }
     if (lane_id() == 0 && (nh | nv)) {
@@ -170,17 +211,20 @@ __global__ void __launch_bounds__(256) k_refresh(GridView g, const int32_t* __re
 
 template <int WH, int WV>
 static cudaError_t launch_t(fgr_grid* g, cudaStream_t st, bool full, int blocks) {
-    const int consume = g->parity ^ 1;   // the list the last DP filled
-    k_refresh<WH, WV><<<blocks, 256, 0, st>>>(g->view, g->d_list[consume], g->d_count + consume, full ? 1 : 0);
+    const int ps = fgr_prof_begin(g, PROF_REFRESH, st);
+    k_refresh<WH, WV><<<blocks, 256, 0, st>>>(g->view, full ? 1 : 0);
+    fgr_prof_end(g, ps, st);
     return cudaGetLastError();
 }
 
-// Upper bound on tasks is passed through g->stats.kernel_launches bookkeeping by the caller.
+// One warp per (line, chunk) task; grid capped at 8 CTAs per SM (grid-stride beyond).
 cudaError_t fgr_launch_refresh_sized(fgr_grid* g, cudaStream_t st, bool full, long long max_tasks) {
-    int cap_blocks = g->num_sms * 8;
-    long long tasks = full ? (long long)g->total_segs : max_tasks;
-    if (tasks <= 0) return cudaSuccess;
+    (void)max_tasks;
+    const GridView& v = g->view;
+    const long long tasks = (long long)v.h.lines * ((v.h.nseg + FGR_CHUNK_SEGS - 1) / FGR_CHUNK_SEGS) +
+                            (long long)v.v.lines * ((v.v.nseg + FGR_CHUNK_SEGS - 1) / FGR_CHUNK_SEGS);
     int blocks = (int)((tasks + 7) / 8);
+    const int cap_blocks = g->num_sms * 8;
     if (blocks > cap_blocks) blocks = cap_blocks;
     if (blocks < 1) blocks = 1;
     g->stats.kernel_launches++;
@@ -193,5 +237,5 @@ cudaError_t fgr_launch_refresh_sized(fgr_grid* g, cudaStream_t st, bool full, lo
 }
 
 cudaError_t fgr_launch_refresh(fgr_grid* g, cudaStream_t st, bool full) {
-    return fgr_launch_refresh_sized(g, st, full, (long long)g->total_segs);
+    return fgr_launch_refresh_sized(g, st, full, 0);
 }

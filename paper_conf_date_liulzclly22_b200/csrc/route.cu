@@ -82,8 +82,6 @@ bool nets_equal(const fgr_nets& a, const fgr_nets& b) {
 // the segments the last commit dirtied (bounded by `max_tasks`).
 static cudaError_t refresh_before_dp(fgr_grid* g, cudaStream_t st, long long max_tasks) {
     if (g->full_dirty) {
-        cudaError_t e = cudaMemsetAsync(g->d_count, 0, 2 * sizeof(int32_t), st);
-        if (e != cudaSuccess) return e;
         g->full_dirty = false;
         return fgr_launch_refresh_sized(g, st, true, 0);
     }
@@ -113,7 +111,6 @@ extern "C" FGR_API fgr_status fgr_route_batch(fgr_grid* g, const fgr_nets* nets,
     const NetsView nv = fgr_nets_view(nets);
     FGR_CHECK_CUDA(g, fgr_launch_dp(g, st, nv, list, count, hc[0], hc[2], seg_out, net_cost, nullptr, nullptr,
                                     nullptr, 0, true));
-    fgr_flip_lists(g);
     return FGR_OK;
 }
 
@@ -189,8 +186,7 @@ extern "C" FGR_API fgr_status fgr_route_all(fgr_grid* g, const fgr_nets* nets, c
             const int o0 = c.h_off[b], cnt = c.h_off[b + 1] - o0;
             FGR_CHECK_CUDA(g, fgr_launch_dp(g, st, nv, order + o0, cnt, c.h_nlarge[b], c.h_maxm[b], seg_out,
                                             net_cost, nullptr, nullptr, nullptr, 0, true));
-            fgr_flip_lists(g);
-        }
+                }
         return FGR_OK;
     }
     // ---- multi-GPU: split each batch, exchange route records, commit everywhere
@@ -235,6 +231,7 @@ extern "C" FGR_API fgr_status fgr_route_all(fgr_grid* g, const fgr_nets* nets, c
             ce = fgr_launch_dp(g, st, nv, order + o0 + nl + s0, s1 - s0, 0, 0, nullptr, nullptr, rec, rec_off,
                                rec_cost, o0 + nl + s0, false);
         if (ce != cudaSuccess) { rs = fgr_cuda_fail(g, ce, "dp"); break; }
+        const int ps = fgr_prof_begin(g, PROF_EXCHANGE, st);
         ncclResult_t nr = ncclGroupStart();
         if (nr == ncclSuccess)
             nr = ncclAllReduce(rec + h_roff[b], rec + h_roff[b], (size_t)(h_roff[b + 1] - h_roff[b]), ncclUint32,
@@ -242,6 +239,7 @@ extern "C" FGR_API fgr_status fgr_route_all(fgr_grid* g, const fgr_nets* nets, c
         if (nr == ncclSuccess)
             nr = ncclAllReduce(rec_cost + o0, rec_cost + o0, (size_t)cnt, ncclUint32, ncclSum, g->comm, st);
         ncclResult_t ne = ncclGroupEnd();
+        fgr_prof_end(g, ps, st);
         if (nr != ncclSuccess || ne != ncclSuccess) {
             g->broken = true;
             rs = fgr_set_error(FGR_ERR_NCCL, "NCCL all-reduce failed: %s", ncclGetErrorString(nr != ncclSuccess ? nr : ne));
@@ -249,8 +247,7 @@ extern "C" FGR_API fgr_status fgr_route_all(fgr_grid* g, const fgr_nets* nets, c
         }
         ce = fgr_launch_commit(g, st, nv, order + o0, cnt, rec, rec_off, o0);
         if (ce != cudaSuccess) { rs = fgr_cuda_fail(g, ce, "commit"); break; }
-        fgr_flip_lists(g);
-    }
+        }
     free(h_roff);
     if (rs != FGR_OK) return rs;
     if (R > 0) {

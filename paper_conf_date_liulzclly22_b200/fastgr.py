@@ -24,7 +24,10 @@ STATUS_NAMES = ["OK", "INVALID", "RANGE", "OOM", "CUDA", "NCCL", "STATE"]
 # every entry point include/fastgr.h declares
 EXPORTS = ["fgr_last_error", "fgr_version", "fgr_cost_table", "fgr_grid_create", "fgr_grid_destroy",
            "fgr_grid_set_demand", "fgr_grid_get_demand", "fgr_plan", "fgr_route_batch", "fgr_route_all",
-           "fgr_comm_unique_id", "fgr_comm_init", "fgr_run_host", "fgr_get_stats"]
+           "fgr_comm_unique_id", "fgr_comm_init", "fgr_run_host", "fgr_get_stats", "fgr_profile_enable",
+           "fgr_profile_read"]
+PROF_CLASSES = ["refresh", "dp_small", "dp_large", "commit", "plan_preprocess", "plan_sort", "plan_color",
+                "plan_other", "exchange"]
 
 
 class FgrError(RuntimeError):
@@ -76,6 +79,8 @@ def lib():
             "fgr_comm_init": ([P, P, S, S], S),
             "fgr_run_host": ([P, I, I, P, P, P, P, P, P, P, P, P, P], S),
             "fgr_get_stats": ([P, P], S),
+            "fgr_profile_enable": ([P, S], S),
+            "fgr_profile_read": ([P, P, P], S),
         }
         for name, (args, res) in sig.items():
             f = getattr(L, name)
@@ -192,6 +197,17 @@ def fgr_get_stats(h) -> dict:
     s = fgr_stats()
     _check(lib().fgr_get_stats(h, ctypes.byref(s)))
     return {k: getattr(s, k) for k, _ in fgr_stats._fields_}
+
+
+def fgr_profile_enable(h, enable=True):
+    _check(lib().fgr_profile_enable(h, 1 if enable else 0))
+
+
+def fgr_profile_read(h) -> dict:
+    ms = np.zeros(len(PROF_CLASSES), np.float64)
+    n = np.zeros(len(PROF_CLASSES), np.int64)
+    _check(lib().fgr_profile_read(h, ms.ctypes.data, n.ctypes.data))
+    return {c: (float(ms[i]), int(n[i])) for i, c in enumerate(PROF_CLASSES)}
 
 
 # ----------------------------------------------------------------- conveniences (marshalling only)
