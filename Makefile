@@ -11,7 +11,7 @@ NCCL_LIB := $(SITE)/nccl/lib
 PKG     := paper_conf_date_liulzclly22_b200
 CSRC    := $(PKG)/csrc
 ARCH    := -gencode arch=compute_100a,code=sm_100a
-NVFLAGS := -O3 -std=c++17 $(ARCH) -lineinfo -Xcompiler -fPIC -Xcompiler -fvisibility=hidden \
+NVFLAGS := $(EXTRA) -O3 -std=c++17 $(ARCH) -lineinfo -Xcompiler -fPIC -Xcompiler -fvisibility=hidden \
            -Iinclude -I$(NCCL_INC) --expt-relaxed-constexpr -Xptxas -v
 CFLAGS  := -O2 -std=c11 -fPIC -Wall -Wextra -Wno-unused-parameter
 

@@ -130,21 +130,25 @@ struct Out {
     int list_base;
 };
 
-// Per-lane constants of the group lane that owns layer `gl`.
+// Per-lane constants of the group lane that owns layer `gl` (= lo in span_rows, = lt in edge_table).
 template <int LT>
 struct LaneConst {
-    uint32_t vp[LT + 1];   // via prefix: V(lo,hi) = vp[hi] - vp[lo]
+    uint32_t vme[LT];      // V(min(l, gl), max(l, gl)): via stack between layer l and this lane's layer
     uint32_t hmask;        // layers with dir == H
     int my_dir, my_slot;
     __device__ __forceinline__ void load(const Hdr* h, int gl) {
+        const int me = gl < LT ? gl : 0;
+        const uint32_t vpm = h->viapre[me];
 #pragma unroll
-        for (int i = 0; i <= LT; i++) vp[i] = h->viapre[i];
+        for (int i = 0; i < LT; i++) {
+            const uint32_t vi = h->viapre[i];
+            vme[i] = vi >= vpm ? vi - vpm : vpm - vi;   // viapre is non-decreasing
+        }
         hmask = 0;
 #pragma unroll
         for (int i = 0; i < LT; i++) hmask |= (h->dir[i] == 0 ? 1u : 0u) << i;
-        const int l = gl < LT ? gl : 0;
-        my_dir = h->dir[l];
-        my_slot = h->slot[l];
+        my_dir = h->dir[me];
+        my_slot = h->slot[me];
     }
 };
 
@@ -196,7 +200,7 @@ __device__ __forceinline__ void span_rows(const LaneConst<LT>& c, const Tabs& t,
     if (!act) return;
     uint32_t acc[LT];
 #pragma unroll
-    for (int hi = 0; hi < LT; hi++) acc[hi] = hi >= lo ? c.vp[hi] - c.vp[lo] : FGR_INF;
+    for (int hi = 0; hi < LT; hi++) acc[hi] = hi >= lo ? c.vme[hi] : FGR_INF;   // lo == this lane's layer
     auto add_child = [&](int ch) {
         const uint32_t* Ec = t.E + (size_t)ch * LT;
         uint32_t run = FGR_INF;
@@ -268,15 +272,11 @@ __device__ __forceinline__ void edge_table(const LaneConst<LT>& c, const Tabs& t
         const uint32_t leg2 = b0 ? t.legV[((size_t)v * 2 + 1) * nV + c.my_slot] : t.legH[((size_t)v * 2 + 1) * nH + c.my_slot];
         const uint32_t* l1 = b0 ? t.legH + (size_t)v * 2 * nH : t.legV + (size_t)v * 2 * nV;
         const uint32_t opp = b0 ? c.hmask : ~c.hmask;
-        uint32_t vplt = 0;
-#pragma unroll
-        for (int l = 0; l < LT; l++)
-            if (l == lt) vplt = c.vp[l];
         int s = 0;
 #pragma unroll
         for (int ls = 0; ls < LT; ls++)
             if ((opp >> ls) & 1u) {
-                const uint32_t via = ls < lt ? vplt - c.vp[ls] : c.vp[ls] - vplt;
+                const uint32_t via = c.vme[ls];   // lt == this lane's layer
                 const uint32_t cst = sat_add(sat_add(sat_add(w.B[ls], l1[s]), via), leg2);
                 if (cst < best) { best = cst; bls = ls; }
                 s++;
@@ -538,8 +538,14 @@ __global__ void __launch_bounds__(32 * kGroupWarps) k_dp_group(GridView g, NetsV
 }
 
 // ------------------------------------------------------------- CTA kernel (nets > 32 nodes)
+#ifdef FGR_TIMING
+#define TMARK(i) do { if (threadIdx.x == 0) tm[i] = clock64(); } while (0)
+#else
+#define TMARK(i) do { } while (0)
+#endif
+
 template <int LT>
-__global__ void __launch_bounds__(FGR_CTA_THREADS) k_dp_large(GridView g, NetsView nv, const int32_t* __restrict__ list,
+__global__ void __launch_bounds__(FGR_CTA_THREADS, 1) k_dp_large(GridView g, NetsView nv, const int32_t* __restrict__ list,
                                                                int count, Out o, int commit) {
     constexpr int G = groups_of(LT);
     extern __shared__ __align__(16) unsigned char smem[];
@@ -554,6 +560,10 @@ __global__ void __launch_bounds__(FGR_CTA_THREADS) k_dp_large(GridView g, NetsVi
     const int gl = lane - gi * LT;
     const bool glane = gi < G && gl < LT;
     const int idx = blockIdx.x;
+#ifdef FGR_TIMING
+    long long tm[8];
+#endif
+    TMARK(0);
     const int net = list[idx];
     const int a0 = nv.off[net];
     const int m = nv.off[net + 1] - a0;
@@ -626,27 +636,57 @@ __global__ void __launch_bounds__(FGR_CTA_THREADS) k_dp_large(GridView g, NetsVi
         t.anc[atomicAdd(&dcnt[t.depth[i]], 1u)] = (uint16_t)i;   // nodes grouped by level
     }
     __syncthreads();
+    TMARK(1);
 #pragma unroll 2
     for (int task = tid; task < 4 * (m - 1); task += T) gather_task(g, t, task);
     __syncthreads();
+    TMARK(2);
     // bottom-up DP: 8 warps x G groups evaluate nodes of one level side by side
     constexpr int SLOTS = FGR_WARPS_PER_CTA * G;
     const int myslot = warp * G + gi;
+#ifdef FGR_TIMING
+    long long ph[4] = {0, 0, 0, 0};
+#endif
     for (int d = maxd; d >= 1; d--) {
         const int k0 = t.lvstart[d], k1 = t.lvstart[d + 1];
         for (int kb = k0; kb < k1; kb += SLOTS) {
             const int k = kb + myslot;
             const bool act = glane && k < k1;
             const int v = act ? t.anc[k] : 0;
+#ifdef FGR_TIMING
+            long long q0 = clock64();
+#endif
             span_rows<LT, true>(c, t, w, v, gl, act);
             __syncwarp();
+#ifdef FGR_TIMING
+            long long q1 = clock64();
+#endif
             node_table<LT>(t, w, v, gl, act);
             __syncwarp();
+#ifdef FGR_TIMING
+            long long q2 = clock64();
+#endif
             edge_table<LT>(c, t, w, v, gl, nH, nV, act);
             __syncwarp();
+#ifdef FGR_TIMING
+            long long q3 = clock64();
+            if (kb == k0) { ph[0] += q1 - q0; ph[1] += q2 - q1; ph[2] += q3 - q2; }
+#endif
         }
+#ifdef FGR_TIMING
+        long long q4 = clock64();
+#endif
         __syncthreads();
+#ifdef FGR_TIMING
+        ph[3] += clock64() - q4;
+#endif
     }
+#ifdef FGR_TIMING
+    if (tid == 0 && m > 880)
+        printf("LEVELS m=%d maxd=%d span=%lld node=%lld edge=%lld barrier=%lld (cycles summed over levels, warp 0)\n", m,
+               maxd, ph[0], ph[1], ph[2], ph[3]);
+#endif
+    TMARK(3);
     if (warp == 0) {
         const bool act = glane && gi == 0;
         span_rows<LT, true>(c, t, w, 0, gl, act);
@@ -657,6 +697,7 @@ __global__ void __launch_bounds__(FGR_CTA_THREADS) k_dp_large(GridView g, NetsVi
     __syncthreads();
     if (tid == 0) t.span[0] = (uint8_t)(s_root & 0xFF);
     __syncthreads();
+    TMARK(4);
     for (int d = 1; d <= maxd; d++) {
         const int k1 = t.lvstart[d + 1];
         for (int k = t.lvstart[d] + tid; k < k1; k += T) {
@@ -668,6 +709,7 @@ __global__ void __launch_bounds__(FGR_CTA_THREADS) k_dp_large(GridView g, NetsVi
         }
         __syncthreads();
     }
+    TMARK(5);
     // S6 for the whole net in one pass (the atomics' latencies overlap across threads)
     if (commit)
         for (int i = 1 + tid; i < m; i += T) {
@@ -675,6 +717,13 @@ __global__ void __launch_bounds__(FGR_CTA_THREADS) k_dp_large(GridView g, NetsVi
             const int u = t.par[i];
             commit_edge(g, h, t.x[i], t.y[i], t.x[u], t.y[u], s);
         }
+#ifdef FGR_TIMING
+    __syncthreads();
+    TMARK(6);
+    if (tid == 0 && m > 600)
+        printf("TIMING m=%d maxd=%d prologue=%lld gather=%lld dp=%lld root=%lld backtrack=%lld commit=%lld\n", m, maxd,
+               tm[1] - tm[0], tm[2] - tm[1], tm[3] - tm[2], tm[4] - tm[3], tm[5] - tm[4], tm[6] - tm[5]);
+#endif
     if (tid == 0) {
         const uint32_t total = (uint32_t)(s_root >> 8);
         if (o.rec_seg) { o.rec_seg[o.rec_off[o.list_base + idx]] = 0xFFFFFFFFu; o.rec_cost[o.list_base + idx] = total; }

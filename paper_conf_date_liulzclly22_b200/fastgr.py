@@ -15,7 +15,7 @@ from typing import Optional
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libfastgr.so")
+LIB_PATH = os.environ.get("FGR_LIB_PATH") or os.path.join(_HERE, "libfastgr.so")
 _LIB = None
 
 FGR_OK, FGR_ERR_INVALID, FGR_ERR_RANGE, FGR_ERR_OOM, FGR_ERR_CUDA, FGR_ERR_NCCL, FGR_ERR_STATE = range(7)
