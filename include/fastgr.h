@@ -153,14 +153,21 @@ FGR_API fgr_status fgr_route_batch(fgr_grid* grid, const fgr_nets* nets, const i
  * order/batch_offset/num_batches as returned by fgr_plan for the same nets.
  * seg_out [num_nodes] and net_cost [num_nets] are fully written (trivial nets:
  * seg 0xFFFFFFFF, cost 0).  With a communicator (fgr_comm_init, world > 1),
- * each batch's nets are split across ranks and the routes are exchanged with
- * one NCCL all-reduce per batch; every rank ends with identical outputs and
- * demand, bitwise equal to world = 1.  No host synchronisation when the
+ * each batch's nets are split across ranks (fgr_split_batch) and the routes are
+ * exchanged with one NCCL all-reduce per batch; every rank ends with identical
+ * outputs and demand, bitwise equal to world = 1.  (A communicator of world 1
+ * takes the same exchange path, which is how it is tested on one GPU.)  No host synchronisation when the
  * arguments are those of the grid's last fgr_plan call.
  */
 FGR_API fgr_status fgr_route_all(fgr_grid* grid, const fgr_nets* nets, const int32_t* order,
                                  const int32_t* batch_offset, int32_t num_batches, uint32_t* seg_out,
                                  uint32_t* net_cost, void* stream);
+
+/* The multi-GPU split rule fgr_route_all applies to one batch (host-only, no GPU):
+ * the batch's `count` nets are ordered large nets first (`nlarge` of them); rank r
+ * of `world` routes the large nets [out[0], out[1]) and the small nets
+ * [out[2], out[3]) (indices into the batch).  Contiguous, disjoint, covering. */
+FGR_API fgr_status fgr_split_batch(int32_t count, int32_t nlarge, int32_t rank, int32_t world, int32_t* out4);
 
 /* Multi-GPU (one process per GPU).  fgr_comm_unique_id fills 128 bytes on the
  * root rank; broadcast them (e.g. torch.distributed) and call fgr_comm_init on

@@ -88,6 +88,17 @@ static cudaError_t refresh_before_dp(fgr_grid* g, cudaStream_t st, long long max
     return fgr_launch_refresh_sized(g, st, false, max_tasks);
 }
 
+extern "C" FGR_API fgr_status fgr_split_batch(int32_t count, int32_t nlarge, int32_t rank, int32_t world, int32_t* out) {
+    if (!out || count < 0 || nlarge < 0 || nlarge > count || world < 1 || rank < 0 || rank >= world)
+        return fgr_set_error(FGR_ERR_INVALID, "bad split arguments");
+    const long long ns = count - nlarge;
+    out[0] = (int32_t)((long long)nlarge * rank / world);
+    out[1] = (int32_t)((long long)nlarge * (rank + 1) / world);
+    out[2] = nlarge + (int32_t)(ns * rank / world);
+    out[3] = nlarge + (int32_t)(ns * (rank + 1) / world);
+    return FGR_OK;
+}
+
 extern "C" FGR_API fgr_status fgr_route_batch(fgr_grid* g, const fgr_nets* nets, const int32_t* net_ids, int32_t count,
                                               uint32_t* seg_out, uint32_t* net_cost, void* stream) {
     if (!g || !nets) return fgr_set_error(FGR_ERR_INVALID, "NULL argument");
@@ -179,7 +190,7 @@ extern "C" FGR_API fgr_status fgr_route_all(fgr_grid* g, const fgr_nets* nets, c
     g->stats.dp_nets = B > 0 ? c.h_off[B] : 0;
     g->stats.kernel_launches = 0;
     FGR_CHECK_CUDA(g, cudaMemsetAsync(g->d_stats, 0, 4 * sizeof(unsigned long long), st));
-    if (g->world <= 1) {
+    if (!g->comm) {
         for (int b = 0; b < B; b++) {
             const long long bound = b > 0 ? c.h_segb[b - 1] : (long long)g->total_segs;
             FGR_CHECK_CUDA(g, refresh_before_dp(g, st, bound));
@@ -190,7 +201,6 @@ extern "C" FGR_API fgr_status fgr_route_all(fgr_grid* g, const fgr_nets* nets, c
         return FGR_OK;
     }
     // ---- multi-GPU: split each batch, exchange route records, commit everywhere
-    if (!g->comm) return fgr_set_error(FGR_ERR_STATE, "world > 1 without a communicator");
     cudaError_t e;
     const int R = B > 0 ? c.h_off[B] : 0;
     int32_t* rec_off = (int32_t*)fgr_scratch(g->s_rec[2], sizeof(int32_t) * ((size_t)R + 1) * 2 + 64, &e);
@@ -220,16 +230,15 @@ extern "C" FGR_API fgr_status fgr_route_all(fgr_grid* g, const fgr_nets* nets, c
         const long long bound = b > 0 ? c.h_segb[b - 1] : (long long)g->total_segs;
         cudaError_t ce = refresh_before_dp(g, st, bound);
         if (ce != cudaSuccess) { rs = fgr_cuda_fail(g, ce, "refresh"); break; }
-        const int o0 = c.h_off[b], cnt = c.h_off[b + 1] - o0, nl = c.h_nlarge[b], ns = cnt - nl;
-        // contiguous chunks of the large and of the small nets per rank
-        const int l0 = (int)((long long)nl * g->rank / g->world), l1 = (int)((long long)nl * (g->rank + 1) / g->world);
-        const int s0 = (int)((long long)ns * g->rank / g->world), s1 = (int)((long long)ns * (g->rank + 1) / g->world);
-        if (l1 > l0)
-            ce = fgr_launch_dp(g, st, nv, order + o0 + l0, l1 - l0, l1 - l0, c.h_maxm[b], nullptr, nullptr, rec,
-                               rec_off, rec_cost, o0 + l0, false);
-        if (ce == cudaSuccess && s1 > s0)
-            ce = fgr_launch_dp(g, st, nv, order + o0 + nl + s0, s1 - s0, 0, 0, nullptr, nullptr, rec, rec_off,
-                               rec_cost, o0 + nl + s0, false);
+        const int o0 = c.h_off[b], cnt = c.h_off[b + 1] - o0, nl = c.h_nlarge[b];
+        int32_t sp[4];
+        fgr_split_batch(cnt, nl, g->rank, g->world, sp);
+        if (sp[1] > sp[0])
+            ce = fgr_launch_dp(g, st, nv, order + o0 + sp[0], sp[1] - sp[0], sp[1] - sp[0], c.h_maxm[b], nullptr,
+                               nullptr, rec, rec_off, rec_cost, o0 + sp[0], false);
+        if (ce == cudaSuccess && sp[3] > sp[2])
+            ce = fgr_launch_dp(g, st, nv, order + o0 + sp[2], sp[3] - sp[2], 0, 0, nullptr, nullptr, rec, rec_off,
+                               rec_cost, o0 + sp[2], false);
         if (ce != cudaSuccess) { rs = fgr_cuda_fail(g, ce, "dp"); break; }
         const int ps = fgr_prof_begin(g, PROF_EXCHANGE, st);
         ncclResult_t nr = ncclGroupStart();

@@ -25,7 +25,7 @@ STATUS_NAMES = ["OK", "INVALID", "RANGE", "OOM", "CUDA", "NCCL", "STATE"]
 EXPORTS = ["fgr_last_error", "fgr_version", "fgr_cost_table", "fgr_grid_create", "fgr_grid_destroy",
            "fgr_grid_set_demand", "fgr_grid_get_demand", "fgr_plan", "fgr_route_batch", "fgr_route_all",
            "fgr_comm_unique_id", "fgr_comm_init", "fgr_run_host", "fgr_get_stats", "fgr_profile_enable",
-           "fgr_profile_read"]
+           "fgr_profile_read", "fgr_split_batch"]
 PROF_CLASSES = ["refresh", "dp_small", "dp_large", "commit", "plan_preprocess", "plan_sort", "plan_color",
                 "plan_other", "exchange"]
 
@@ -81,6 +81,7 @@ def lib():
             "fgr_get_stats": ([P, P], S),
             "fgr_profile_enable": ([P, S], S),
             "fgr_profile_read": ([P, P, P], S),
+            "fgr_split_batch": ([I, I, I, I, P], S),
         }
         for name, (args, res) in sig.items():
             f = getattr(L, name)
@@ -197,6 +198,13 @@ def fgr_get_stats(h) -> dict:
     s = fgr_stats()
     _check(lib().fgr_get_stats(h, ctypes.byref(s)))
     return {k: getattr(s, k) for k, _ in fgr_stats._fields_}
+
+
+def fgr_split_batch(count, nlarge, rank, world):
+    """(large_lo, large_hi, small_lo, small_hi) of `rank` for one batch (host-only)."""
+    out = np.zeros(4, np.int32)
+    _check(lib().fgr_split_batch(int(count), int(nlarge), int(rank), int(world), out.ctypes.data))
+    return tuple(int(v) for v in out)
 
 
 def fgr_profile_enable(h, enable=True):

@@ -186,3 +186,17 @@ def test_invalid_nets_rejected():
 def test_t9_full_size_bit_exact():
     """BASELINE.json's headline config at full size (~900k nets), as bench.py runs it."""
     check_against_oracle(gen.make_config("t9"))
+
+
+@pytest.mark.parametrize("cfg", ["tiny", "t5"])
+def test_exchange_path_world1_bit_exact(cfg):
+    """The multi-GPU path (split -> route records -> NCCL all-reduce -> commit from
+    records) run with a world-1 NCCL communicator on one GPU."""
+    from paper_conf_date_liulzclly22_b200 import fastgr as F
+    d = gen.make_config(cfg)
+    r = _router(d)
+    F.fgr_comm_init(r.h, F.fgr_comm_unique_id(), 0, 1)
+    check_against_oracle(d, r=r)
+    st = F.fgr_get_stats(r.h)
+    assert st["world"] == 1
+    r.close()
