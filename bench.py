@@ -46,6 +46,21 @@ def peaks():
         return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
+def committed_traffic(kernel_class):
+    """DRAM bytes per launch of a kernel class from the newest committed ncu capture
+    (profiles/<tag>_traffic.json, written by tools/summarize_profiles.py), or None."""
+    import glob
+    files = sorted(glob.glob(os.path.join(ROOT, "profiles", "*_traffic.json")), key=os.path.getmtime)
+    for f in reversed(files):
+        try:
+            j = json.load(open(f))
+            if kernel_class in j.get("bytes_per_launch", {}):
+                return j["bytes_per_launch"][kernel_class], os.path.relpath(f, ROOT)
+        except Exception:
+            continue
+    return None, None
+
+
 def design_stats(d):
     """Per-design algorithmic quantities (independent of the routes chosen)."""
     sizes = d.net_sizes()
@@ -276,8 +291,9 @@ def main():
         per_launch = alg_bytes_step * steps / dom_n
         avg_s = dom_ms / dom_n / 1000.0
         ach = per_launch / avg_s / 1e9
+        traffic, tsrc = committed_traffic(dom)
         roof = {"bound": "hbm", "kernel": dom, "achieved": ach, "peak": peak, "unit": "GB/s", "frac": ach / peak,
-                "traffic": None, "bytes_per_launch": per_launch, "avg_launch_us": avg_s * 1e6,
+                "traffic": traffic, "traffic_source": tsrc, "bytes_per_launch": per_launch, "avg_launch_us": avg_s * 1e6,
                 "launches_per_step": dom_n / steps, "share_of_step": dom_ms / steps / ms_per_step,
                 "peak_source": peak_src, "byte_model": unit_note}
 
