@@ -30,6 +30,7 @@ namespace {
 
 constexpr int kMC = FGR_SMALL_NET;          // node capacity of one group in k_dp_group
 constexpr int kGroupWarps = 4;              // warps per CTA in k_dp_group
+constexpr int kLargeWarps = 16;             // warps per CTA in k_dp_large (one path-walking group each)
 
 __host__ __device__ constexpr int groups_of(int LT) { return (32 / LT) < 4 ? (32 / LT) : 4; }
 __host__ __device__ inline size_t a16(size_t b) { return (b + 15) & ~(size_t)15; }
@@ -38,6 +39,7 @@ struct Hdr {                  // per-block constants copied to shared memory
     uint32_t viapre[FGR_MAXL + 1];
     uint8_t dir[FGR_MAXL];
     uint8_t slot[FGR_MAXL];
+    uint8_t zlo[FGR_MAXL];    // smallest lo with V(lo, a) == 0 (zero-cost via run below a)
 };
 
 struct Tabs {
@@ -53,6 +55,12 @@ struct Tabs {
     uint16_t* clist;  // CTA path: [m]
     uint16_t* anc;    // CTA path: pointer-jumping scratch [m], then the nodes sorted by level
     uint16_t* lvstart;// CTA path: level CSR [m+1]
+    uint16_t* hv;     // CTA path: heavy child (0xFFFF = leaf)
+    uint16_t* top;    // CTA path: top node of the heavy path holding v
+    uint16_t* bot;    // CTA path: bottom (leaf) of the path topped by v
+    uint16_t* pq;     // CTA path: path tops, deepest top first
+    uint8_t* done;    // CTA path: E_v final (values pass)
+    uint8_t* sready;  // CTA path: span_v final (backtrack)
     int8_t* plo;
     int8_t* phi;
     uint8_t* span;    // chosen via span (lo << 4) | hi  (low byte of the packed (value, lo, hi) key)
@@ -72,7 +80,7 @@ __host__ __device__ inline size_t tabs_bytes(int m, int L, int nH, int nV, bool 
     b += a16((size_t)m * 2 * nV * 4);
     if (!cta) b += a16((size_t)m * 4);
     b += 4 * a16((size_t)m * 2);
-    if (cta) b += 2 * a16((size_t)(m + 1) * 2) + 2 * a16((size_t)m * 2);
+    if (cta) b += 2 * a16((size_t)(m + 1) * 2) + 6 * a16((size_t)m * 2) + 2 * a16((size_t)m);
     b += 3 * a16((size_t)m);
     b += 2 * a16((size_t)m * L);
     return b;
@@ -91,12 +99,19 @@ __device__ inline Tabs carve_tabs(unsigned char* p, int m, int L, int nH, int nV
     t.y = (int16_t*)p; p += a16((size_t)m * 2);
     t.par = (int16_t*)p; p += a16((size_t)m * 2);
     t.depth = (uint16_t*)p; p += a16((size_t)m * 2);
-    t.cstart = t.clist = t.anc = t.lvstart = nullptr;
+    t.cstart = t.clist = t.anc = t.lvstart = t.hv = t.top = t.bot = t.pq = nullptr;
+    t.done = t.sready = nullptr;
     if (cta) {
         t.cstart = (uint16_t*)p; p += a16((size_t)(m + 1) * 2);
         t.lvstart = (uint16_t*)p; p += a16((size_t)(m + 1) * 2);
         t.clist = (uint16_t*)p; p += a16((size_t)m * 2);
         t.anc = (uint16_t*)p; p += a16((size_t)m * 2);
+        t.hv = (uint16_t*)p; p += a16((size_t)m * 2);
+        t.top = (uint16_t*)p; p += a16((size_t)m * 2);
+        t.bot = (uint16_t*)p; p += a16((size_t)m * 2);
+        t.pq = (uint16_t*)p; p += a16((size_t)m * 2);
+        t.done = (uint8_t*)p; p += a16((size_t)m);
+        t.sready = (uint8_t*)p; p += a16((size_t)m);
     }
     t.plo = (int8_t*)p; p += a16((size_t)m);
     t.phi = (int8_t*)p; p += a16((size_t)m);
@@ -118,6 +133,9 @@ __device__ inline void init_hdr(Hdr* h, const GridView& g) {
     for (int i = threadIdx.x; i < FGR_MAXL; i += blockDim.x) {
         h->dir[i] = g.dir[i];
         h->slot[i] = g.slot[i];
+        int z = i;
+        while (z > 0 && g.viapre[z - 1] == g.viapre[i]) z--;
+        h->zlo[i] = (uint8_t)z;
     }
 }
 
@@ -134,6 +152,8 @@ struct Out {
 template <int LT>
 struct LaneConst {
     uint32_t vme[LT];      // V(min(l, gl), max(l, gl)): via stack between layer l and this lane's layer
+    uint32_t vp[LT];       // viapre[l]       (indexed only by compile-time l)
+    uint32_t zl[LT];       // zlo[l]
     uint32_t hmask;        // layers with dir == H
     int my_dir, my_slot;
     __device__ __forceinline__ void load(const Hdr* h, int gl) {
@@ -142,6 +162,8 @@ struct LaneConst {
 #pragma unroll
         for (int i = 0; i < LT; i++) {
             const uint32_t vi = h->viapre[i];
+            vp[i] = vi;
+            zl[i] = h->zlo[i];
             vme[i] = vi >= vpm ? vi - vpm : vpm - vi;   // viapre is non-decreasing
         }
         hmask = 0;
@@ -538,27 +560,49 @@ __global__ void __launch_bounds__(32 * kGroupWarps) k_dp_group(GridView g, NetsV
 }
 
 // ------------------------------------------------------------- CTA kernel (nets > 32 nodes)
+// Heavy-path form of the same recurrences.  Split the tree into heavy paths (heavy
+// child = largest subtree).  With every child of v known except the heavy child h,
+// Eq. (2) becomes a min-plus product in E_h:
+//     B_v(ls) = min_l [ E_h(l) + G_v(min(l, a), max(l, b)) ],  a = min(ls, pin_lo), b = max(ls, pin_hi)
+// where K_v(S) = V(S) + sum_{light c} min_{l in S} E_c(l) and G_v(a, b) = min over spans
+// S = [lo, hi] with lo <= a, hi >= b of K_v(S).  Carrying packed (value, lo, hi) keys
+// through G and through the min over l reproduces R11's lexicographic span choice
+// exactly (the optimal span is S*_l of some optimal l).  Without light
+// children K = V and G has a closed form.  A path is then walked bottom-up by one
+// lane group with one short vector step per node, and paths run as a dataflow (a
+// node waits only for its light children), so the CTA never synchronises per
+// tree level.  The backtrack walks the same paths top-down.
+
 #ifdef FGR_TIMING
 #define TMARK(i) do { if (threadIdx.x == 0) tm[i] = clock64(); } while (0)
 #else
 #define TMARK(i) do { } while (0)
 #endif
 
+// Packed G entry of a node without light children (K = V): value V(a,b), span (zlo[a], b).
+__device__ __forceinline__ unsigned long long gclosed(const Hdr* h, int a, int b) {
+    return ((unsigned long long)(h->viapre[b] - h->viapre[a]) << 8) | (unsigned)(h->zlo[a] << 4) | (unsigned)b;
+}
+
+__device__ __forceinline__ int ld_flag(const uint8_t* f) { return *(volatile const uint8_t*)f; }
+
 template <int LT>
-__global__ void __launch_bounds__(FGR_CTA_THREADS, 1) k_dp_large(GridView g, NetsView nv, const int32_t* __restrict__ list,
-                                                               int count, Out o, int commit) {
-    constexpr int G = groups_of(LT);
+__global__ void __launch_bounds__(32 * kLargeWarps, 1) k_dp_large(GridView g, NetsView nv, const int32_t* __restrict__ list,
+                                                                  int count, Out o, int commit) {
+    constexpr int G = 1;   // one lane group per warp: a path walk never shares its warp's issue slots
     extern __shared__ __align__(16) unsigned char smem[];
     Hdr* h = reinterpret_cast<Hdr*>(smem);
-    __shared__ int s_maxd;
+    __shared__ int s_maxd, s_ticket, s_ticket2, s_npaths;
     __shared__ unsigned long long s_root;
     init_hdr(h, g);
-    if (threadIdx.x == 0) { s_maxd = 0; s_root = ~0ull; }
+    if (threadIdx.x == 0) { s_maxd = 0; s_root = ~0ull; s_ticket = 0; s_ticket2 = 0; s_npaths = 0; }
     const int nH = g.h.cnt, nV = g.v.cnt;
     const int warp = threadIdx.x >> 5, lane = lane_id(), tid = threadIdx.x, T = blockDim.x;
     const int gi = lane / LT < G ? lane / LT : G;
     const int gl = lane - gi * LT;
     const bool glane = gi < G && gl < LT;
+    const int gbase = gi * LT;
+    const unsigned gmask = glane ? (((1u << LT) - 1u) << gbase) : 0u;
     const int idx = blockIdx.x;
 #ifdef FGR_TIMING
     long long tm[8];
@@ -569,15 +613,16 @@ __global__ void __launch_bounds__(FGR_CTA_THREADS, 1) k_dp_large(GridView g, Net
     const int m = nv.off[net + 1] - a0;
     unsigned char* base = smem + a16(sizeof(Hdr));
     const WScr w = carve_wscr(base + ((size_t)warp * G + (gi < G ? gi : 0)) * wscr_bytes(LT), LT);
-    const Tabs t = carve_tabs(base + (size_t)FGR_WARPS_PER_CTA * G * wscr_bytes(LT), m, LT, nH, nV, true);
+    const Tabs t = carve_tabs(base + (size_t)kLargeWarps * G * wscr_bytes(LT), m, LT, nH, nV, true);
     for (int i = tid; i < m; i += T) {
         const int p = nv.par[a0 + i];
         t.x[i] = nv.x[a0 + i]; t.y[i] = nv.y[a0 + i]; t.par[i] = (int16_t)p;
         t.plo[i] = nv.plo[a0 + i]; t.phi[i] = nv.phi[a0 + i];
         t.depth[i] = i ? 1 : 0;
         t.anc[i] = (uint16_t)(i ? p : 0);
+        t.done[i] = 0; t.sready[i] = 0;
     }
-    uint32_t* cnt = t.legH;   // child counts and level counts reuse the leg areas before the gathers
+    uint32_t* cnt = t.legH;   // scratch in the leg areas before the gathers
     uint32_t* dcnt = t.legV;
     for (int i = tid; i <= m; i += T) { cnt[i] = 0; dcnt[i] = 0; }
     __syncthreads();
@@ -633,96 +678,366 @@ __global__ void __launch_bounds__(FGR_CTA_THREADS, 1) k_dp_large(GridView g, Net
     __syncthreads();
     for (int i = tid; i < m; i += T) {
         if (i > 0) t.clist[atomicAdd(&cnt[t.par[i]], 1u)] = (uint16_t)i;
-        t.anc[atomicAdd(&dcnt[t.depth[i]], 1u)] = (uint16_t)i;   // nodes grouped by level
+        t.anc[atomicAdd(&dcnt[t.depth[i]], 1u)] = (uint16_t)i;   // nodes grouped by level, shallow first
     }
     __syncthreads();
+    // Path decomposition: the ancestors of the deepest node (ties: smallest index)
+    // form the root path, every other node continues through its smallest-index
+    // child.  Any decomposition is exact; this one puts the deepest chain on one path.
+    __shared__ int s_deep;
+    if (tid == 0) s_deep = 0x7FFFFFFF;
+    __syncthreads();
+    for (int v = tid; v < m; v += T)
+        if (t.depth[v] == maxd) atomicMin(&s_deep, v);
+    for (int v = tid; v < m; v += T) {
+        int best = -1;
+        for (int k = t.cstart[v]; k < t.cstart[v + 1]; k++) {
+            const int ch = t.clist[k];
+            if (best < 0 || ch < best) best = ch;
+        }
+        t.hv[v] = best < 0 ? (uint16_t)0xFFFF : (uint16_t)best;
+    }
+    __syncthreads();
+    if (tid == 0)
+        for (int w = s_deep; w > 0; w = t.par[w]) t.hv[t.par[w]] = (uint16_t)w;
+    __syncthreads();
+    // top of each node's heavy path by pointer jumping over heavy edges
+    for (int v = tid; v < m; v += T) t.top[v] = (v > 0 && t.hv[t.par[v]] == v) ? (uint16_t)t.par[v] : (uint16_t)v;
+    __syncthreads();
+    for (int r = 1; r <= maxd; r <<= 1) {
+        uint16_t nt[8];
+#pragma unroll
+        for (int q = 0; q < 8; q++) {
+            const int i = tid + q * T;
+            if (i < m) nt[q] = t.top[t.top[i]];
+        }
+        __syncthreads();
+#pragma unroll
+        for (int q = 0; q < 8; q++) {
+            const int i = tid + q * T;
+            if (i < m) t.top[i] = nt[q];
+        }
+        __syncthreads();
+    }
+    for (int v = tid; v < m; v += T)
+        if (t.hv[v] == 0xFFFF) t.bot[t.top[v]] = (uint16_t)v;
+    // path tops, deepest first (a light child's top is deeper than its parent's path top)
+    if (warp == 0) {
+        int n = 0;
+        for (int c0 = m - 1; c0 >= 0; c0 -= 32) {
+            const int k = c0 - lane;
+            const int v = k >= 0 ? t.anc[k] : 0;
+            const bool is_top = k >= 0 && t.top[v] == v;
+            const unsigned b = __ballot_sync(0xffffffffu, is_top);
+            if (is_top) t.pq[n + __popc(b & ((1u << lane) - 1u))] = (uint16_t)v;
+            n += __popc(b);
+        }
+        if (lane == 0) s_npaths = n;
+    }
     TMARK(1);
 #pragma unroll 2
     for (int task = tid; task < 4 * (m - 1); task += T) gather_task(g, t, task);
     __syncthreads();
     TMARK(2);
-    // bottom-up DP: 8 warps x G groups evaluate nodes of one level side by side
-    constexpr int SLOTS = FGR_WARPS_PER_CTA * G;
-    const int myslot = warp * G + gi;
+    const int npaths = s_npaths;
+    // ---------------- values: bottom-up path walks
 #ifdef FGR_TIMING
-    long long ph[4] = {0, 0, 0, 0};
+    long long vw_wait = 0, vw_nodes = 0, vw_paths = 0, vw_light = 0, vw_t0 = clock64();
+    long long f_rows = 0, f_pref = 0, f_B = 0, f_E = 0, f_fin = 0, f_x;
 #endif
-    for (int d = maxd; d >= 1; d--) {
-        const int k0 = t.lvstart[d], k1 = t.lvstart[d + 1];
-        for (int kb = k0; kb < k1; kb += SLOTS) {
-            const int k = kb + myslot;
-            const bool act = glane && k < k1;
-            const int v = act ? t.anc[k] : 0;
+    if (glane) {
+        const uint32_t opp = c.my_dir == 1 ? c.hmask : (~c.hmask & ((1u << LT) - 1u));   // bend partner layers
+        bool first = (warp == 0);   // warp 0 starts on the root path right away
+        for (;;) {
+            int tp;
+            if (first) {
+                tp = 0;
+                first = false;
+            } else {
+                int p = 0;
+                if (gl == 0) p = atomicAdd(&s_ticket, 1);
+                p = __shfl_sync(gmask, p, gbase);
+                if (p >= npaths - 1) break;   // pq[npaths-1] is the root path
+                tp = t.pq[p];
+            }
+            int v = t.bot[tp];
 #ifdef FGR_TIMING
-            long long q0 = clock64();
+            vw_paths++;
 #endif
-            span_rows<LT, true>(c, t, w, v, gl, act);
-            __syncwarp();
+            uint32_t Eprev = FGR_INF;
+            bool has_prev = false;
+            for (;;) {
+                const int hvv = t.hv[v];
+                const int k0 = t.cstart[v], k1 = t.cstart[v + 1];
+                const bool light = (k1 - k0) > 1;
 #ifdef FGR_TIMING
-            long long q1 = clock64();
+                vw_nodes++;
 #endif
-            node_table<LT>(t, w, v, gl, act);
-            __syncwarp();
+                if (light) {
 #ifdef FGR_TIMING
-            long long q2 = clock64();
+                    long long q0 = clock64();
+                    vw_light++;
 #endif
-            edge_table<LT>(c, t, w, v, gl, nH, nV, act);
-            __syncwarp();
+                    for (int k = k0 + gl; k < k1; k += LT) {
+                        const int ch = t.clist[k];
+                        if (ch != hvv) while (ld_flag(&t.done[ch]) == 0) __nanosleep(40);
+                    }
+                    __syncwarp(gmask);
 #ifdef FGR_TIMING
-            long long q3 = clock64();
-            if (kb == k0) { ph[0] += q1 - q0; ph[1] += q2 - q1; ph[2] += q3 - q2; }
+                    vw_wait += clock64() - q0;
+                    f_x = clock64();
+#endif
+                    __threadfence_block();
+                    // K rows (light children only) -> suffix minima R(lo, b) -> column prefix G(a, b), in w.R
+                    const int lo = gl;
+                    uint32_t acc[LT];
+#pragma unroll
+                    for (int hi = 0; hi < LT; hi++) acc[hi] = hi >= lo ? c.vme[hi] : FGR_INF;
+                    for (int k = k0; k < k1; k++) {
+                        const int ch = t.clist[k];
+                        if (ch == hvv) continue;
+                        const uint32_t* Ec = t.E + (size_t)ch * LT;
+                        uint32_t run = FGR_INF;
+#pragma unroll
+                        for (int hi = 0; hi < LT; hi++) {
+                            const uint32_t e = Ec[hi];
+                            if (hi >= lo) { run = min(run, e); acc[hi] = sat_add(acc[hi], run); }
+                        }
+                    }
+                    unsigned long long run = ~0ull;
+#pragma unroll
+                    for (int hi = LT - 1; hi >= 0; hi--)
+                        if (hi >= lo) {
+                            const unsigned long long key = ((unsigned long long)acc[hi] << 8) | (unsigned)(lo << 4) | (unsigned)hi;
+                            run = key < run ? key : run;
+                            w.R[lo * LT + hi] = run;
+                        }
+                    __syncwarp(gmask);
+#ifdef FGR_TIMING
+                    f_rows += clock64() - f_x; f_x = clock64();
+#endif
+                    const int bcol = gl;
+                    unsigned long long pr = ~0ull;
+#pragma unroll
+                    for (int a = 0; a < LT; a++)
+                        if (a <= bcol) {
+                            const unsigned long long x = w.R[a * LT + bcol];
+                            pr = x < pr ? x : pr;
+                            w.R[a * LT + bcol] = pr;
+                        }
+                    __syncwarp(gmask);
+#ifdef FGR_TIMING
+                    f_pref += clock64() - f_x;
+#endif
+                }
+#ifdef FGR_TIMING
+                f_x = clock64();
+#endif
+                const int plo = t.plo[v], phi = t.phi[v];
+                if (v == 0) {
+                    // generalised Eq. (4): min over l of E_h(l) + G(hull({l} + pins)) (any span for a Steiner root)
+                    const int ra = plo >= 0 ? plo : LT - 1, rb = plo >= 0 ? phi : 0;
+                    unsigned long long best = ~0ull;
+#pragma unroll
+                    for (int l = 0; l < LT; l++) {
+                        const uint32_t e = __shfl_sync(gmask, Eprev, gbase + l);
+                        const int a = min(ra, l), b = max(rb, l);
+                        const unsigned long long gk = light ? w.R[a * LT + b] : gclosed(h, a, b);
+                        const unsigned long long key = ((unsigned long long)sat_add(e, (uint32_t)(gk >> 8)) << 8) | (gk & 0xFFull);
+                        best = key < best ? key : best;
+                    }
+                    if (gl == 0) { s_root = best; t.span[0] = (uint8_t)(best & 0xFF); }
+                    __syncwarp(gmask);
+                    __threadfence_block();
+                    if (gl == 0) { t.done[0] = 1; *(volatile uint8_t*)&t.sready[0] = 1; }
+                    break;
+                }
+                // Eq. (2) in product form, lane = ls
+                const int ls = gl;
+                int a0 = ls, b0 = ls;
+                if (plo >= 0) { a0 = min(a0, plo); b0 = max(b0, phi); }
+                unsigned long long bk = ~0ull;
+                if (light) {
+                    if (!has_prev) bk = w.R[a0 * LT + b0];
+                    else {
+                        unsigned long long gk[LT];
+#pragma unroll
+                        for (int l = 0; l < LT; l++) gk[l] = w.R[min(a0, l) * LT + max(b0, l)];
+#pragma unroll
+                        for (int l = 0; l < LT; l++) {
+                            const uint32_t e = __shfl_sync(gmask, Eprev, gbase + l);
+                            const unsigned long long key =
+                                ((unsigned long long)sat_add(e, (uint32_t)(gk[l] >> 8)) << 8) | (gk[l] & 0xFFull);
+                            bk = key < bk ? key : bk;
+                        }
+                    }
+                } else {
+                    // K = V: G(a, b) = (V(a, b), span (zlo[a], b)) in closed form, a = min(a0, l), b = max(b0, l)
+                    uint32_t va0 = 0, vb0 = 0, za0 = 0;
+#pragma unroll
+                    for (int l = 0; l < LT; l++) {
+                        va0 = (l == a0) ? c.vp[l] : va0;
+                        vb0 = (l == b0) ? c.vp[l] : vb0;
+                        za0 = (l == a0) ? c.zl[l] : za0;
+                    }
+                    if (!has_prev) bk = ((unsigned long long)(vb0 - va0) << 8) | (za0 << 4) | (unsigned)b0;
+                    else {
+#pragma unroll
+                        for (int l = 0; l < LT; l++) {
+                            const uint32_t e = __shfl_sync(gmask, Eprev, gbase + l);
+                            const bool la = l < a0, lb = l > b0;
+                            const uint32_t va = la ? c.vp[l] : va0, vb = lb ? c.vp[l] : vb0;
+                            const uint32_t za = la ? c.zl[l] : za0;
+                            const uint32_t bb = lb ? (uint32_t)l : (uint32_t)b0;
+                            const unsigned long long key =
+                                ((unsigned long long)sat_add(e, vb - va) << 8) | (za << 4) | bb;
+                            bk = key < bk ? key : bk;
+                        }
+                    }
+                }
+                const uint32_t Bv = (uint32_t)(bk >> 8);
+                t.recB[(size_t)v * LT + ls] = (uint8_t)(bk & 0xFF);
+#ifdef FGR_TIMING
+                f_B += clock64() - f_x; f_x = clock64();
+#endif
+                // Eqs. (1),(3),(5)-(7), lane = lt
+                const int lt = gl;
+                const int u = t.par[v];
+                const int xv = t.x[v], yv = t.y[v], xu = t.x[u], yu = t.y[u];
+                uint32_t best = FGR_INF;
+                int bls = lt;
+                uint32_t Bl[LT];
+#pragma unroll
+                for (int l = 0; l < LT; l++) Bl[l] = __shfl_sync(gmask, Bv, gbase + l);
+                if (yv == yu || xv == xu) {
+                    const int de = (yv == yu) ? 0 : 1;
+                    if (c.my_dir == de) {
+                        const uint32_t leg = de == 0 ? t.legH[(size_t)v * 2 * nH + c.my_slot] : t.legV[(size_t)v * 2 * nV + c.my_slot];
+                        best = sat_add(Bv, leg);
+                    }
+                } else {
+                    const bool b0v = c.my_dir == 1;
+                    const uint32_t leg2 = b0v ? t.legV[((size_t)v * 2 + 1) * nV + c.my_slot] : t.legH[((size_t)v * 2 + 1) * nH + c.my_slot];
+                    const uint32_t* l1 = b0v ? t.legH + (size_t)v * 2 * nH : t.legV + (size_t)v * 2 * nV;
+                    int sidx = 0;
+#pragma unroll
+                    for (int l = 0; l < LT; l++)
+                        if ((opp >> l) & 1u) {
+                            const uint32_t cst = sat_add(sat_add(sat_add(Bl[l], l1[sidx]), c.vme[l]), leg2);
+                            if (cst < best) { best = cst; bls = l; }
+                            sidx++;
+                        }
+                }
+                t.E[(size_t)v * LT + lt] = best;
+                t.recE[(size_t)v * LT + lt] = (uint8_t)bls;
+#ifdef FGR_TIMING
+                f_E += clock64() - f_x; f_x = clock64();
+#endif
+                __syncwarp(gmask);
+                __threadfence_block();
+                if (gl == 0) *(volatile uint8_t*)&t.done[v] = 1;
+#ifdef FGR_TIMING
+                f_fin += clock64() - f_x;
+#endif
+                if (v == tp) break;
+                Eprev = best;
+                has_prev = true;
+                v = u;
+            }
+        }
+    }
+#ifdef FGR_TIMING
+    if (gl == 0 && glane && m > 900)
+        printf("VAL m=%d warp=%d paths=%lld nodes=%lld light=%lld wait=%lld total=%lld rows=%lld pref=%lld B=%lld E=%lld fin=%lld\n", m, warp, vw_paths, vw_nodes,
+               vw_light, vw_wait, clock64() - vw_t0, f_rows, f_pref, f_B, f_E, f_fin);
+#endif
+    __syncthreads();
+    TMARK(3);
+    // ---------------- backtrack: top-down path walks (S5)
+#ifdef FGR_TIMING
+    long long bt_wait = 0, bt_walk = 0, bt_nodes = 0, bt_paths = 0;
+#endif
+    if (glane) {
+        for (;;) {
+            int p = 0;
+            if (gl == 0) p = atomicAdd(&s_ticket2, 1);   // ticket 0 = the root path (shallowest top)
+            p = __shfl_sync(gmask, p, gbase);
+            if (p >= npaths) break;
+            const int tp = t.pq[npaths - 1 - p];
+            int v;
+#ifdef FGR_TIMING
+            long long w0 = clock64();
+#endif
+            if (tp == 0) v = t.hv[0];
+            else {
+                while (ld_flag(&t.sready[t.par[tp]]) == 0) __nanosleep(40);
+                __threadfence_block();
+                v = tp;
+            }
+#ifdef FGR_TIMING
+            long long w1 = clock64();
+            bt_wait += w1 - w0;
+            bt_paths++;
+#endif
+            while (v != 0xFFFF) {
+#ifdef FGR_TIMING
+                bt_nodes++;
+#endif
+                const int u = t.par[v];
+                const int sp = t.span[u];
+                const int lo = sp >> 4, hi = sp & 15;
+                const int l = gl;
+                const unsigned long long cand =
+                    (l >= lo && l <= hi) ? (((unsigned long long)t.E[(size_t)v * LT + l] << 4) | (unsigned)l) : ~0ull;
+                unsigned long long bst = ~0ull;
+#pragma unroll
+                for (int k = 0; k < LT; k++) {
+                    const unsigned long long x = __shfl_sync(gmask, cand, gbase + k);
+                    bst = x < bst ? x : bst;
+                }
+                if (gl == 0) {
+                    const int lt = (int)(bst & 15);
+                    const int ls = t.recE[(size_t)v * LT + lt];
+                    t.span[v] = t.recB[(size_t)v * LT + ls];
+                    const bool straight = (t.x[v] == t.x[u]) || (t.y[v] == t.y[u]);
+                    const uint32_t bend = straight ? 0u : (h->dir[lt] == 1 ? 0u : 1u);
+                    const uint32_t sg = bend | ((uint32_t)ls << 8) | ((uint32_t)lt << 16) | ((uint32_t)straight << 24);
+                    t.legH[(size_t)v * 2 * nH] = sg;   // the leg costs are dead now: keep the route (shared memory only)
+                }
+                __syncwarp(gmask);
+                __threadfence_block();
+                if (gl == 0) *(volatile uint8_t*)&t.sready[v] = 1;
+                v = t.hv[v];
+            }
+#ifdef FGR_TIMING
+            bt_walk += clock64() - w1;
 #endif
         }
-#ifdef FGR_TIMING
-        long long q4 = clock64();
-#endif
-        __syncthreads();
-#ifdef FGR_TIMING
-        ph[3] += clock64() - q4;
-#endif
     }
 #ifdef FGR_TIMING
-    if (tid == 0 && m > 880)
-        printf("LEVELS m=%d maxd=%d span=%lld node=%lld edge=%lld barrier=%lld (cycles summed over levels, warp 0)\n", m,
-               maxd, ph[0], ph[1], ph[2], ph[3]);
+    if (gl == 0 && glane && m > 900)
+        printf("BT m=%d warp=%d paths=%lld nodes=%lld wait=%lld walk=%lld per_node=%lld\n", m, warp, bt_paths, bt_nodes,
+               bt_wait, bt_walk, bt_nodes ? bt_walk / bt_nodes : 0);
 #endif
-    TMARK(3);
-    if (warp == 0) {
-        const bool act = glane && gi == 0;
-        span_rows<LT, true>(c, t, w, 0, gl, act);
-        __syncwarp();
-        const unsigned long long rc = root_cand<LT>(t, w, gl, act);
-        if (act) atomicMin(&s_root, rc);
-    }
-    __syncthreads();
-    if (tid == 0) t.span[0] = (uint8_t)(s_root & 0xFF);
     __syncthreads();
     TMARK(4);
-    for (int d = 1; d <= maxd; d++) {
-        const int k1 = t.lvstart[d + 1];
-        for (int k = t.lvstart[d] + tid; k < k1; k += T) {
-            const int i = t.anc[k];
-            const uint32_t s = backtrack_node<LT>(h, t, i);
-            if (o.rec_seg) o.rec_seg[o.rec_off[o.list_base + idx] + i] = s;
-            else o.seg[a0 + i] = s;
-            t.legH[(size_t)i * 2 * nH] = s;   // the leg costs are dead now: keep the route for the commit
-        }
-        __syncthreads();
-    }
     TMARK(5);
-    // S6 for the whole net in one pass (the atomics' latencies overlap across threads)
-    if (commit)
-        for (int i = 1 + tid; i < m; i += T) {
-            const uint32_t s = t.legH[(size_t)i * 2 * nH];
+    // outputs and S6 for the whole net in one pass (the atomics' latencies overlap across threads)
+    for (int i = 1 + tid; i < m; i += T) {
+        const uint32_t s = t.legH[(size_t)i * 2 * nH];
+        if (o.rec_seg) o.rec_seg[o.rec_off[o.list_base + idx] + i] = s;
+        else o.seg[a0 + i] = s;
+        if (commit) {
             const int u = t.par[i];
             commit_edge(g, h, t.x[i], t.y[i], t.x[u], t.y[u], s);
         }
+    }
 #ifdef FGR_TIMING
     __syncthreads();
     TMARK(6);
     if (tid == 0 && m > 600)
-        printf("TIMING m=%d maxd=%d prologue=%lld gather=%lld dp=%lld root=%lld backtrack=%lld commit=%lld\n", m, maxd,
-               tm[1] - tm[0], tm[2] - tm[1], tm[3] - tm[2], tm[4] - tm[3], tm[5] - tm[4], tm[6] - tm[5]);
+        printf("TIMING m=%d maxd=%d paths=%d prologue=%lld gather=%lld dp=%lld backtrack=%lld commit=%lld\n", m, maxd,
+               npaths, tm[1] - tm[0], tm[2] - tm[1], tm[3] - tm[2], tm[4] - tm[3], tm[6] - tm[5]);
 #endif
     if (tid == 0) {
         const uint32_t total = (uint32_t)(s_root >> 8);
@@ -757,8 +1072,7 @@ size_t smem_group(int L, int nH, int nV) {
 }
 
 size_t smem_large(int L, int nH, int nV, int m) {
-    return a16(sizeof(Hdr)) + (size_t)FGR_WARPS_PER_CTA * groups_of(L) * wscr_bytes(L) +
-           tabs_bytes(m, L, nH, nV, true);
+    return a16(sizeof(Hdr)) + (size_t)kLargeWarps * wscr_bytes(L) + tabs_bytes(m, L, nH, nV, true);
 }
 
 template <int LT>
@@ -781,7 +1095,7 @@ cudaError_t launch_lt(fgr_grid* g, cudaStream_t st, const NetsView& nv, const in
     const GridView& v = g->view;
     if (nlarge > 0) {
         const int ps = fgr_prof_begin(g, PROF_DP_LARGE, st);
-        k_dp_large<LT><<<nlarge, FGR_CTA_THREADS, smem_large(LT, g->nH, g->nV, maxm_large), st>>>(
+        k_dp_large<LT><<<nlarge, 32 * kLargeWarps, smem_large(LT, g->nH, g->nV, maxm_large), st>>>(
             v, nv, list, nlarge, o, commit ? 1 : 0);
         fgr_prof_end(g, ps, st);
         g->stats.kernel_launches++;
