@@ -217,6 +217,12 @@ extern "C" FGR_API fgr_status fgr_grid_create(const fgr_grid_desc* d, int device
     if (e == cudaSuccess) e = cudaGetLastError();
     if (e != cudaSuccess) { fgr_grid_destroy(g); return fgr_cuda_fail(nullptr, e, "grid init"); }
     g->full_dirty = true;
+    if (cudaStreamCreateWithFlags(&g->side, cudaStreamNonBlocking) != cudaSuccess ||
+        cudaEventCreateWithFlags(&g->ev_fork, cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventCreateWithFlags(&g->ev_join, cudaEventDisableTiming) != cudaSuccess) {
+        fgr_grid_destroy(g);
+        return fgr_set_error(FGR_ERR_CUDA, "stream/event creation failed");
+    }
     cudaDeviceGetAttribute(&g->max_smem, cudaDevAttrMaxSharedMemoryPerBlockOptin, device);
     cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, device);
     g->stats.world = 1;
@@ -234,6 +240,9 @@ extern "C" FGR_API fgr_status fgr_grid_destroy(fgr_grid* g) {
     for (auto& s : g->s_plan) cudaFree(s.p);
     for (auto& s : g->s_rec) cudaFree(s.p);
     for (auto e : g->prof.pool) cudaEventDestroy(e);
+    if (g->side) cudaStreamDestroy(g->side);
+    if (g->ev_fork) cudaEventDestroy(g->ev_fork);
+    if (g->ev_join) cudaEventDestroy(g->ev_join);
     free(g->cache.h_off);
     free(g->cache.h_nlarge);
     free(g->cache.h_maxm);

@@ -586,6 +586,16 @@ __device__ __forceinline__ unsigned long long gclosed(const Hdr* h, int a, int b
 
 __device__ __forceinline__ int ld_flag(const uint8_t* f) { return *(volatile const uint8_t*)f; }
 
+// min of N packed keys as a balanced tree (dependency depth log2 N instead of N)
+template <int N>
+__device__ __forceinline__ unsigned long long tree_min(unsigned long long (&k)[N]) {
+#pragma unroll
+    for (int s = 1; s < N; s <<= 1)
+#pragma unroll
+        for (int i = 0; i + s < N; i += 2 * s) k[i] = k[i + s] < k[i] ? k[i + s] : k[i];
+    return k[0];
+}
+
 template <int LT>
 __global__ void __launch_bounds__(32 * kLargeWarps, 1) k_dp_large(GridView g, NetsView nv, const int32_t* __restrict__ list,
                                                                   int count, Out o, int commit) {
@@ -866,10 +876,9 @@ __global__ void __launch_bounds__(32 * kLargeWarps, 1) k_dp_large(GridView g, Ne
 #pragma unroll
                         for (int l = 0; l < LT; l++) {
                             const uint32_t e = __shfl_sync(gmask, Eprev, gbase + l);
-                            const unsigned long long key =
-                                ((unsigned long long)sat_add(e, (uint32_t)(gk[l] >> 8)) << 8) | (gk[l] & 0xFFull);
-                            bk = key < bk ? key : bk;
+                            gk[l] = ((unsigned long long)sat_add(e, (uint32_t)(gk[l] >> 8)) << 8) | (gk[l] & 0xFFull);
                         }
+                        bk = tree_min<LT>(gk);
                     }
                 } else {
                     // K = V: G(a, b) = (V(a, b), span (zlo[a], b)) in closed form, a = min(a0, l), b = max(b0, l)
@@ -882,6 +891,7 @@ __global__ void __launch_bounds__(32 * kLargeWarps, 1) k_dp_large(GridView g, Ne
                     }
                     if (!has_prev) bk = ((unsigned long long)(vb0 - va0) << 8) | (za0 << 4) | (unsigned)b0;
                     else {
+                        unsigned long long kk[LT];
 #pragma unroll
                         for (int l = 0; l < LT; l++) {
                             const uint32_t e = __shfl_sync(gmask, Eprev, gbase + l);
@@ -889,10 +899,9 @@ __global__ void __launch_bounds__(32 * kLargeWarps, 1) k_dp_large(GridView g, Ne
                             const uint32_t va = la ? c.vp[l] : va0, vb = lb ? c.vp[l] : vb0;
                             const uint32_t za = la ? c.zl[l] : za0;
                             const uint32_t bb = lb ? (uint32_t)l : (uint32_t)b0;
-                            const unsigned long long key =
-                                ((unsigned long long)sat_add(e, vb - va) << 8) | (za << 4) | bb;
-                            bk = key < bk ? key : bk;
+                            kk[l] = ((unsigned long long)sat_add(e, vb - va) << 8) | (za << 4) | bb;
                         }
+                        bk = tree_min<LT>(kk);
                     }
                 }
                 const uint32_t Bv = (uint32_t)(bk >> 8);
@@ -946,7 +955,7 @@ __global__ void __launch_bounds__(32 * kLargeWarps, 1) k_dp_large(GridView g, Ne
             }
         }
     }
-#ifdef FGR_TIMING
+#ifdef FGR_TIMING_DETAIL
     if (gl == 0 && glane && m > 900)
         printf("VAL m=%d warp=%d paths=%lld nodes=%lld light=%lld wait=%lld total=%lld rows=%lld pref=%lld B=%lld E=%lld fin=%lld\n", m, warp, vw_paths, vw_nodes,
                vw_light, vw_wait, clock64() - vw_t0, f_rows, f_pref, f_B, f_E, f_fin);
@@ -987,16 +996,11 @@ __global__ void __launch_bounds__(32 * kLargeWarps, 1) k_dp_large(GridView g, Ne
                 const int sp = t.span[u];
                 const int lo = sp >> 4, hi = sp & 15;
                 const int l = gl;
-                const unsigned long long cand =
-                    (l >= lo && l <= hi) ? (((unsigned long long)t.E[(size_t)v * LT + l] << 4) | (unsigned)l) : ~0ull;
-                unsigned long long bst = ~0ull;
-#pragma unroll
-                for (int k = 0; k < LT; k++) {
-                    const unsigned long long x = __shfl_sync(gmask, cand, gbase + k);
-                    bst = x < bst ? x : bst;
-                }
+                const uint32_t cand = (l >= lo && l <= hi) ? t.E[(size_t)v * LT + l] : 0xFFFFFFFFu;
+                const uint32_t mn = __reduce_min_sync(gmask, cand);
+                const unsigned bal = __ballot_sync(gmask, cand == mn) >> gbase;   // smallest l attaining the min (R11)
                 if (gl == 0) {
-                    const int lt = (int)(bst & 15);
+                    const int lt = __ffs(bal) - 1;
                     const int ls = t.recE[(size_t)v * LT + lt];
                     t.span[v] = t.recB[(size_t)v * LT + ls];
                     const bool straight = (t.x[v] == t.x[u]) || (t.y[v] == t.y[u]);
@@ -1014,7 +1018,7 @@ __global__ void __launch_bounds__(32 * kLargeWarps, 1) k_dp_large(GridView g, Ne
 #endif
         }
     }
-#ifdef FGR_TIMING
+#ifdef FGR_TIMING_DETAIL
     if (gl == 0 && glane && m > 900)
         printf("BT m=%d warp=%d paths=%lld nodes=%lld wait=%lld walk=%lld per_node=%lld\n", m, warp, bt_paths, bt_nodes,
                bt_wait, bt_walk, bt_nodes ? bt_walk / bt_nodes : 0);
@@ -1093,27 +1097,38 @@ cudaError_t launch_lt(fgr_grid* g, cudaStream_t st, const NetsView& nv, const in
         configured = true;
     }
     const GridView& v = g->view;
+    const int nsmall = count - nlarge;
+    // Large and small nets of one batch are independent: when both exist the small
+    // nets run on a side stream beside the large-net CTAs (fork/join with events).
+    const bool fork = nlarge > 0 && nsmall > 0;
+    cudaStream_t ss = fork ? g->side : st;
+    cudaError_t e;
+    if (fork) {
+        if ((e = cudaEventRecord(g->ev_fork, st)) != cudaSuccess) return e;
+        if ((e = cudaStreamWaitEvent(g->side, g->ev_fork, 0)) != cudaSuccess) return e;
+    }
+    if (nsmall > 0) {
+        Out os = o;
+        os.list_base = o.list_base + nlarge;
+        const int per_cta = kGroupWarps * groups_of(LT);
+        const int ps = fgr_prof_begin(g, PROF_DP_SMALL, ss);
+        k_dp_group<LT><<<(nsmall + per_cta - 1) / per_cta, 32 * kGroupWarps, smem_group(LT, g->nH, g->nV), ss>>>(
+            v, nv, list + nlarge, nsmall, os, commit ? 1 : 0);
+        fgr_prof_end(g, ps, ss);
+        g->stats.kernel_launches++;
+        if ((e = cudaGetLastError()) != cudaSuccess) return e;
+    }
     if (nlarge > 0) {
         const int ps = fgr_prof_begin(g, PROF_DP_LARGE, st);
         k_dp_large<LT><<<nlarge, 32 * kLargeWarps, smem_large(LT, g->nH, g->nV, maxm_large), st>>>(
             v, nv, list, nlarge, o, commit ? 1 : 0);
         fgr_prof_end(g, ps, st);
         g->stats.kernel_launches++;
-        cudaError_t e = cudaGetLastError();
-        if (e != cudaSuccess) return e;
+        if ((e = cudaGetLastError()) != cudaSuccess) return e;
     }
-    const int nsmall = count - nlarge;
-    if (nsmall > 0) {
-        Out os = o;
-        os.list_base = o.list_base + nlarge;
-        const int per_cta = kGroupWarps * groups_of(LT);
-        const int ps = fgr_prof_begin(g, PROF_DP_SMALL, st);
-        k_dp_group<LT><<<(nsmall + per_cta - 1) / per_cta, 32 * kGroupWarps, smem_group(LT, g->nH, g->nV), st>>>(
-            v, nv, list + nlarge, nsmall, os, commit ? 1 : 0);
-        fgr_prof_end(g, ps, st);
-        g->stats.kernel_launches++;
-        cudaError_t e = cudaGetLastError();
-        if (e != cudaSuccess) return e;
+    if (fork) {
+        if ((e = cudaEventRecord(g->ev_join, g->side)) != cudaSuccess) return e;
+        if ((e = cudaStreamWaitEvent(st, g->ev_join, 0)) != cudaSuccess) return e;
     }
     return cudaSuccess;
 }

@@ -132,6 +132,8 @@ struct fgr_grid {
     int max_smem = 0;
     int num_sms = 0;
     Profiler prof;
+    cudaStream_t side = nullptr;      // second stream: small nets run beside the large-net CTAs
+    cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
 };
 
 // Profiling brackets around a launch (no-ops unless fgr_profile_enable(grid, 1)).
