@@ -122,7 +122,7 @@ struct fgr_grid {
     bool broken = false;
     int total_segs = 0;
     // plan scratch
-    Scratch s_plan[12];
+    Scratch s_plan[14];
     PlanCache cache;
     // multi-GPU
     ncclComm_t comm = nullptr;

@@ -126,12 +126,15 @@ __global__ void k_tile_emit(int R, const unsigned long long* __restrict__ box_r,
 }
 
 __global__ void k_tile_bounds(int T, const unsigned long long* __restrict__ tkeys, int* __restrict__ tstart,
-                              int* __restrict__ tend, int* __restrict__ entries) {
+                              int* __restrict__ tend, uint4* __restrict__ entries,
+                              const unsigned long long* __restrict__ box_r) {
     const int i = blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= T) return;
     const unsigned long long k = tkeys[i];
     const int t = (int)(k >> 32);
-    entries[i] = (int)(k & 0xFFFFFFFFu);
+    const unsigned r = (unsigned)(k & 0xFFFFFFFFu);
+    const unsigned long long b = box_r[r];
+    entries[i] = make_uint4(r, (unsigned)(b & 0xFFFFFFFFu), (unsigned)(b >> 32), 0u);   // rank + its box: one load
     if (i == 0 || (int)(tkeys[i - 1] >> 32) != t) tstart[t] = i;
     if (i == T - 1 || (int)(tkeys[i + 1] >> 32) != t) tend[t] = i + 1;
 }
@@ -143,7 +146,7 @@ __global__ void k_tile_bounds(int T, const unsigned long long* __restrict__ tkey
 // overlap and only the (short) publish chain is serial.
 #define COLOR_BITS 1024
 #define COLOR_DEFER 128
-#define COLOR_UNROLL 4
+#define COLOR_UNROLL 8
 __device__ __forceinline__ void mark_colour(uint32_t* bw, int c, int wb) {
     c -= wb;
     if (c >= 0 && c < COLOR_BITS) atomicOr(&bw[c >> 5], 1u << (c & 31));
@@ -151,7 +154,7 @@ __device__ __forceinline__ void mark_colour(uint32_t* bw, int c, int wb) {
 
 __global__ void __launch_bounds__(256) k_color(int R, const unsigned long long* __restrict__ box_r,
                                                const int* __restrict__ tstart, const int* __restrict__ tend,
-                                               const int* __restrict__ entries, int tiles_x, int* color,
+                                               const uint4* __restrict__ entries, int tiles_x, int* color,
                                                int* __restrict__ ticket, int* __restrict__ nbatches,
                                                int* __restrict__ bcount) {
     __shared__ uint32_t bits[8][COLOR_BITS / 32];
@@ -182,10 +185,15 @@ __global__ void __launch_bounds__(256) k_color(int R, const unsigned long long* 
 #pragma unroll
                         for (int u = 0; u < COLOR_UNROLL; u++) {
                             const int j = base + u * 32 + lane;
-                            rr[u] = j < e ? __ldg(entries + j) : 0x7FFFFFFF;
+                            if (j < e) {
+                                const uint4 q = __ldg(entries + j);
+                                rr[u] = (int)q.x;
+                                bb[u] = (unsigned long long)q.y | ((unsigned long long)q.z << 32);
+                            } else {
+                                rr[u] = 0x7FFFFFFF;
+                                bb[u] = 0ull;
+                            }
                         }
-#pragma unroll
-                        for (int u = 0; u < COLOR_UNROLL; u++) bb[u] = rr[u] < r ? __ldg(box_r + rr[u]) : 0ull;
                         bool stop = false;
 #pragma unroll
                         for (int u = 0; u < COLOR_UNROLL; u++) {
@@ -202,7 +210,7 @@ __global__ void __launch_bounds__(256) k_color(int R, const unsigned long long* 
                                         if (k < COLOR_DEFER) defer[w][k] = rr[u];
                                         else {
                                             int cc;
-                                            while ((cc = vcolor[rr[u]]) < 0) __nanosleep(64);
+                                            while ((cc = vcolor[rr[u]]) < 0) __nanosleep(20);
                                             mark_colour(bw, cc, wb);
                                         }
                                     }
@@ -216,7 +224,7 @@ __global__ void __launch_bounds__(256) k_color(int R, const unsigned long long* 
             const int nd = min(ndefer[w], COLOR_DEFER);
             for (int k = lane; k < nd; k += 32) {
                 int cc;
-                while ((cc = vcolor[defer[w][k]]) < 0) __nanosleep(32);
+                while ((cc = vcolor[defer[w][k]]) < 0) __nanosleep(20);
                 mark_colour(bw, cc, wb);
             }
             __syncwarp();
@@ -236,7 +244,7 @@ __global__ void __launch_bounds__(256) k_color(int R, const unsigned long long* 
             if (found >= 0) result = wb + found;
         }
         if (lane == 0) {
-            __threadfence();
+            // the colour word is the only datum a waiting warp reads: publish it without a fence
             atomicExch(&color[r], result);
             atomicMax(nbatches, result + 1);
             atomicAdd(&bcount[result], 1);
@@ -393,7 +401,8 @@ extern "C" FGR_API fgr_status fgr_plan(fgr_grid* g, const fgr_nets* nets, int32_
     auto* tkeys = take<unsigned long long>(g, 9, (size_t)T + 1, &e);
     auto* tkeys_s = take<unsigned long long>(g, 10, (size_t)T + 1, &e);
     if (e != cudaSuccess) return fgr_cuda_fail(g, e, "plan tile scratch");
-    int* entries = (int*)tkeys;   // reused after the sort
+    uint4* entries = take<uint4>(g, 12, (size_t)T + 1, &e);   // (rank, box) per tile entry
+    if (e != cudaSuccess) return fgr_cuda_fail(g, e, "plan tile entries");
     int* color = tcount;          // N+1 ints, tcount no longer needed after the scan
     if (R > 0) {
         k_tile_emit<<<(R + 255) / 256, 256, 0, st>>>(R, box_r, toff, tkeys, tiles_x);
@@ -406,7 +415,7 @@ extern "C" FGR_API fgr_status fgr_plan(fgr_grid* g, const fgr_nets* nets, int32_
         ps = fgr_prof_begin(g, PROF_SORT, st);
         FGR_CHECK_CUDA(g, cub::DeviceRadixSort::SortKeys(tmp, tmp_bytes, tkeys, tkeys_s, T, 0, tb, st));
         fgr_prof_end(g, ps, st);
-        k_tile_bounds<<<(T + 255) / 256, 256, 0, st>>>(T, tkeys_s, tstart, tend, entries);
+        k_tile_bounds<<<(T + 255) / 256, 256, 0, st>>>(T, tkeys_s, tstart, tend, entries, box_r);
         FGR_CHECK_CUDA(g, cudaGetLastError());
     }
     // colouring
