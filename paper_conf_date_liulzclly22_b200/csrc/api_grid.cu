@@ -217,9 +217,11 @@ extern "C" FGR_API fgr_status fgr_grid_create(const fgr_grid_desc* d, int device
     if (e == cudaSuccess) e = cudaGetLastError();
     if (e != cudaSuccess) { fgr_grid_destroy(g); return fgr_cuda_fail(nullptr, e, "grid init"); }
     g->full_dirty = true;
-    if (cudaStreamCreateWithFlags(&g->side, cudaStreamNonBlocking) != cudaSuccess ||
-        cudaEventCreateWithFlags(&g->ev_fork, cudaEventDisableTiming) != cudaSuccess ||
-        cudaEventCreateWithFlags(&g->ev_join, cudaEventDisableTiming) != cudaSuccess) {
+    bool sok = cudaEventCreateWithFlags(&g->ev_fork, cudaEventDisableTiming) == cudaSuccess;
+    for (int i = 0; i < 3 && sok; i++)
+        sok = cudaStreamCreateWithFlags(&g->side[i], cudaStreamNonBlocking) == cudaSuccess &&
+              cudaEventCreateWithFlags(&g->ev_join[i], cudaEventDisableTiming) == cudaSuccess;
+    if (!sok) {
         fgr_grid_destroy(g);
         return fgr_set_error(FGR_ERR_CUDA, "stream/event creation failed");
     }
@@ -239,14 +241,19 @@ extern "C" FGR_API fgr_status fgr_grid_destroy(fgr_grid* g) {
     cudaFree(g->d_stats);
     for (auto& s : g->s_plan) cudaFree(s.p);
     for (auto& s : g->s_rec) cudaFree(s.p);
+    cudaFree(g->s_prep.p);
     for (auto e : g->prof.pool) cudaEventDestroy(e);
-    if (g->side) cudaStreamDestroy(g->side);
+    for (int i = 0; i < 3; i++) {
+        if (g->side[i]) cudaStreamDestroy(g->side[i]);
+        if (g->ev_join[i]) cudaEventDestroy(g->ev_join[i]);
+    }
     if (g->ev_fork) cudaEventDestroy(g->ev_fork);
-    if (g->ev_join) cudaEventDestroy(g->ev_join);
     free(g->cache.h_off);
     free(g->cache.h_nlarge);
     free(g->cache.h_maxm);
     free(g->cache.h_segb);
+    free(g->cache.h_ntwo);
+    free(g->cache.h_n9);
     delete g;
     return FGR_OK;
 }

@@ -28,7 +28,6 @@
 
 namespace {
 
-constexpr int kMC = FGR_SMALL_NET;          // node capacity of one group in k_dp_group
 constexpr int kGroupWarps = 4;              // warps per CTA in k_dp_group
 constexpr int kLargeWarps = 16;             // warps per CTA in k_dp_large (one path-walking group each)
 
@@ -365,6 +364,137 @@ __device__ __forceinline__ void commit_edge(const GridView& g, const Hdr* h, int
     }
 }
 
+// Packed G entry of a node without light children (K = V): value V(a,b), span (zlo[a], b).
+__device__ __forceinline__ unsigned long long gclosed(const Hdr* h, int a, int b) {
+    return ((unsigned long long)(h->viapre[b] - h->viapre[a]) << 8) | (unsigned)(h->zlo[a] << 4) | (unsigned)b;
+}
+
+// min of N packed keys as a balanced tree (dependency depth log2 N instead of N)
+template <int N>
+__device__ __forceinline__ unsigned long long tree_min(unsigned long long (&k)[N]) {
+#pragma unroll
+    for (int s = 1; s < N; s <<= 1)
+#pragma unroll
+        for (int i = 0; i + s < N; i += 2 * s) k[i] = k[i + s] < k[i] ? k[i + s] : k[i];
+    return k[0];
+}
+
+// Product-form node step (the identity of the k_dp_large header comment) for one lane
+// group of a warp whose groups run in lockstep: every lane of the warp calls it (the
+// shuffles are full-warp).  All children of v are final; the highest-index child plays
+// the "heavy" child, the others fold into G.  Writes E_v / recE_v / recB_v, or returns
+// the root's packed (total, lo, hi) key when is_root.
+template <int LT>
+__device__ __forceinline__ unsigned long long node_step_group(const Hdr* h, const LaneConst<LT>& c, const Tabs& t,
+                                                              const WScr& w, int v, bool act, bool is_root, int gl,
+                                                              int gbase, int nH, int nV, uint32_t opp) {
+    const uint32_t cm = act ? t.aux[v] : 0u;
+    const int hc = cm ? 31 - __clz(cm) : -1;
+    const uint32_t lm = hc >= 0 ? (cm & ~(1u << hc)) : 0u;
+    const bool light = lm != 0;
+    if (light) {   // K rows from the light children, suffix minima over hi (lane = lo)
+        const int lo = gl;
+        uint32_t acc[LT];
+#pragma unroll
+        for (int hi = 0; hi < LT; hi++) acc[hi] = hi >= lo ? c.vme[hi] : FGR_INF;
+        uint32_t lmm = lm;
+        while (lmm) {
+            const int ch = __ffs(lmm) - 1;
+            lmm &= lmm - 1;
+            const uint32_t* Ec = t.E + (size_t)ch * LT;
+            uint32_t run = FGR_INF;
+#pragma unroll
+            for (int hi = 0; hi < LT; hi++) {
+                const uint32_t e = Ec[hi];
+                if (hi >= lo) { run = min(run, e); acc[hi] = sat_add(acc[hi], run); }
+            }
+        }
+        unsigned long long run = ~0ull;
+#pragma unroll
+        for (int hi = LT - 1; hi >= 0; hi--)
+            if (hi >= lo) {
+                const unsigned long long key = ((unsigned long long)acc[hi] << 8) | (unsigned)(lo << 4) | (unsigned)hi;
+                run = key < run ? key : run;
+                w.R[lo * LT + hi] = run;
+            }
+    }
+    __syncwarp();
+    if (light) {   // column prefix over lo: G(a, b) = min_{lo <= a} R(lo, b) (lane = b)
+        unsigned long long pr = ~0ull;
+#pragma unroll
+        for (int a = 0; a < LT; a++)
+            if (a <= gl) {
+                const unsigned long long x = w.R[a * LT + gl];
+                pr = x < pr ? x : pr;
+                w.R[a * LT + gl] = pr;
+            }
+    }
+    __syncwarp();
+    const uint32_t eh = (act && hc >= 0) ? t.E[(size_t)hc * LT + gl] : FGR_INF;
+    int plo = -1, phi = -1;
+    if (act) { plo = t.plo[v]; phi = t.phi[v]; }
+    int a0, b0;
+    if (is_root) { a0 = plo >= 0 ? plo : LT - 1; b0 = plo >= 0 ? phi : 0; }
+    else { a0 = gl; b0 = gl; if (plo >= 0) { a0 = min(a0, plo); b0 = max(b0, phi); } }
+    unsigned long long kk[LT];
+    uint32_t va0 = 0, vb0 = 0, za0 = 0;
+#pragma unroll
+    for (int l = 0; l < LT; l++) {
+        va0 = (l == a0) ? c.vp[l] : va0;
+        vb0 = (l == b0) ? c.vp[l] : vb0;
+        za0 = (l == a0) ? c.zl[l] : za0;
+    }
+#pragma unroll
+    for (int l = 0; l < LT; l++) {
+        const uint32_t e = __shfl_sync(0xffffffffu, eh, (gbase + l) & 31);
+        if (light) {
+            const unsigned long long gk = w.R[min(a0, l) * LT + max(b0, l)];
+            kk[l] = ((unsigned long long)sat_add(e, (uint32_t)(gk >> 8)) << 8) | (gk & 0xFFull);
+        } else {
+            const bool la = l < a0, lb = l > b0;
+            const uint32_t va = la ? c.vp[l] : va0, vb = lb ? c.vp[l] : vb0;
+            const uint32_t za = la ? c.zl[l] : za0;
+            const uint32_t bb = lb ? (uint32_t)l : (uint32_t)b0;
+            kk[l] = ((unsigned long long)sat_add(e, vb - va) << 8) | (za << 4) | bb;
+        }
+    }
+    unsigned long long bk = tree_min<LT>(kk);
+    if (hc < 0) bk = ((unsigned long long)(vb0 - va0) << 8) | (za0 << 4) | (unsigned)b0;   // leaf: no child term
+    if (is_root) return bk;
+    const uint32_t Bv = (uint32_t)(bk >> 8);
+    uint32_t Bl[LT];
+#pragma unroll
+    for (int l = 0; l < LT; l++) Bl[l] = __shfl_sync(0xffffffffu, Bv, (gbase + l) & 31);
+    if (!act) return 0;
+    t.recB[(size_t)v * LT + gl] = (uint8_t)(bk & 0xFF);
+    const int u = t.par[v];
+    const int xv = t.x[v], yv = t.y[v], xu = t.x[u], yu = t.y[u];
+    uint32_t best = FGR_INF;
+    int bls = gl;
+    if (yv == yu || xv == xu) {                   // straight: one leg on ls = lt (R7)
+        const int de = (yv == yu) ? 0 : 1;
+        if (c.my_dir == de) {
+            const uint32_t leg = de == 0 ? t.legH[(size_t)v * 2 * nH + c.my_slot] : t.legV[(size_t)v * 2 * nV + c.my_slot];
+            best = sat_add(Bv, leg);
+        }
+    } else {
+        const bool b0v = c.my_dir == 1;
+        const uint32_t leg2 = b0v ? t.legV[((size_t)v * 2 + 1) * nV + c.my_slot] : t.legH[((size_t)v * 2 + 1) * nH + c.my_slot];
+        const uint32_t* l1 = b0v ? t.legH + (size_t)v * 2 * nH : t.legV + (size_t)v * 2 * nV;
+        int sidx = 0;
+#pragma unroll
+        for (int l = 0; l < LT; l++)
+            if ((opp >> l) & 1u) {
+                const uint32_t cst = sat_add(sat_add(sat_add(Bl[l], l1[sidx]), c.vme[l]), leg2);
+                if (cst < best) { best = cst; bls = l; }
+                sidx++;
+            }
+    }
+    t.E[(size_t)v * LT + gl] = best;
+    t.recE[(size_t)v * LT + gl] = (uint8_t)bls;
+    return 0;
+}
+
 // ------------------------------------------------------------- group kernel (nets <= 32 nodes)
 // Flattened (group, item) iteration: item counts per group n[q]; returns the group of item `it`.
 template <int G>
@@ -390,7 +520,7 @@ struct Flat {
     }
 };
 
-template <int LT>
+template <int LT, int kMC>
 __global__ void __launch_bounds__(32 * kGroupWarps) k_dp_group(GridView g, NetsView nv, const int32_t* __restrict__ list,
                                                                int count, Out o, int commit) {
     constexpr int G = groups_of(LT);
@@ -460,29 +590,19 @@ __global__ void __launch_bounds__(32 * kGroupWarps) k_dp_group(GridView g, NetsV
     const WScr w = wscr_of(gi < G ? gi : 0);
     const bool glane = gi < G && gl < LT;
     unsigned long long rootkey = ~0ull;
+    const uint32_t opp = c.my_dir == 1 ? c.hmask : (~c.hmask & ((1u << LT) - 1u));   // bend partner layers
+    const int gbase = (gi < G ? gi : 0) * LT;
     for (int k = 0; k + 1 < maxm; k++) {
         const int v = my_m - 1 - k;
-        const bool act = glane && v >= 1;
-        span_rows<LT, false>(c, t, w, v, gl, act);
-        __syncwarp();
-        node_table<LT>(t, w, v, gl, act);
-        __syncwarp();
-        edge_table<LT>(c, t, w, v, gl, nH, nV, act);
+        node_step_group<LT>(h, c, t, w, v, glane && v >= 1, false, gl, gbase, nH, nV, opp);
         __syncwarp();
     }
-    // root (generalised Eq. (4)); a group's lanes reduce through the B scratch row
-    span_rows<LT, false>(c, t, w, 0, gl, glane && my_m >= 2);
-    __syncwarp();
-    const unsigned long long rc = root_cand<LT>(t, w, gl, glane && my_m >= 2);
-    __syncwarp();
-    if (glane && my_m >= 2) w.R[LT * LT - 1 - gl] = rc;   // R is dead now: reuse its tail for the reduction
-    __syncwarp();
-    if (glane && gl == 0 && my_m >= 2) {
-        unsigned long long b = ~0ull;
-#pragma unroll
-        for (int l = 0; l < LT; l++) { const unsigned long long x = w.R[LT * LT - 1 - l]; b = x < b ? x : b; }
-        t.span[0] = (uint8_t)(b & 0xFF);
-        rootkey = b;
+    // root (generalised Eq. (4))
+    {
+        const bool act = glane && my_m >= 2;
+        const unsigned long long rk = node_step_group<LT>(h, c, t, w, 0, act, true, gl, gbase, nH, nV, opp);
+        if (act && gl == 0) { t.span[0] = (uint8_t)(rk & 0xFF); rootkey = rk; }
+        __syncwarp();
     }
     // depth by pointer jumping (aux = ancestor), then a level-ordered backtrack
     for (int it = lane; it < nodes.total(); it += 32) {
@@ -493,7 +613,7 @@ __global__ void __launch_bounds__(32 * kGroupWarps) k_dp_group(GridView g, NetsV
     }
     __syncwarp();
 #pragma unroll 1
-    for (int r = 0; r < 5; r++) {
+    for (int r = 1; r < kMC; r <<= 1) {   // depth < kMC: log2(kMC) pointer-jumping rounds
         uint32_t nd[G], na[G];
 #pragma unroll
         for (int s = 0; s < G; s++) {
@@ -573,57 +693,10 @@ __global__ void __launch_bounds__(32 * kGroupWarps) k_dp_group(GridView g, NetsV
 // node waits only for its light children), so the CTA never synchronises per
 // tree level.  The backtrack walks the same paths top-down.
 
-#ifdef FGR_TIMING
-#define TMARK(i) do { if (threadIdx.x == 0) tm[i] = clock64(); } while (0)
-#else
-#define TMARK(i) do { } while (0)
-#endif
-
-// Packed G entry of a node without light children (K = V): value V(a,b), span (zlo[a], b).
-__device__ __forceinline__ unsigned long long gclosed(const Hdr* h, int a, int b) {
-    return ((unsigned long long)(h->viapre[b] - h->viapre[a]) << 8) | (unsigned)(h->zlo[a] << 4) | (unsigned)b;
-}
-
-__device__ __forceinline__ int ld_flag(const uint8_t* f) { return *(volatile const uint8_t*)f; }
-
-// min of N packed keys as a balanced tree (dependency depth log2 N instead of N)
-template <int N>
-__device__ __forceinline__ unsigned long long tree_min(unsigned long long (&k)[N]) {
-#pragma unroll
-    for (int s = 1; s < N; s <<= 1)
-#pragma unroll
-        for (int i = 0; i + s < N; i += 2 * s) k[i] = k[i + s] < k[i] ? k[i + s] : k[i];
-    return k[0];
-}
-
-template <int LT>
-__global__ void __launch_bounds__(32 * kLargeWarps, 1) k_dp_large(GridView g, NetsView nv, const int32_t* __restrict__ list,
-                                                                  int count, Out o, int commit) {
-    constexpr int G = 1;   // one lane group per warp: a path walk never shares its warp's issue slots
-    extern __shared__ __align__(16) unsigned char smem[];
-    Hdr* h = reinterpret_cast<Hdr*>(smem);
-    __shared__ int s_maxd, s_ticket, s_ticket2, s_npaths;
-    __shared__ unsigned long long s_root;
-    init_hdr(h, g);
-    if (threadIdx.x == 0) { s_maxd = 0; s_root = ~0ull; s_ticket = 0; s_ticket2 = 0; s_npaths = 0; }
-    const int nH = g.h.cnt, nV = g.v.cnt;
-    const int warp = threadIdx.x >> 5, lane = lane_id(), tid = threadIdx.x, T = blockDim.x;
-    const int gi = lane / LT < G ? lane / LT : G;
-    const int gl = lane - gi * LT;
-    const bool glane = gi < G && gl < LT;
-    const int gbase = gi * LT;
-    const unsigned gmask = glane ? (((1u << LT) - 1u) << gbase) : 0u;
-    const int idx = blockIdx.x;
-#ifdef FGR_TIMING
-    long long tm[8];
-#endif
-    TMARK(0);
-    const int net = list[idx];
-    const int a0 = nv.off[net];
-    const int m = nv.off[net + 1] - a0;
-    unsigned char* base = smem + a16(sizeof(Hdr));
-    const WScr w = carve_wscr(base + ((size_t)warp * G + (gi < G ? gi : 0)) * wscr_bytes(LT), LT);
-    const Tabs t = carve_tabs(base + (size_t)kLargeWarps * G * wscr_bytes(LT), m, LT, nH, nV, true);
+// Demand-independent tree analysis of a large net in shared memory: depths, child CSR,
+// level CSR, path decomposition (heavy child, path tops / bottoms) and the path queue.
+__device__ __forceinline__ void large_prologue(const Tabs& t, const NetsView& nv, int a0, int m, int tid, int T,
+                                               int warp, int lane, int* s_maxd, int* s_npaths, int* s_deep) {
     for (int i = tid; i < m; i += T) {
         const int p = nv.par[a0 + i];
         t.x[i] = nv.x[a0 + i]; t.y[i] = nv.y[a0 + i]; t.par[i] = (int16_t)p;
@@ -636,8 +709,6 @@ __global__ void __launch_bounds__(32 * kLargeWarps, 1) k_dp_large(GridView g, Ne
     uint32_t* dcnt = t.legV;
     for (int i = tid; i <= m; i += T) { cnt[i] = 0; dcnt[i] = 0; }
     __syncthreads();
-    LaneConst<LT> c;
-    c.load(h, gl);
     for (int i = 1 + tid; i < m; i += T) atomicAdd(&cnt[t.par[i]], 1u);
     // depth by pointer jumping: ceil(log2 m) rounds
     for (int r = 1; r < m; r <<= 1) {
@@ -660,9 +731,9 @@ __global__ void __launch_bounds__(32 * kLargeWarps, 1) k_dp_large(GridView g, Ne
         md = max(md, (int)t.depth[i]);
         atomicAdd(&dcnt[t.depth[i]], 1u);
     }
-    atomicMax(&s_maxd, md);
+    atomicMax(&(*s_maxd), md);
     __syncthreads();
-    const int maxd = s_maxd;
+    const int maxd = (*s_maxd);
     // warp 0: child CSR; warp 1: level CSR (exclusive scans)
     if (warp < 2) {
         const uint32_t* src = warp == 0 ? cnt : dcnt;
@@ -694,11 +765,10 @@ __global__ void __launch_bounds__(32 * kLargeWarps, 1) k_dp_large(GridView g, Ne
     // Path decomposition: the ancestors of the deepest node (ties: smallest index)
     // form the root path, every other node continues through its smallest-index
     // child.  Any decomposition is exact; this one puts the deepest chain on one path.
-    __shared__ int s_deep;
-    if (tid == 0) s_deep = 0x7FFFFFFF;
+    if (tid == 0) (*s_deep) = 0x7FFFFFFF;
     __syncthreads();
     for (int v = tid; v < m; v += T)
-        if (t.depth[v] == maxd) atomicMin(&s_deep, v);
+        if (t.depth[v] == maxd) atomicMin(&(*s_deep), v);
     for (int v = tid; v < m; v += T) {
         int best = -1;
         for (int k = t.cstart[v]; k < t.cstart[v + 1]; k++) {
@@ -709,7 +779,7 @@ __global__ void __launch_bounds__(32 * kLargeWarps, 1) k_dp_large(GridView g, Ne
     }
     __syncthreads();
     if (tid == 0)
-        for (int w = s_deep; w > 0; w = t.par[w]) t.hv[t.par[w]] = (uint16_t)w;
+        for (int w = (*s_deep); w > 0; w = t.par[w]) t.hv[t.par[w]] = (uint16_t)w;
     __syncthreads();
     // top of each node's heavy path by pointer jumping over heavy edges
     for (int v = tid; v < m; v += T) t.top[v] = (v > 0 && t.hv[t.par[v]] == v) ? (uint16_t)t.par[v] : (uint16_t)v;
@@ -742,9 +812,65 @@ __global__ void __launch_bounds__(32 * kLargeWarps, 1) k_dp_large(GridView g, Ne
             if (is_top) t.pq[n + __popc(b & ((1u << lane) - 1u))] = (uint16_t)v;
             n += __popc(b);
         }
-        if (lane == 0) s_npaths = n;
+        if (lane == 0) (*s_npaths) = n;
     }
+}
+
+#ifdef FGR_TIMING
+#define TMARK(i) do { if (threadIdx.x == 0) tm[i] = clock64(); } while (0)
+#else
+#define TMARK(i) do { } while (0)
+#endif
+
+__device__ __forceinline__ int ld_flag(const uint8_t* f) { return *(volatile const uint8_t*)f; }
+
+
+template <int LT>
+__global__ void __launch_bounds__(32 * kLargeWarps, 1) k_dp_large(GridView g, NetsView nv, const int32_t* __restrict__ list,
+                                                                  int count, Out o, int commit, Prep prep) {
+    constexpr int G = 1;   // one lane group per warp: a path walk never shares its warp's issue slots
+    extern __shared__ __align__(16) unsigned char smem[];
+    Hdr* h = reinterpret_cast<Hdr*>(smem);
+    __shared__ int s_maxd, s_ticket, s_ticket2, s_npaths, s_deep;
+    __shared__ unsigned long long s_root;
+    init_hdr(h, g);
+    if (threadIdx.x == 0) { s_maxd = 0; s_root = ~0ull; s_ticket = 0; s_ticket2 = 0; s_npaths = 0; }
+    const int nH = g.h.cnt, nV = g.v.cnt;
+    const int warp = threadIdx.x >> 5, lane = lane_id(), tid = threadIdx.x, T = blockDim.x;
+    const int gi = lane / LT < G ? lane / LT : G;
+    const int gl = lane - gi * LT;
+    const bool glane = gi < G && gl < LT;
+    const int gbase = gi * LT;
+    const unsigned gmask = glane ? (((1u << LT) - 1u) << gbase) : 0u;
+    const int idx = blockIdx.x;
+#ifdef FGR_TIMING
+    long long tm[8];
+#endif
+    TMARK(0);
+    const int net = list[idx];
+    const int a0 = nv.off[net];
+    const int m = nv.off[net + 1] - a0;
+    unsigned char* base = smem + a16(sizeof(Hdr));
+    const WScr w = carve_wscr(base + ((size_t)warp * G + (gi < G ? gi : 0)) * wscr_bytes(LT), LT);
+    const Tabs t = carve_tabs(base + (size_t)kLargeWarps * G * wscr_bytes(LT), m, LT, nH, nV, true);
+    if (prep.cs) {
+        // tree analysis precomputed once per stage by k_large_prep: just load it
+        for (int i = tid; i < m; i += T) {
+            t.x[i] = nv.x[a0 + i]; t.y[i] = nv.y[a0 + i]; t.par[i] = (int16_t)nv.par[a0 + i];
+            t.plo[i] = nv.plo[a0 + i]; t.phi[i] = nv.phi[a0 + i];
+            t.cstart[i] = prep.cs[a0 + i]; t.clist[i] = prep.cl[a0 + i]; t.hv[i] = prep.hv[a0 + i];
+            t.bot[i] = prep.bot[a0 + i]; t.pq[i] = prep.pq[a0 + i];
+            t.done[i] = 0; t.sready[i] = 0;
+        }
+        if (tid == 0) { t.cstart[m] = (uint16_t)(m - 1); s_npaths = prep.npaths[net]; }
+        __syncthreads();
+    } else {
+        large_prologue(t, nv, a0, m, tid, T, warp, lane, &s_maxd, &s_npaths, &s_deep);
+    }
+    LaneConst<LT> c;
+    c.load(h, gl);
     TMARK(1);
+    pdl_wait();   // everything above is demand-independent; the refresh must be done before the gathers
 #pragma unroll 2
     for (int task = tid; task < 4 * (m - 1); task += T) gather_task(g, t, task);
     __syncthreads();
@@ -1050,6 +1176,191 @@ __global__ void __launch_bounds__(32 * kLargeWarps, 1) k_dp_large(GridView g, Ne
     }
 }
 
+// One CTA per large net: the demand-independent tree analysis, written to global memory once per stage.
+template <int LT>
+__global__ void __launch_bounds__(32 * kLargeWarps, 1) k_large_prep(GridView g, NetsView nv, const int32_t* __restrict__ list,
+                                                                    uint16_t* cs, uint16_t* cl, uint16_t* hv, uint16_t* bot,
+                                                                    uint16_t* pq, int32_t* npaths) {
+    extern __shared__ __align__(16) unsigned char smem[];
+    __shared__ int s_maxd, s_npaths, s_deep;
+    if (threadIdx.x == 0) { s_maxd = 0; s_npaths = 0; }
+    const int nH = g.h.cnt, nV = g.v.cnt;
+    const int warp = threadIdx.x >> 5, lane = lane_id(), tid = threadIdx.x, T = blockDim.x;
+    const int net = list[blockIdx.x];
+    const int a0 = nv.off[net];
+    const int m = nv.off[net + 1] - a0;
+    const Tabs t = carve_tabs(smem + a16(sizeof(Hdr)) + (size_t)kLargeWarps * wscr_bytes(LT), m, LT, nH, nV, true);
+    large_prologue(t, nv, a0, m, tid, T, warp, lane, &s_maxd, &s_npaths, &s_deep);
+    __syncthreads();
+    for (int i = tid; i < m; i += T) {
+        cs[a0 + i] = t.cstart[i]; cl[a0 + i] = t.clist[i]; hv[a0 + i] = t.hv[i];
+        bot[a0 + i] = t.bot[i]; pq[a0 + i] = t.pq[i];
+    }
+    if (tid == 0) npaths[net] = s_npaths;
+}
+
+// ------------------------------------------------------------- thread kernel (2-node nets)
+// Half of all nets have one tree edge.  One thread routes one such net with the
+// whole DP in registers: leaf B(ls) and the root minimum in the closed form of
+// G for K = V (no light children), the edge step of Eqs. (1),(3),(5)-(7) over
+// both bends, the R11 tie-breaks, the backtrack and the commit.
+constexpr int kTwoThreads = 128;
+
+// leg costs for one leg into a transposed per-thread scratch column (stride kTwoThreads)
+__device__ __forceinline__ void leg_cost_col(const DirView& d, int line, int a, int b, uint32_t* col) {
+    const size_t pa = ((size_t)line * d.len + a) * d.W, pb = ((size_t)line * d.len + b) * d.W;
+    const size_t sa = ((size_t)line * d.nseg + (a >> FGR_SEG_SHIFT)) * d.W;
+    const size_t sb = ((size_t)line * d.nseg + (b >> FGR_SEG_SHIFT)) * d.W;
+    const int nq = d.W >> 2;
+#pragma unroll
+    for (int q = 0; q < 4; q++) {
+        if (q < nq) {
+            const uint4 Pa = __ldg(reinterpret_cast<const uint4*>(d.P + pa) + q);
+            const uint4 Pb = __ldg(reinterpret_cast<const uint4*>(d.P + pb) + q);
+            const uint4 Sa = __ldg(reinterpret_cast<const uint4*>(d.SB + sa) + q);
+            const uint4 Sb = __ldg(reinterpret_cast<const uint4*>(d.SB + sb) + q);
+            col[(4 * q + 0) * kTwoThreads] = (Sb.x + Pb.x) - (Sa.x + Pa.x);
+            col[(4 * q + 1) * kTwoThreads] = (Sb.y + Pb.y) - (Sa.y + Pa.y);
+            col[(4 * q + 2) * kTwoThreads] = (Sb.z + Pb.z) - (Sa.z + Pa.z);
+            col[(4 * q + 3) * kTwoThreads] = (Sb.w + Pb.w) - (Sa.w + Pa.w);
+        }
+    }
+}
+
+template <int LT>
+__global__ void __launch_bounds__(kTwoThreads) k_dp_two(GridView g, NetsView nv, const int32_t* __restrict__ list,
+                                                        int count, Out o, int commit) {
+    __shared__ Hdr hs;
+    __shared__ uint32_t legs[4 * 16 * kTwoThreads];   // [leg][slot][thread]
+    init_hdr(&hs, g);
+    __syncthreads();
+    const int tid = threadIdx.x;
+    const int idx = blockIdx.x * kTwoThreads + tid;
+    if (idx >= count) return;
+    uint32_t vp[LT], zl[LT], sl[LT];
+    uint32_t hmask = 0;
+#pragma unroll
+    for (int l = 0; l < LT; l++) {
+        vp[l] = hs.viapre[l]; zl[l] = hs.zlo[l]; sl[l] = hs.slot[l];
+        hmask |= (hs.dir[l] == 0 ? 1u : 0u) << l;
+    }
+    const int net = list[idx];
+    const int a0 = nv.off[net];
+    if (nv.off[net + 1] - a0 < 2) {   // trivial net: no edge, cost 0
+        if (o.rec_seg) { o.rec_seg[o.rec_off[o.list_base + idx]] = 0xFFFFFFFFu; o.rec_cost[o.list_base + idx] = 0; }
+        else { o.seg[a0] = 0xFFFFFFFFu; o.cost[net] = 0; }
+        return;
+    }
+    const int x0 = nv.x[a0], y0 = nv.y[a0], x1 = nv.x[a0 + 1], y1 = nv.y[a0 + 1];
+    const int plo0 = nv.plo[a0], phi0 = nv.phi[a0], plo1 = nv.plo[a0 + 1], phi1 = nv.phi[a0 + 1];
+    const bool sh = (y0 == y1), sv = (x0 == x1), straight = sh || sv;
+    uint32_t* col = legs + tid;
+    // legs: 0 = H row y1, 1 = H row y0, 2 = V col x1, 3 = V col x0   (x1..x0 / y1..y0)
+    const int xa = min(x0, x1), xb = max(x0, x1), ya = min(y0, y1), yb = max(y0, y1);
+    if (!sv) leg_cost_col(g.h, y1, xa, xb, col + 0 * 16 * kTwoThreads);
+    if (!straight) leg_cost_col(g.h, y0, xa, xb, col + 1 * 16 * kTwoThreads);
+    if (!sh) leg_cost_col(g.v, x1, ya, yb, col + 2 * 16 * kTwoThreads);
+    if (!straight) leg_cost_col(g.v, x0, ya, yb, col + 3 * 16 * kTwoThreads);
+    uint32_t c1[LT], c2[LT];   // leg 1 on layer l (from the leaf), leg 2 on layer l (into the root)
+#pragma unroll
+    for (int l = 0; l < LT; l++) {
+        const bool hl = (hmask >> l) & 1u;
+        c1[l] = col[((hl ? 0 : 2) * 16 + sl[l]) * kTwoThreads];
+        c2[l] = straight ? 0u : col[((hl ? 1 : 3) * 16 + sl[l]) * kTwoThreads];
+    }
+    // leaf: B(ls) = G(a, b), a = min(ls, pin_lo), b = max(ls, pin_hi), closed form (K = V)
+    uint32_t vplo = 0, vphi = 0, zplo = 0;
+#pragma unroll
+    for (int l = 0; l < LT; l++) {
+        vplo = (l == plo1) ? vp[l] : vplo;
+        vphi = (l == phi1) ? vp[l] : vphi;
+        zplo = (l == plo1) ? zl[l] : zplo;
+    }
+    uint32_t Bv[LT];
+    uint8_t recB[LT];
+#pragma unroll
+    for (int ls = 0; ls < LT; ls++) {
+        uint32_t va, vb, za, bb;
+        if (plo1 >= 0) {
+            va = ls <= plo1 ? vp[ls] : vplo;
+            za = ls <= plo1 ? zl[ls] : zplo;
+            vb = ls >= phi1 ? vp[ls] : vphi;
+            bb = ls >= phi1 ? (uint32_t)ls : (uint32_t)phi1;
+        } else {
+            va = vb = vp[ls]; za = zl[ls]; bb = ls;
+        }
+        Bv[ls] = vb - va;
+        recB[ls] = (uint8_t)((za << 4) | bb);
+    }
+    // edge: E(lt), recE(lt)
+    uint32_t E[LT];
+    uint8_t recE[LT];
+    const int de = sh ? 0 : 1;
+#pragma unroll
+    for (int lt = 0; lt < LT; lt++) {
+        const bool hlt = (hmask >> lt) & 1u;
+        uint32_t best = FGR_INF;
+        int bls = lt;
+        if (straight) {
+            if ((hlt ? 0 : 1) == de) best = sat_add(Bv[lt], c1[lt]);
+        } else {
+#pragma unroll
+            for (int ls = 0; ls < LT; ls++) {
+                const bool hls = (hmask >> ls) & 1u;
+                if (hls != hlt) {
+                    const uint32_t via = vp[ls] > vp[lt] ? vp[ls] - vp[lt] : vp[lt] - vp[ls];
+                    const uint32_t cst = sat_add(sat_add(sat_add(Bv[ls], c1[ls]), via), c2[lt]);
+                    if (cst < best) { best = cst; bls = ls; }
+                }
+            }
+        }
+        E[lt] = best;
+        recE[lt] = (uint8_t)bls;
+    }
+    // root, generalised Eq. (4): min over l of E(l) + G(hull({l} + pins))
+    uint32_t vrlo = 0, vrhi = 0, zrlo = 0;
+#pragma unroll
+    for (int l = 0; l < LT; l++) {
+        vrlo = (l == plo0) ? vp[l] : vrlo;
+        vrhi = (l == phi0) ? vp[l] : vrhi;
+        zrlo = (l == plo0) ? zl[l] : zrlo;
+    }
+    unsigned long long kk[LT];
+#pragma unroll
+    for (int l = 0; l < LT; l++) {
+        uint32_t va, vb, za, bb;
+        if (plo0 >= 0) {
+            va = l <= plo0 ? vp[l] : vrlo;
+            za = l <= plo0 ? zl[l] : zrlo;
+            vb = l >= phi0 ? vp[l] : vrhi;
+            bb = l >= phi0 ? (uint32_t)l : (uint32_t)phi0;
+        } else {
+            va = vb = vp[l]; za = zl[l]; bb = l;
+        }
+        kk[l] = ((unsigned long long)sat_add(E[l], vb - va) << 8) | (za << 4) | bb;
+    }
+    const unsigned long long rk = tree_min<LT>(kk);
+    // backtrack: lt = smallest layer in the root span minimising E (R11)
+    const int lo = (int)((rk >> 4) & 15), hi = (int)(rk & 15);
+    uint32_t be = FGR_INF + 1u;
+    int lt = lo, ls = lo;
+#pragma unroll
+    for (int l = 0; l < LT; l++)
+        if (l >= lo && l <= hi && E[l] < be) { be = E[l]; lt = l; ls = recE[l]; }
+    (void)recB;
+    const uint32_t bend = straight ? 0u : (((hmask >> lt) & 1u) ? 1u : 0u);
+    const uint32_t sg = bend | ((uint32_t)ls << 8) | ((uint32_t)lt << 16) | ((uint32_t)(straight ? 1 : 0) << 24);
+    if (o.rec_seg) {
+        uint32_t* rs = o.rec_seg + o.rec_off[o.list_base + idx];
+        rs[0] = 0xFFFFFFFFu; rs[1] = sg;
+        o.rec_cost[o.list_base + idx] = (uint32_t)(rk >> 8);
+    } else {
+        o.seg[a0] = 0xFFFFFFFFu; o.seg[a0 + 1] = sg;
+        o.cost[net] = (uint32_t)(rk >> 8);
+    }
+    if (commit) commit_edge(g, &hs, x1, y1, x0, y0, sg);
+}
+
 // Commit from route records (multi-GPU: after the exchange every rank commits every net).
 __global__ void __launch_bounds__(256) k_commit_records(GridView g, NetsView nv, const int32_t* __restrict__ list, int count,
                                                         const uint32_t* __restrict__ rec_seg,
@@ -1071,8 +1382,8 @@ __global__ void __launch_bounds__(256) k_commit_records(GridView g, NetsView nv,
 }
 
 // ------------------------------------------------------------- host side
-size_t smem_group(int L, int nH, int nV) {
-    return a16(sizeof(Hdr)) + (size_t)kGroupWarps * groups_of(L) * (tabs_bytes(kMC, L, nH, nV, false) + wscr_bytes(L));
+size_t smem_group(int L, int nH, int nV, int mc) {
+    return a16(sizeof(Hdr)) + (size_t)kGroupWarps * groups_of(L) * (tabs_bytes(mc, L, nH, nV, false) + wscr_bytes(L));
 }
 
 size_t smem_large(int L, int nH, int nV, int m) {
@@ -1080,8 +1391,8 @@ size_t smem_large(int L, int nH, int nV, int m) {
 }
 
 template <int LT>
-cudaError_t launch_lt(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int count, int nlarge,
-                      int maxm_large, const Out& o, bool commit) {
+cudaError_t launch_lt(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int nlarge, int nmidL,
+                      int nmidS, int ntwo, int maxm_large, const Out& o, bool commit, const Prep& prep) {
     static bool configured = false;   // one device per process is the supported configuration
     if (!configured) {
         cudaFuncAttributes fa;
@@ -1089,64 +1400,134 @@ cudaError_t launch_lt(fgr_grid* g, cudaStream_t st, const NetsView& nv, const in
         if (e == cudaSuccess)
             e = cudaFuncSetAttribute(k_dp_large<LT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                      g->max_smem - (int)fa.sharedSizeBytes);
-        if (e == cudaSuccess) e = cudaFuncGetAttributes(&fa, k_dp_group<LT>);
+        if (e == cudaSuccess) e = cudaFuncGetAttributes(&fa, k_large_prep<LT>);
         if (e == cudaSuccess)
-            e = cudaFuncSetAttribute(k_dp_group<LT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+            e = cudaFuncSetAttribute(k_large_prep<LT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                     g->max_smem - (int)fa.sharedSizeBytes);
+        if (e == cudaSuccess) e = cudaFuncGetAttributes(&fa, k_dp_group<LT, FGR_SMALL_NET>);
+        if (e == cudaSuccess)
+            e = cudaFuncSetAttribute(k_dp_group<LT, FGR_SMALL_NET>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                     g->max_smem - (int)fa.sharedSizeBytes);
+        if (e == cudaSuccess) e = cudaFuncGetAttributes(&fa, k_dp_group<LT, FGR_MID_NET>);
+        if (e == cudaSuccess)
+            e = cudaFuncSetAttribute(k_dp_group<LT, FGR_MID_NET>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                      g->max_smem - (int)fa.sharedSizeBytes);
         if (e != cudaSuccess) return e;
         configured = true;
     }
     const GridView& v = g->view;
-    const int nsmall = count - nlarge;
-    // Large and small nets of one batch are independent: when both exist the small
-    // nets run on a side stream beside the large-net CTAs (fork/join with events).
-    const bool fork = nlarge > 0 && nsmall > 0;
-    cudaStream_t ss = fork ? g->side : st;
+    // The four size classes of one batch are independent: each non-empty class gets its
+    // own stream (forked from and joined back into the caller's stream).
+    const int cls_n[4] = {nlarge, nmidL, nmidS, ntwo};
+    int used = 0;
+    for (int k = 0; k < 4; k++) used += cls_n[k] > 0;
+    const bool fork = used > 1;
     cudaError_t e;
     if (fork) {
+        // recorded before any launch: the side streams wait for the refresh, not for the large class
         if ((e = cudaEventRecord(g->ev_fork, st)) != cudaSuccess) return e;
-        if ((e = cudaStreamWaitEvent(g->side, g->ev_fork, 0)) != cudaSuccess) return e;
+        for (int i = 0; i < 3; i++)
+            if ((e = cudaStreamWaitEvent(g->side[i], g->ev_fork, 0)) != cudaSuccess) return e;
     }
-    if (nsmall > 0) {
-        Out os = o;
-        os.list_base = o.list_base + nlarge;
-        const int per_cta = kGroupWarps * groups_of(LT);
-        const int ps = fgr_prof_begin(g, PROF_DP_SMALL, ss);
-        k_dp_group<LT><<<(nsmall + per_cta - 1) / per_cta, 32 * kGroupWarps, smem_group(LT, g->nH, g->nV), ss>>>(
-            v, nv, list + nlarge, nsmall, os, commit ? 1 : 0);
-        fgr_prof_end(g, ps, ss);
-        g->stats.kernel_launches++;
-        if ((e = cudaGetLastError()) != cudaSuccess) return e;
-    }
-    if (nlarge > 0) {
-        const int ps = fgr_prof_begin(g, PROF_DP_LARGE, st);
-        k_dp_large<LT><<<nlarge, 32 * kLargeWarps, smem_large(LT, g->nH, g->nV, maxm_large), st>>>(
-            v, nv, list, nlarge, o, commit ? 1 : 0);
-        fgr_prof_end(g, ps, st);
-        g->stats.kernel_launches++;
-        if ((e = cudaGetLastError()) != cudaSuccess) return e;
+    cudaStream_t sk[4] = {st, fork ? g->side[0] : st, fork ? g->side[1] : st, fork ? g->side[2] : st};
+    int base = 0;
+    for (int k = 0; k < 4; k++) {
+        const int n = cls_n[k];
+        if (n > 0) {
+            Out os = o;
+            os.list_base = o.list_base + base;
+            const int32_t* l = list + base;
+            const int ps = fgr_prof_begin(g, k == 0 ? PROF_DP_LARGE : PROF_DP_SMALL, sk[k]);
+            if (k == 0) {
+                // programmatic dependent launch: the prologue overlaps the refresh that precedes it
+                cudaLaunchConfig_t cfg = {};
+                cfg.gridDim = dim3(n);
+                cfg.blockDim = dim3(32 * kLargeWarps);
+                cfg.dynamicSmemBytes = smem_large(LT, g->nH, g->nV, maxm_large);
+                cfg.stream = sk[k];
+                cudaLaunchAttribute at[1];
+                at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+                at[0].val.programmaticStreamSerializationAllowed = 1;
+                cfg.attrs = at;
+                cfg.numAttrs = 1;
+                e = cudaLaunchKernelEx(&cfg, k_dp_large<LT>, v, nv, l, n, os, commit ? 1 : 0, prep);
+                if (e != cudaSuccess) return e;
+            }
+            else if (k == 1) {
+                const int per_cta = kGroupWarps * groups_of(LT);
+                k_dp_group<LT, FGR_SMALL_NET><<<(n + per_cta - 1) / per_cta, 32 * kGroupWarps,
+                                                 smem_group(LT, g->nH, g->nV, FGR_SMALL_NET), sk[k]>>>(v, nv, l, n, os,
+                                                                                                      commit ? 1 : 0);
+            } else if (k == 2) {
+                const int per_cta = kGroupWarps * groups_of(LT);
+                k_dp_group<LT, FGR_MID_NET><<<(n + per_cta - 1) / per_cta, 32 * kGroupWarps,
+                                               smem_group(LT, g->nH, g->nV, FGR_MID_NET), sk[k]>>>(v, nv, l, n, os,
+                                                                                                  commit ? 1 : 0);
+            } else {
+                k_dp_two<LT><<<(n + kTwoThreads - 1) / kTwoThreads, kTwoThreads, 0, sk[k]>>>(v, nv, l, n, os,
+                                                                                              commit ? 1 : 0);
+            }
+            fgr_prof_end(g, ps, sk[k]);
+            g->stats.kernel_launches++;
+            if ((e = cudaGetLastError()) != cudaSuccess) return e;
+        }
+        base += n;
     }
     if (fork) {
-        if ((e = cudaEventRecord(g->ev_join, g->side)) != cudaSuccess) return e;
-        if ((e = cudaStreamWaitEvent(st, g->ev_join, 0)) != cudaSuccess) return e;
+        for (int i = 0; i < 3; i++) {
+            if ((e = cudaEventRecord(g->ev_join[i], g->side[i])) != cudaSuccess) return e;
+            if ((e = cudaStreamWaitEvent(st, g->ev_join[i], 0)) != cudaSuccess) return e;
+        }
     }
     return cudaSuccess;
 }
 
 }  // namespace
 
-size_t fgr_dp_smem_small(const fgr_grid* g) { return smem_group(g->L, g->nH, g->nV); }
+size_t fgr_dp_smem_small(const fgr_grid* g) { return smem_group(g->L, g->nH, g->nV, FGR_SMALL_NET); }
 
 size_t fgr_dp_smem_large(const fgr_grid* g, int m) { return smem_large(g->L, g->nH, g->nV, m); }
 
-cudaError_t fgr_launch_dp(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int count, int nlarge,
-                          int maxm_large, uint32_t* seg_out, uint32_t* cost_out, uint32_t* rec_seg,
-                          const int32_t* rec_off, uint32_t* rec_cost, int list_base, bool commit) {
+cudaError_t fgr_launch_dp(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int nlarge, int nmidL,
+                          int nmidS, int ntwo, int maxm_large, uint32_t* seg_out, uint32_t* cost_out, uint32_t* rec_seg,
+                          const int32_t* rec_off, uint32_t* rec_cost, int list_base, bool commit, const Prep* prep) {
+    const Prep pz = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
+    const Prep& pp = prep ? *prep : pz;
     Out o;
     o.seg = seg_out; o.cost = cost_out; o.rec_seg = rec_seg; o.rec_off = rec_off; o.rec_cost = rec_cost;
     o.list_base = list_base;
     switch (g->L) {
-#define FGR_LT(n) case n: return launch_lt<n>(g, st, nv, list, count, nlarge, maxm_large, o, commit);
+#define FGR_LT(n) case n: return launch_lt<n>(g, st, nv, list, nlarge, nmidL, nmidS, ntwo, maxm_large, o, commit, pp);
+        FGR_LT(2) FGR_LT(3) FGR_LT(4) FGR_LT(5) FGR_LT(6) FGR_LT(7) FGR_LT(8) FGR_LT(9) FGR_LT(10) FGR_LT(11)
+        FGR_LT(12) FGR_LT(13) FGR_LT(14) FGR_LT(15) FGR_LT(16)
+#undef FGR_LT
+        default: return cudaErrorInvalidValue;
+    }
+}
+
+namespace {
+template <int LT>
+cudaError_t launch_prep_lt(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int count, int maxm,
+                           uint16_t* cs, uint16_t* cl, uint16_t* hv, uint16_t* bot, uint16_t* pq, int32_t* np) {
+    cudaFuncAttributes fa;
+    cudaError_t e = cudaFuncGetAttributes(&fa, k_large_prep<LT>);
+    if (e == cudaSuccess)
+        e = cudaFuncSetAttribute(k_large_prep<LT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 g->max_smem - (int)fa.sharedSizeBytes);
+    if (e != cudaSuccess) return e;
+    k_large_prep<LT><<<count, 32 * kLargeWarps, smem_large(LT, g->nH, g->nV, maxm), st>>>(g->view, nv, list, cs, cl, hv,
+                                                                                        bot, pq, np);
+    g->stats.kernel_launches++;
+    return cudaGetLastError();
+}
+}  // namespace
+
+cudaError_t fgr_launch_large_prep(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int count,
+                                  int maxm, uint16_t* cs, uint16_t* cl, uint16_t* hv, uint16_t* bot, uint16_t* pq,
+                                  int32_t* np) {
+    if (count <= 0) return cudaSuccess;
+    switch (g->L) {
+#define FGR_LT(n) case n: return launch_prep_lt<n>(g, st, nv, list, count, maxm, cs, cl, hv, bot, pq, np);
         FGR_LT(2) FGR_LT(3) FGR_LT(4) FGR_LT(5) FGR_LT(6) FGR_LT(7) FGR_LT(8) FGR_LT(9) FGR_LT(10) FGR_LT(11)
         FGR_LT(12) FGR_LT(13) FGR_LT(14) FGR_LT(15) FGR_LT(16)
 #undef FGR_LT

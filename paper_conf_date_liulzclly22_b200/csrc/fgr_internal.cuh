@@ -29,7 +29,8 @@
 #define FGR_CHUNK_SEGS 8    // segments per refresh task (one warp)
 #define FGR_INF 0x7FFFFFFFu // "impossible" cost; finite costs are < FGR_INF (R19)
 #define FGR_MAXL 16
-#define FGR_SMALL_NET 32    // nets with <= this many nodes take the warp path
+#define FGR_SMALL_NET 32    // nets with <= this many nodes take the lane-group path
+#define FGR_MID_NET 8       // ... with a node capacity of 8 (3..8 nodes) or 32 (9..32 nodes)
 #define FGR_CTA_THREADS 256
 #define FGR_WARPS_PER_CTA (FGR_CTA_THREADS / 32)
 
@@ -73,6 +74,16 @@ struct NetsView {
 };
 
 // ------------------------------------------------------------------ host state
+// Per-node results of the large-net tree analysis (global, indexed by global node index).
+struct Prep {
+    const uint16_t* cs;    // child CSR start (net-local); cs of local m is m - 1 and not stored
+    const uint16_t* cl;    // child list
+    const uint16_t* hv;    // heavy child
+    const uint16_t* bot;   // bottom of the path topped by the node
+    const uint16_t* pq;    // path queue (path tops, deepest first)
+    const int32_t* npaths; // [num_nets]
+};
+
 struct PlanCache {
     bool valid = false;
     fgr_nets nets{};
@@ -83,6 +94,11 @@ struct PlanCache {
     int* h_off = nullptr;      // [B+1]
     int* h_nlarge = nullptr;   // [B]
     int* h_maxm = nullptr;     // [B] max nodes of a large net in the batch
+    int* h_ntwo = nullptr;     // [B] 2-node nets (the tail of each batch in exec order)
+    int* h_n9 = nullptr;       // [B] nets with 9..32 nodes
+    const int32_t* exec = nullptr;  // exec order actually used (order itself, or a re-sorted copy)
+    bool prep_valid = false;        // large-net tree analysis computed for these nets
+    Prep prep{};
     long long* h_segb = nullptr;  // [B] upper bound on segments the batch can dirty
     int cap = 0;
 };
@@ -128,12 +144,13 @@ struct fgr_grid {
     ncclComm_t comm = nullptr;
     int rank = 0, world = 1;
     Scratch s_rec[4];
+    Scratch s_prep;
     fgr_stats stats{};
     int max_smem = 0;
     int num_sms = 0;
     Profiler prof;
-    cudaStream_t side = nullptr;      // second stream: small nets run beside the large-net CTAs
-    cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+    cudaStream_t side[3] = {nullptr, nullptr, nullptr};   // size classes of one batch run side by side
+    cudaEvent_t ev_fork = nullptr, ev_join[3] = {nullptr, nullptr, nullptr};
 };
 
 // Profiling brackets around a launch (no-ops unless fgr_profile_enable(grid, 1)).
@@ -156,10 +173,14 @@ void* fgr_scratch(Scratch& s, size_t bytes, cudaError_t* err);
 // launchers (defined in the .cu files)
 cudaError_t fgr_launch_refresh(fgr_grid* g, cudaStream_t st, bool full);
 cudaError_t fgr_launch_refresh_sized(fgr_grid* g, cudaStream_t st, bool full, long long max_tasks);
-cudaError_t fgr_launch_dp(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int count,
-                          int nlarge, int maxm_large, uint32_t* seg_out, uint32_t* cost_out,
+// list = [large (> 32 nodes) | midL (9..32) | midS (3..8) | two (2 nodes)] nets, contiguous
+cudaError_t fgr_launch_dp(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int nlarge,
+                          int nmidL, int nmidS, int ntwo, int maxm_large, uint32_t* seg_out, uint32_t* cost_out,
                           uint32_t* rec_seg, const int32_t* rec_off, uint32_t* rec_cost, int list_base,
-                          bool commit);
+                          bool commit, const Prep* prep);
+cudaError_t fgr_launch_large_prep(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int count,
+                                  int maxm, uint16_t* cs, uint16_t* cl, uint16_t* hv, uint16_t* bot, uint16_t* pq,
+                                  int32_t* np);
 cudaError_t fgr_launch_commit(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int count,
                               const uint32_t* rec_seg, const int32_t* rec_off, int list_base);
 size_t fgr_dp_smem_small(const fgr_grid* g);
@@ -176,6 +197,12 @@ static inline NetsView fgr_nets_view(const fgr_nets* n) {
 __device__ __forceinline__ uint32_t sat_add(uint32_t a, uint32_t b) { return __viaddmin_u32(a, b, FGR_INF); }
 
 __device__ __forceinline__ int lane_id() { return threadIdx.x & 31; }
+
+// Programmatic dependent launch (sm_90+): let the next kernel on the stream start its
+// demand-independent prologue early; wait for the previous kernel before touching its
+// results.  Both are no-ops when the launch did not request PDL.
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
 
 template <int N>
 struct U32Vec { uint32_t v[N]; };

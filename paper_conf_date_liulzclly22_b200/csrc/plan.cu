@@ -265,7 +265,8 @@ __global__ void k_batch_keys(int R, const int* __restrict__ color, const unsigne
 __global__ void k_finalize(int N, const int* __restrict__ counters, const unsigned long long* __restrict__ keys,
                            const unsigned long long* __restrict__ bkeys, const int* __restrict__ msize,
                            const int* __restrict__ segb, int* __restrict__ order, int* __restrict__ batch_of_net,
-                           int* __restrict__ nlarge, int* __restrict__ maxm, unsigned long long* __restrict__ segsum) {
+                           int* __restrict__ nlarge, int* __restrict__ maxm, unsigned long long* __restrict__ segsum,
+                           int* __restrict__ ntwo, int* __restrict__ n9) {
     const int i = blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= N) return;
     const int R = N - counters[0];
@@ -286,9 +287,17 @@ __global__ void k_finalize(int N, const int* __restrict__ counters, const unsign
         const int c0 = __shfl_sync(act, c, lead);
         if (__all_sync(act, c == c0)) {
             const unsigned sum = __reduce_add_sync(act, (unsigned)v);
-            if (lane_id() == lead) atomicAdd(&segsum[c], (unsigned long long)sum);
+            const unsigned two = __reduce_add_sync(act, m == 2 ? 1u : 0u);
+            const unsigned nine = __reduce_add_sync(act, (m > FGR_MID_NET && m <= FGR_SMALL_NET) ? 1u : 0u);
+            if (lane_id() == lead) {
+                atomicAdd(&segsum[c], (unsigned long long)sum);
+                if (two) atomicAdd(&ntwo[c], (int)two);
+                if (nine) atomicAdd(&n9[c], (int)nine);
+            }
         } else {
             atomicAdd(&segsum[c], v);
+            if (m == 2) atomicAdd(&ntwo[c], 1);
+            if (m > FGR_MID_NET && m <= FGR_SMALL_NET) atomicAdd(&n9[c], 1);
         }
     } else {
         const int id = (int)(keys[i] & 0xFFFFFFFFu);
@@ -334,6 +343,8 @@ extern "C" FGR_API fgr_status fgr_plan(fgr_grid* g, const fgr_nets* nets, int32_
         FGR_CHECK_CUDA(g, cudaMemsetAsync(batch_offset, 0, sizeof(int32_t), st));
         FGR_CHECK_CUDA(g, cudaStreamSynchronize(st));
         g->cache.valid = true;
+        g->cache.prep_valid = false;
+        g->cache.exec = order;
         g->cache.nets = *nets; g->cache.order = order; g->cache.batch_offset = batch_offset; g->cache.num_batches = 0;
         return FGR_OK;
     }
@@ -419,12 +430,14 @@ extern "C" FGR_API fgr_status fgr_plan(fgr_grid* g, const fgr_nets* nets, int32_
         FGR_CHECK_CUDA(g, cudaGetLastError());
     }
     // colouring
-    auto* bc = take<int>(g, 11, 3 * ((size_t)R + 1), &e);   // bcount | nlarge | maxm
+    auto* bc = take<int>(g, 11, 5 * ((size_t)R + 1), &e);   // bcount | nlarge | maxm | ntwo | n9
     if (e != cudaSuccess) return fgr_cuda_fail(g, e, "plan batch scratch");
     int* d_bcount = bc;
     int* d_nlarge = bc + (R + 1);
     int* d_maxm = bc + 2 * (R + 1);
-    FGR_CHECK_CUDA(g, cudaMemsetAsync(bc, 0, 3 * sizeof(int) * ((size_t)R + 1), st));
+    int* d_ntwo = bc + 3 * (R + 1);
+    int* d_n9 = bc + 4 * (R + 1);
+    FGR_CHECK_CUDA(g, cudaMemsetAsync(bc, 0, 5 * sizeof(int) * ((size_t)R + 1), st));
     FGR_CHECK_CUDA(g, cudaMemsetAsync(color, 0xFF, sizeof(int) * ((size_t)N + 1), st));
     FGR_CHECK_CUDA(g, cudaMemsetAsync(batch_of_net, 0xFF, sizeof(int) * (size_t)N, st));
     if (R > 0) {
@@ -463,7 +476,7 @@ extern "C" FGR_API fgr_status fgr_plan(fgr_grid* g, const fgr_nets* nets, int32_
     auto* segsum = (unsigned long long*)box_r;   // box_r no longer needed after colouring
     FGR_CHECK_CUDA(g, cudaMemsetAsync(segsum, 0, sizeof(unsigned long long) * ((size_t)R + 1), st));
     k_finalize<<<(N + 255) / 256, 256, 0, st>>>(N, counters, keys_s, bkeys_s, msize, segb, order, batch_of_net,
-                                                d_nlarge, d_maxm, segsum);
+                                                d_nlarge, d_maxm, segsum, d_ntwo, d_n9);
     FGR_CHECK_CUDA(g, cudaGetLastError());
     g->stats.kernel_launches += 6;
     int B = 0;
@@ -471,20 +484,26 @@ extern "C" FGR_API fgr_status fgr_plan(fgr_grid* g, const fgr_nets* nets, int32_
     FGR_CHECK_CUDA(g, cudaStreamSynchronize(st));  // sync 2 of 2
     PlanCache& c = g->cache;
     if (c.cap < B + 1) {
-        free(c.h_off); free(c.h_nlarge); free(c.h_maxm);
+        free(c.h_off); free(c.h_nlarge); free(c.h_maxm); free(c.h_segb); free(c.h_ntwo); free(c.h_n9);
         c.cap = B + 1;
         c.h_off = (int*)malloc(sizeof(int) * c.cap);
         c.h_nlarge = (int*)malloc(sizeof(int) * c.cap);
         c.h_maxm = (int*)malloc(sizeof(int) * c.cap);
         c.h_segb = (long long*)malloc(sizeof(long long) * c.cap);
+        c.h_ntwo = (int*)malloc(sizeof(int) * c.cap);
+        c.h_n9 = (int*)malloc(sizeof(int) * c.cap);
     }
     if (B > 0) {
         FGR_CHECK_CUDA(g, cudaMemcpy(c.h_off, batch_offset, sizeof(int) * (B + 1), cudaMemcpyDeviceToHost));
         FGR_CHECK_CUDA(g, cudaMemcpy(c.h_nlarge, d_nlarge, sizeof(int) * B, cudaMemcpyDeviceToHost));
         FGR_CHECK_CUDA(g, cudaMemcpy(c.h_maxm, d_maxm, sizeof(int) * B, cudaMemcpyDeviceToHost));
+        FGR_CHECK_CUDA(g, cudaMemcpy(c.h_ntwo, d_ntwo, sizeof(int) * B, cudaMemcpyDeviceToHost));
+        FGR_CHECK_CUDA(g, cudaMemcpy(c.h_n9, d_n9, sizeof(int) * B, cudaMemcpyDeviceToHost));
         FGR_CHECK_CUDA(g, cudaMemcpy(c.h_segb, segsum, sizeof(long long) * B, cudaMemcpyDeviceToHost));
     }
     c.valid = true;
+    c.prep_valid = false;
+    c.exec = order;
     c.nets = *nets;
     c.order = order;
     c.batch_offset = batch_offset;

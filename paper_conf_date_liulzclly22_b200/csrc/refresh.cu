@@ -186,6 +186,8 @@ __device__ __forceinline__ int refresh_chunk(const GridView& g, const DirView& d
 
 template <int WH, int WV>
 __global__ void __launch_bounds__(256) k_refresh(GridView g, int full) {
+    pdl_trigger();   // the next DP kernel may start its prologue now
+    pdl_wait();      // the previous batch's commits must be complete
     const int chH = (g.h.nseg + FGR_CHUNK_SEGS - 1) / FGR_CHUNK_SEGS;
     const int chV = (g.v.nseg + FGR_CHUNK_SEGS - 1) / FGR_CHUNK_SEGS;
     const int tH = g.h.lines * chH;

@@ -16,18 +16,29 @@
 
 namespace {
 
+// route_batch: split a net list into large (> 32 nodes) | midL (9..32) | midS (3..8) | two (2 nodes)
+__device__ __forceinline__ int size_class(int m) {
+    return m > FGR_SMALL_NET ? 0 : (m > FGR_MID_NET ? 1 : (m > 2 ? 2 : 3));   // m <= 2 (incl. trivial) -> 3
+}
+
 __global__ void k_classify(int count, const int32_t* __restrict__ ids, const int32_t* __restrict__ off,
-                           int32_t* __restrict__ out, int* __restrict__ ctr /* [0] large, [1] small, [2] maxm */) {
+                           int32_t* __restrict__ tmp, int* __restrict__ ctr /* [0..3] class counts, [4] maxm */) {
     const int i = blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= count) return;
     const int id = ids[i];
     const int m = off[id + 1] - off[id];
-    if (m > FGR_SMALL_NET) {
-        out[atomicAdd(&ctr[0], 1)] = id;
-        atomicMax(&ctr[2], m);
-    } else {
-        out[count - 1 - atomicAdd(&ctr[1], 1)] = id;
-    }
+    const int k = size_class(m);
+    tmp[(size_t)k * count + atomicAdd(&ctr[k], 1)] = id;
+    if (k == 0) atomicMax(&ctr[4], m);
+}
+
+__global__ void k_concat4(int count, const int32_t* __restrict__ tmp, const int* __restrict__ ctr,
+                          int32_t* __restrict__ out) {
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= count) return;
+    int k = 0, base = 0;
+    while (k < 3 && i >= base + ctr[k]) { base += ctr[k]; k++; }
+    out[i] = tmp[(size_t)k * count + (i - base)];
 }
 
 __global__ void k_net_sizes(int n, const int32_t* __restrict__ order, const int32_t* __restrict__ off,
@@ -39,24 +50,45 @@ __global__ void k_net_sizes(int n, const int32_t* __restrict__ order, const int3
 __global__ void k_batch_info(int B, const int32_t* __restrict__ boff, const int32_t* __restrict__ order,
                              const int32_t* __restrict__ off, const int16_t* __restrict__ x,
                              const int16_t* __restrict__ y, const int32_t* __restrict__ par,
-                             int* __restrict__ nlarge, int* __restrict__ maxm, unsigned long long* __restrict__ segb) {
+                             int* __restrict__ nlarge, int* __restrict__ maxm, unsigned long long* __restrict__ segb,
+                             int* __restrict__ ntwo, int* __restrict__ n9, unsigned long long* __restrict__ keys) {
     // one block per batch
     const int b = blockIdx.x;
     if (b >= B) return;
-    int nl = 0, mm = 0;
+    int nl = 0, mm = 0, n2 = 0, nn9 = 0;
     unsigned long long sb = 0;
     for (int i = boff[b] + threadIdx.x; i < boff[b + 1]; i += blockDim.x) {
         const int id = order[i];
         const int a0 = off[id], m = off[id + 1] - a0;
         if (m > FGR_SMALL_NET) { nl++; mm = max(mm, m); }
+        if (m <= 2) n2++;   // the 2-node kernel also finishes trivial nets
+        if (m > FGR_MID_NET && m <= FGR_SMALL_NET) nn9++;
         for (int j = 1; j < m; j++) {
             const int u = a0 + par[a0 + j];
             sb += (unsigned)((abs(x[a0 + j] - x[u]) >> 5) + (abs(y[a0 + j] - y[u]) >> 5) + 4);
         }
+        // exec order inside the batch: larger nets first (same key layout as fgr_plan)
+        const unsigned inv = 2047u - (unsigned)min(m, 2047);
+        keys[i] = ((unsigned long long)b << 42) | ((unsigned long long)inv << 31) | (unsigned)id;
     }
     atomicAdd(&nlarge[b], nl);
     atomicMax(&maxm[b], mm);
     atomicAdd(&segb[b], sb);
+    atomicAdd(&ntwo[b], n2);
+    atomicAdd(&n9[b], nn9);
+}
+
+__global__ void k_large_list(int n, const int32_t* __restrict__ exec, const int32_t* __restrict__ off,
+                             int32_t* __restrict__ out, int* __restrict__ cnt) {
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    const int id = exec[i];
+    if (off[id + 1] - off[id] > FGR_SMALL_NET) out[atomicAdd(cnt, 1)] = id;
+}
+
+__global__ void k_keys_to_ids(int n, const unsigned long long* __restrict__ keys, int32_t* __restrict__ ids) {
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i < n) ids[i] = (int32_t)(keys[i] & 0x7FFFFFFFu);
 }
 
 __global__ void k_scatter_records(int n, const int32_t* __restrict__ order, const int32_t* __restrict__ off,
@@ -109,19 +141,21 @@ extern "C" FGR_API fgr_status fgr_route_batch(fgr_grid* g, const fgr_nets* nets,
     cudaStream_t st = (cudaStream_t)stream;
     FGR_CHECK_CUDA(g, cudaSetDevice(g->device));
     cudaError_t e;
-    int32_t* list = (int32_t*)fgr_scratch(g->s_rec[0], sizeof(int32_t) * (size_t)count + 64, &e);
+    int32_t* list = (int32_t*)fgr_scratch(g->s_rec[0], sizeof(int32_t) * (size_t)count * 5 + 64, &e);
     if (e != cudaSuccess) return fgr_cuda_fail(g, e, "route_batch scratch");
-    int* ctr = (int*)(list + count);
-    FGR_CHECK_CUDA(g, cudaMemsetAsync(ctr, 0, 4 * sizeof(int), st));
-    k_classify<<<(count + 255) / 256, 256, 0, st>>>(count, net_ids, nets->node_offset, list, ctr);
+    int32_t* tmp = list + count;
+    int* ctr = (int*)(list + 5 * (size_t)count);
+    FGR_CHECK_CUDA(g, cudaMemsetAsync(ctr, 0, 8 * sizeof(int), st));
+    k_classify<<<(count + 255) / 256, 256, 0, st>>>(count, net_ids, nets->node_offset, tmp, ctr);
+    k_concat4<<<(count + 255) / 256, 256, 0, st>>>(count, tmp, ctr, list);
     FGR_CHECK_CUDA(g, cudaGetLastError());
-    int hc[4];
+    int hc[8];
     FGR_CHECK_CUDA(g, cudaMemcpyAsync(hc, ctr, sizeof(hc), cudaMemcpyDeviceToHost, st));
     FGR_CHECK_CUDA(g, cudaStreamSynchronize(st));
     FGR_CHECK_CUDA(g, refresh_before_dp(g, st, g->total_segs));
     const NetsView nv = fgr_nets_view(nets);
-    FGR_CHECK_CUDA(g, fgr_launch_dp(g, st, nv, list, count, hc[0], hc[2], seg_out, net_cost, nullptr, nullptr,
-                                    nullptr, 0, true));
+    FGR_CHECK_CUDA(g, fgr_launch_dp(g, st, nv, list, hc[0], hc[1], hc[2], hc[3], hc[4], seg_out, net_cost, nullptr,
+                                    nullptr, nullptr, 0, true, nullptr));
     return FGR_OK;
 }
 
@@ -133,37 +167,89 @@ static fgr_status batch_info(fgr_grid* g, const fgr_nets* nets, const int32_t* o
         nets_equal(c.nets, *nets))
         return FGR_OK;
     cudaError_t e;
-    void* p = fgr_scratch(g->s_rec[1], (size_t)B * 16 + 64, &e);
+    const int R = 0;   // net count of the batches is read back below
+    (void)R;
+    void* p = fgr_scratch(g->s_rec[1], (size_t)B * 24 + 64, &e);
     if (e != cudaSuccess) return fgr_cuda_fail(g, e, "batch info scratch");
     unsigned long long* d_segb = (unsigned long long*)p;
     int* d_nl = (int*)(d_segb + B);
     int* d_mm = d_nl + B;
-    FGR_CHECK_CUDA(g, cudaMemsetAsync(p, 0, (size_t)B * 16, st));
-    if (B > 0) {
-        k_batch_info<<<B, 256, 0, st>>>(B, batch_offset, order, nets->node_offset, nets->x, nets->y, nets->parent,
-                                        d_nl, d_mm, d_segb);
-        FGR_CHECK_CUDA(g, cudaGetLastError());
-    }
+    int* d_n2 = d_mm + B;
+    int* d_n9 = d_n2 + B;
+    FGR_CHECK_CUDA(g, cudaMemsetAsync(p, 0, (size_t)B * 24, st));
     if (c.cap < B + 1) {
-        free(c.h_off); free(c.h_nlarge); free(c.h_maxm); free(c.h_segb);
+        free(c.h_off); free(c.h_nlarge); free(c.h_maxm); free(c.h_segb); free(c.h_ntwo); free(c.h_n9);
         c.cap = B + 1;
+        c.h_n9 = (int*)malloc(sizeof(int) * c.cap);
         c.h_off = (int*)malloc(sizeof(int) * c.cap);
         c.h_nlarge = (int*)malloc(sizeof(int) * c.cap);
         c.h_maxm = (int*)malloc(sizeof(int) * c.cap);
         c.h_segb = (long long*)malloc(sizeof(long long) * c.cap);
+        c.h_ntwo = (int*)malloc(sizeof(int) * c.cap);
     }
     FGR_CHECK_CUDA(g, cudaMemcpyAsync(c.h_off, batch_offset, sizeof(int) * (B + 1), cudaMemcpyDeviceToHost, st));
+    FGR_CHECK_CUDA(g, cudaStreamSynchronize(st));
+    const int nb = B > 0 ? c.h_off[B] : 0;
+    // the exec order is re-sorted inside each batch (larger nets first): any order the caller gives is fine
+    unsigned long long* keys = (unsigned long long*)fgr_scratch(g->s_plan[0], 16 * ((size_t)nb + 1), &e);
+    if (e != cudaSuccess) return fgr_cuda_fail(g, e, "exec keys");
+    unsigned long long* keys_s = keys + nb;
+    int32_t* exec = (int32_t*)fgr_scratch(g->s_plan[13], 4 * ((size_t)nb + 1), &e);
+    if (e != cudaSuccess) return fgr_cuda_fail(g, e, "exec order");
     if (B > 0) {
+        k_batch_info<<<B, 256, 0, st>>>(B, batch_offset, order, nets->node_offset, nets->x, nets->y, nets->parent,
+                                        d_nl, d_mm, d_segb, d_n2, d_n9, keys);
+        FGR_CHECK_CUDA(g, cudaGetLastError());
+        int bits = 42;
+        while ((1LL << (bits - 42)) <= B) bits++;
+        size_t tb = 0;
+        cub::DeviceRadixSort::SortKeys(nullptr, tb, keys, keys_s, nb, 0, bits, st);
+        void* tmp = fgr_scratch(g->s_plan[8], tb, &e);
+        if (e != cudaSuccess) return fgr_cuda_fail(g, e, "exec sort scratch");
+        FGR_CHECK_CUDA(g, cub::DeviceRadixSort::SortKeys(tmp, tb, keys, keys_s, nb, 0, bits, st));
+        k_keys_to_ids<<<(nb + 255) / 256, 256, 0, st>>>(nb, keys_s, exec);
+        FGR_CHECK_CUDA(g, cudaGetLastError());
         FGR_CHECK_CUDA(g, cudaMemcpyAsync(c.h_nlarge, d_nl, sizeof(int) * B, cudaMemcpyDeviceToHost, st));
         FGR_CHECK_CUDA(g, cudaMemcpyAsync(c.h_maxm, d_mm, sizeof(int) * B, cudaMemcpyDeviceToHost, st));
         FGR_CHECK_CUDA(g, cudaMemcpyAsync(c.h_segb, d_segb, sizeof(long long) * B, cudaMemcpyDeviceToHost, st));
+        FGR_CHECK_CUDA(g, cudaMemcpyAsync(c.h_ntwo, d_n2, sizeof(int) * B, cudaMemcpyDeviceToHost, st));
+        FGR_CHECK_CUDA(g, cudaMemcpyAsync(c.h_n9, d_n9, sizeof(int) * B, cudaMemcpyDeviceToHost, st));
     }
     FGR_CHECK_CUDA(g, cudaStreamSynchronize(st));
     c.valid = true;
+    c.prep_valid = false;
+    c.exec = exec;
     c.nets = *nets;
     c.order = order;
     c.batch_offset = batch_offset;
     c.num_batches = B;
+    return FGR_OK;
+}
+
+// Large-net tree analysis once per stage (k_large_prep), reused by every batch's k_dp_large.
+static fgr_status ensure_prep(fgr_grid* g, const fgr_nets* nets, int B, cudaStream_t st) {
+    PlanCache& c = g->cache;
+    if (c.prep_valid) return FGR_OK;
+    const int R = B > 0 ? c.h_off[B] : 0;
+    int maxm = 0, nl = 0;
+    for (int b = 0; b < B; b++) { maxm = c.h_maxm[b] > maxm ? c.h_maxm[b] : maxm; nl += c.h_nlarge[b]; }
+    if (nl == 0) { c.prep = Prep{nullptr, nullptr, nullptr, nullptr, nullptr, nullptr}; c.prep_valid = true; return FGR_OK; }
+    const size_t M = (size_t)nets->num_nodes, N = (size_t)nets->num_nets;
+    cudaError_t e;
+    char* p = (char*)fgr_scratch(g->s_prep, 5 * 2 * M + 4 * N + 4 * (size_t)nl + 64 + 5 * 16, &e);
+    if (e != cudaSuccess) return fgr_cuda_fail(g, e, "prep arrays");
+    auto take16 = [&](size_t n) { uint16_t* q = (uint16_t*)p; p += (2 * n + 15) & ~(size_t)15; return q; };
+    uint16_t* cs = take16(M); uint16_t* cl = take16(M); uint16_t* hv = take16(M); uint16_t* bot = take16(M);
+    uint16_t* pq = take16(M);
+    int32_t* np = (int32_t*)p; p += (4 * N + 15) & ~(size_t)15;
+    int32_t* list = (int32_t*)p; p += 4 * (size_t)nl;
+    int* cnt = (int*)p;
+    FGR_CHECK_CUDA(g, cudaMemsetAsync(cnt, 0, sizeof(int), st));
+    k_large_list<<<(R + 255) / 256, 256, 0, st>>>(R, c.exec, nets->node_offset, list, cnt);
+    FGR_CHECK_CUDA(g, cudaGetLastError());
+    FGR_CHECK_CUDA(g, fgr_launch_large_prep(g, st, fgr_nets_view(nets), list, nl, maxm, cs, cl, hv, bot, pq, np));
+    c.prep = Prep{cs, cl, hv, bot, pq, np};
+    c.prep_valid = true;
     return FGR_OK;
 }
 
@@ -180,6 +266,8 @@ extern "C" FGR_API fgr_status fgr_route_all(fgr_grid* g, const fgr_nets* nets, c
     FGR_CHECK_CUDA(g, cudaSetDevice(g->device));
     fgr_status s = batch_info(g, nets, order, batch_offset, B, st);
     if (s != FGR_OK) return s;
+    s = ensure_prep(g, nets, B, st);
+    if (s != FGR_OK) return s;
     const PlanCache& c = g->cache;
     if (M > 0) FGR_CHECK_CUDA(g, cudaMemsetAsync(seg_out, 0xFF, sizeof(uint32_t) * (size_t)M, st));
     if (N > 0) FGR_CHECK_CUDA(g, cudaMemsetAsync(net_cost, 0, sizeof(uint32_t) * (size_t)N, st));
@@ -194,9 +282,9 @@ extern "C" FGR_API fgr_status fgr_route_all(fgr_grid* g, const fgr_nets* nets, c
         for (int b = 0; b < B; b++) {
             const long long bound = b > 0 ? c.h_segb[b - 1] : (long long)g->total_segs;
             FGR_CHECK_CUDA(g, refresh_before_dp(g, st, bound));
-            const int o0 = c.h_off[b], cnt = c.h_off[b + 1] - o0;
-            FGR_CHECK_CUDA(g, fgr_launch_dp(g, st, nv, order + o0, cnt, c.h_nlarge[b], c.h_maxm[b], seg_out,
-                                            net_cost, nullptr, nullptr, nullptr, 0, true));
+            const int o0 = c.h_off[b], cnt = c.h_off[b + 1] - o0, nl = c.h_nlarge[b], n2 = c.h_ntwo[b], n9 = c.h_n9[b];
+            FGR_CHECK_CUDA(g, fgr_launch_dp(g, st, nv, c.exec + o0, nl, n9, cnt - nl - n9 - n2, n2, c.h_maxm[b],
+                                            seg_out, net_cost, nullptr, nullptr, nullptr, 0, true, &c.prep));
                 }
         return FGR_OK;
     }
@@ -207,7 +295,7 @@ extern "C" FGR_API fgr_status fgr_route_all(fgr_grid* g, const fgr_nets* nets, c
     if (e != cudaSuccess) return fgr_cuda_fail(g, e, "record offsets");
     int32_t* sizes = rec_off + R + 1;
     if (R > 0) {
-        k_net_sizes<<<(R + 255) / 256, 256, 0, st>>>(R, order, nets->node_offset, sizes);
+        k_net_sizes<<<(R + 255) / 256, 256, 0, st>>>(R, c.exec, nets->node_offset, sizes);
         FGR_CHECK_CUDA(g, cudaGetLastError());
     }
     FGR_CHECK_CUDA(g, cudaMemsetAsync(sizes + R, 0, sizeof(int32_t), st));
@@ -230,15 +318,21 @@ extern "C" FGR_API fgr_status fgr_route_all(fgr_grid* g, const fgr_nets* nets, c
         const long long bound = b > 0 ? c.h_segb[b - 1] : (long long)g->total_segs;
         cudaError_t ce = refresh_before_dp(g, st, bound);
         if (ce != cudaSuccess) { rs = fgr_cuda_fail(g, ce, "refresh"); break; }
-        const int o0 = c.h_off[b], cnt = c.h_off[b + 1] - o0, nl = c.h_nlarge[b];
+        const int o0 = c.h_off[b], cnt = c.h_off[b + 1] - o0, nl = c.h_nlarge[b], n2 = c.h_ntwo[b], n9 = c.h_n9[b];
         int32_t sp[4];
         fgr_split_batch(cnt, nl, g->rank, g->world, sp);
         if (sp[1] > sp[0])
-            ce = fgr_launch_dp(g, st, nv, order + o0 + sp[0], sp[1] - sp[0], sp[1] - sp[0], c.h_maxm[b], nullptr,
-                               nullptr, rec, rec_off, rec_cost, o0 + sp[0], false);
-        if (ce == cudaSuccess && sp[3] > sp[2])
-            ce = fgr_launch_dp(g, st, nv, order + o0 + sp[2], sp[3] - sp[2], 0, 0, nullptr, nullptr, rec, rec_off,
-                               rec_cost, o0 + sp[2], false);
+            ce = fgr_launch_dp(g, st, nv, c.exec + o0 + sp[0], sp[1] - sp[0], 0, 0, 0, c.h_maxm[b], nullptr, nullptr,
+                               rec, rec_off, rec_cost, o0 + sp[0], false, &c.prep);
+        if (ce == cudaSuccess && sp[3] > sp[2]) {
+            // the rank's small chunk [sp2, sp3) crosses the class boundaries nl+n9 and cnt-n2
+            const int b1 = nl + n9, b2 = cnt - n2;
+            const int cL = max(0, min(sp[3], b1) - sp[2]);
+            const int cS = max(0, min(sp[3], b2) - max(sp[2], b1));
+            const int cT = sp[3] - sp[2] - cL - cS;
+            ce = fgr_launch_dp(g, st, nv, c.exec + o0 + sp[2], 0, cL, cS, cT, 0, nullptr, nullptr, rec, rec_off,
+                               rec_cost, o0 + sp[2], false, &c.prep);
+        }
         if (ce != cudaSuccess) { rs = fgr_cuda_fail(g, ce, "dp"); break; }
         const int ps = fgr_prof_begin(g, PROF_EXCHANGE, st);
         ncclResult_t nr = ncclGroupStart();
@@ -254,13 +348,13 @@ extern "C" FGR_API fgr_status fgr_route_all(fgr_grid* g, const fgr_nets* nets, c
             rs = fgr_set_error(FGR_ERR_NCCL, "NCCL all-reduce failed: %s", ncclGetErrorString(nr != ncclSuccess ? nr : ne));
             break;
         }
-        ce = fgr_launch_commit(g, st, nv, order + o0, cnt, rec, rec_off, o0);
+        ce = fgr_launch_commit(g, st, nv, c.exec + o0, cnt, rec, rec_off, o0);
         if (ce != cudaSuccess) { rs = fgr_cuda_fail(g, ce, "commit"); break; }
         }
     free(h_roff);
     if (rs != FGR_OK) return rs;
     if (R > 0) {
-        k_scatter_records<<<(unsigned)(((size_t)R * 32 + 255) / 256), 256, 0, st>>>(R, order, nets->node_offset,
+        k_scatter_records<<<(unsigned)(((size_t)R * 32 + 255) / 256), 256, 0, st>>>(R, c.exec, nets->node_offset,
                                                                                      rec_off, rec, rec_cost, seg_out,
                                                                                      net_cost);
         FGR_CHECK_CUDA(g, cudaGetLastError());
