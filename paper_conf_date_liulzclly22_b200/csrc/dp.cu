@@ -58,6 +58,9 @@ struct Tabs {
     uint16_t* top;    // CTA path: top node of the heavy path holding v
     uint16_t* bot;    // CTA path: bottom (leaf) of the path topped by v
     uint16_t* pq;     // CTA path: path tops, deepest top first
+    uint16_t* rpos;   // CTA path: index along the root path from its bottom (0xFFFF off the root path)
+    uint16_t* rp;     // CTA path: root path nodes, bottom first
+    uint16_t* argq;   // CTA path: root-path items whose recB/recE a helper fills in
     uint8_t* done;    // CTA path: E_v final (values pass)
     uint8_t* sready;  // CTA path: span_v final (backtrack)
     int8_t* plo;
@@ -79,7 +82,7 @@ __host__ __device__ inline size_t tabs_bytes(int m, int L, int nH, int nV, bool 
     b += a16((size_t)m * 2 * nV * 4);
     if (!cta) b += a16((size_t)m * 4);
     b += 4 * a16((size_t)m * 2);
-    if (cta) b += 2 * a16((size_t)(m + 1) * 2) + 6 * a16((size_t)m * 2) + 2 * a16((size_t)m);
+    if (cta) b += 2 * a16((size_t)(m + 1) * 2) + 9 * a16((size_t)m * 2) + 2 * a16((size_t)m);
     b += 3 * a16((size_t)m);
     b += 2 * a16((size_t)m * L);
     return b;
@@ -98,7 +101,7 @@ __device__ inline Tabs carve_tabs(unsigned char* p, int m, int L, int nH, int nV
     t.y = (int16_t*)p; p += a16((size_t)m * 2);
     t.par = (int16_t*)p; p += a16((size_t)m * 2);
     t.depth = (uint16_t*)p; p += a16((size_t)m * 2);
-    t.cstart = t.clist = t.anc = t.lvstart = t.hv = t.top = t.bot = t.pq = nullptr;
+    t.cstart = t.clist = t.anc = t.lvstart = t.hv = t.top = t.bot = t.pq = t.rpos = t.rp = t.argq = nullptr;
     t.done = t.sready = nullptr;
     if (cta) {
         t.cstart = (uint16_t*)p; p += a16((size_t)(m + 1) * 2);
@@ -109,6 +112,9 @@ __device__ inline Tabs carve_tabs(unsigned char* p, int m, int L, int nH, int nV
         t.top = (uint16_t*)p; p += a16((size_t)m * 2);
         t.bot = (uint16_t*)p; p += a16((size_t)m * 2);
         t.pq = (uint16_t*)p; p += a16((size_t)m * 2);
+        t.rpos = (uint16_t*)p; p += a16((size_t)m * 2);
+        t.rp = (uint16_t*)p; p += a16((size_t)m * 2);
+        t.argq = (uint16_t*)p; p += a16((size_t)m * 2);
         t.done = (uint8_t*)p; p += a16((size_t)m);
         t.sready = (uint8_t*)p; p += a16((size_t)m);
     }
@@ -801,6 +807,9 @@ __device__ __forceinline__ void large_prologue(const Tabs& t, const NetsView& nv
     }
     for (int v = tid; v < m; v += T)
         if (t.hv[v] == 0xFFFF) t.bot[t.top[v]] = (uint16_t)v;
+    __syncthreads();
+    for (int v = tid; v < m; v += T)
+        t.rpos[v] = t.top[v] == 0 ? (uint16_t)(t.depth[t.bot[0]] - t.depth[v]) : (uint16_t)0xFFFF;
     // path tops, deepest first (a light child's top is deeper than its parent's path top)
     if (warp == 0) {
         int n = 0;
@@ -816,13 +825,200 @@ __device__ __forceinline__ void large_prologue(const Tabs& t, const NetsView& nv
     }
 }
 
+__device__ __forceinline__ int ld_flag(const uint8_t* f) { return *(volatile const uint8_t*)f; }
+
+constexpr int kMR = 16;   // matrix ring slots (root-path transfer matrices in flight)
+template <int LT> struct MStride { static constexpr int v = (LT + 3) & ~3; };
+
+// Wait for v's light children (all children but the heavy one), then build the packed
+// dominance table G_v of K_v in the warp's scratch w.R (lane = lo rows, then lane = b columns).
+template <int LT>
+__device__ __forceinline__ void build_G(const LaneConst<LT>& c, const Tabs& t, const WScr& w, int v, int gl,
+                                        unsigned gmask) {
+    const int hvv = t.hv[v];
+    const int k0 = t.cstart[v], k1 = t.cstart[v + 1];
+    for (int k = k0 + gl; k < k1; k += LT) {
+        const int ch = t.clist[k];
+        if (ch != hvv) {
+            int spins = 0;
+            while (ld_flag(&t.done[ch]) == 0)
+                if (++spins > 64) __nanosleep(20);   // short busy phase first: this may be the critical walker
+        }
+    }
+    __syncwarp(gmask);
+    __threadfence_block();
+    const int lo = gl;
+    uint32_t acc[LT];
+#pragma unroll
+    for (int hi = 0; hi < LT; hi++) acc[hi] = hi >= lo ? c.vme[hi] : FGR_INF;
+    for (int k = k0; k < k1; k++) {
+        const int ch = t.clist[k];
+        if (ch == hvv) continue;
+        const uint32_t* Ec = t.E + (size_t)ch * LT;
+        uint32_t run = FGR_INF;
+#pragma unroll
+        for (int hi = 0; hi < LT; hi++) {
+            const uint32_t e = Ec[hi];
+            if (hi >= lo) { run = min(run, e); acc[hi] = sat_add(acc[hi], run); }
+        }
+    }
+    unsigned long long run = ~0ull;
+#pragma unroll
+    for (int hi = LT - 1; hi >= 0; hi--)
+        if (hi >= lo) {
+            const unsigned long long key = ((unsigned long long)acc[hi] << 8) | (unsigned)(lo << 4) | (unsigned)hi;
+            run = key < run ? key : run;
+            w.R[lo * LT + hi] = run;
+        }
+    __syncwarp(gmask);
+    const int bcol = gl;
+    unsigned long long pr = ~0ull;
+#pragma unroll
+    for (int a = 0; a < LT; a++)
+        if (a <= bcol) {
+            const unsigned long long x = w.R[a * LT + bcol];
+            pr = x < pr ? x : pr;
+            w.R[a * LT + bcol] = pr;
+        }
+    __syncwarp(gmask);
+}
+
+// One non-root node of a path walk in product form (G_v already built when light):
+// B_v / recB_v from E_h (lanes of Eprev), then E_v / recE_v.  Returns this lane's E_v.
+template <int LT>
+__device__ __forceinline__ uint32_t path_node(const LaneConst<LT>& c, const Tabs& t, const WScr& w, int v, uint32_t Eprev,
+                                              bool has_prev, bool light, int gl, int gbase, unsigned gmask, int nH,
+                                              int nV, uint32_t opp, bool store_E) {
+    const int plo = t.plo[v], phi = t.phi[v];
+    const int ls = gl;
+    int a0 = ls, b0 = ls;
+    if (plo >= 0) { a0 = min(a0, plo); b0 = max(b0, phi); }
+    unsigned long long bk;
+    if (light) {
+        if (!has_prev) bk = w.R[a0 * LT + b0];
+        else {
+            unsigned long long gk[LT];
+#pragma unroll
+            for (int l = 0; l < LT; l++) gk[l] = w.R[min(a0, l) * LT + max(b0, l)];
+#pragma unroll
+            for (int l = 0; l < LT; l++) {
+                const uint32_t e = __shfl_sync(gmask, Eprev, gbase + l);
+                gk[l] = ((unsigned long long)sat_add(e, (uint32_t)(gk[l] >> 8)) << 8) | (gk[l] & 0xFFull);
+            }
+            bk = tree_min<LT>(gk);
+        }
+    } else {
+        uint32_t va0 = 0, vb0 = 0, za0 = 0;
+#pragma unroll
+        for (int l = 0; l < LT; l++) {
+            va0 = (l == a0) ? c.vp[l] : va0;
+            vb0 = (l == b0) ? c.vp[l] : vb0;
+            za0 = (l == a0) ? c.zl[l] : za0;
+        }
+        if (!has_prev) bk = ((unsigned long long)(vb0 - va0) << 8) | (za0 << 4) | (unsigned)b0;
+        else {
+            unsigned long long kk[LT];
+#pragma unroll
+            for (int l = 0; l < LT; l++) {
+                const uint32_t e = __shfl_sync(gmask, Eprev, gbase + l);
+                const bool la = l < a0, lb = l > b0;
+                const uint32_t va = la ? c.vp[l] : va0, vb = lb ? c.vp[l] : vb0;
+                const uint32_t za = la ? c.zl[l] : za0;
+                const uint32_t bb = lb ? (uint32_t)l : (uint32_t)b0;
+                kk[l] = ((unsigned long long)sat_add(e, vb - va) << 8) | (za << 4) | bb;
+            }
+            bk = tree_min<LT>(kk);
+        }
+    }
+    const uint32_t Bv = (uint32_t)(bk >> 8);
+    t.recB[(size_t)v * LT + ls] = (uint8_t)(bk & 0xFF);
+    const int lt = gl;
+    const int u = t.par[v];
+    const int xv = t.x[v], yv = t.y[v], xu = t.x[u], yu = t.y[u];
+    uint32_t best = FGR_INF;
+    int bls = lt;
+    uint32_t Bl[LT];
+#pragma unroll
+    for (int l = 0; l < LT; l++) Bl[l] = __shfl_sync(gmask, Bv, gbase + l);
+    if (yv == yu || xv == xu) {
+        const int de = (yv == yu) ? 0 : 1;
+        if (c.my_dir == de) {
+            const uint32_t leg = de == 0 ? t.legH[(size_t)v * 2 * nH + c.my_slot] : t.legV[(size_t)v * 2 * nV + c.my_slot];
+            best = sat_add(Bv, leg);
+        }
+    } else {
+        const bool b0v = c.my_dir == 1;
+        const uint32_t leg2 = b0v ? t.legV[((size_t)v * 2 + 1) * nV + c.my_slot] : t.legH[((size_t)v * 2 + 1) * nH + c.my_slot];
+        const uint32_t* l1 = b0v ? t.legH + (size_t)v * 2 * nH : t.legV + (size_t)v * 2 * nV;
+        int sidx = 0;
+#pragma unroll
+        for (int l = 0; l < LT; l++)
+            if ((opp >> l) & 1u) {
+                const uint32_t cst = sat_add(sat_add(sat_add(Bl[l], l1[sidx]), c.vme[l]), leg2);
+                if (cst < best) { best = cst; bls = l; }
+                sidx++;
+            }
+    }
+    if (store_E) t.E[(size_t)v * LT + lt] = best;
+    t.recE[(size_t)v * LT + lt] = (uint8_t)bls;
+    return best;
+}
+
+// Transfer matrix of node v (values only): E_v(lt) = min_l [E_h(l) + M_v(l, lt)],
+// M_v(l, lt) = min_ls [C_v(l, ls) + W_v(ls, lt)], C_v(l, ls) = value of G_v(hull(l, ls, pins)).
+// Exact: min-plus distributes over the saturating sums.  Lane lt writes column lt.
+template <int LT>
+__device__ __forceinline__ void build_M(const Hdr* h, const LaneConst<LT>& c, const Tabs& t, const WScr& w, int v,
+                                        bool light, int gl, int nH, int nV, uint32_t opp, uint32_t* col) {
+    const int plo = t.plo[v], phi = t.phi[v];
+    const int lt = gl;
+    const int u = t.par[v];
+    const int xv = t.x[v], yv = t.y[v], xu = t.x[u], yu = t.y[u];
+    const bool straight = (yv == yu) || (xv == xu);
+    uint32_t legS = FGR_INF, leg2 = 0;
+    const uint32_t* l1 = nullptr;
+    if (straight) {
+        const int de = (yv == yu) ? 0 : 1;
+        if (c.my_dir == de) legS = de == 0 ? t.legH[(size_t)v * 2 * nH + c.my_slot] : t.legV[(size_t)v * 2 * nV + c.my_slot];
+    } else {
+        const bool b0v = c.my_dir == 1;
+        leg2 = b0v ? t.legV[((size_t)v * 2 + 1) * nV + c.my_slot] : t.legH[((size_t)v * 2 + 1) * nH + c.my_slot];
+        l1 = b0v ? t.legH + (size_t)v * 2 * nH : t.legV + (size_t)v * 2 * nV;
+    }
+    for (int l = 0; l < LT; l++) {
+        uint32_t best = FGR_INF;
+        if (straight) {
+            if (legS != FGR_INF) {
+                int a = lt, b = lt;
+                if (plo >= 0) { a = min(a, plo); b = max(b, phi); }
+                a = min(a, l); b = max(b, l);
+                const uint32_t cv = light ? (uint32_t)(w.R[a * LT + b] >> 8) : h->viapre[b] - h->viapre[a];
+                best = sat_add(cv, legS);
+            }
+        } else {
+            int sidx = 0;
+#pragma unroll
+            for (int ls = 0; ls < LT; ls++)
+                if ((opp >> ls) & 1u) {
+                    int a = ls, b = ls;
+                    if (plo >= 0) { a = min(a, plo); b = max(b, phi); }
+                    a = min(a, l); b = max(b, l);
+                    const uint32_t cv = light ? (uint32_t)(w.R[a * LT + b] >> 8) : h->viapre[b] - h->viapre[a];
+                    const uint32_t cst = sat_add(sat_add(sat_add(cv, l1[sidx]), c.vme[ls]), leg2);
+                    best = min(best, cst);
+                    sidx++;
+                }
+        }
+        col[lt * MStride<LT>::v + l] = best;
+    }
+}
+
 #ifdef FGR_TIMING
 #define TMARK(i) do { if (threadIdx.x == 0) tm[i] = clock64(); } while (0)
 #else
 #define TMARK(i) do { } while (0)
 #endif
 
-__device__ __forceinline__ int ld_flag(const uint8_t* f) { return *(volatile const uint8_t*)f; }
 
 
 template <int LT>
@@ -859,7 +1055,7 @@ __global__ void __launch_bounds__(32 * kLargeWarps, 1) k_dp_large(GridView g, Ne
             t.x[i] = nv.x[a0 + i]; t.y[i] = nv.y[a0 + i]; t.par[i] = (int16_t)nv.par[a0 + i];
             t.plo[i] = nv.plo[a0 + i]; t.phi[i] = nv.phi[a0 + i];
             t.cstart[i] = prep.cs[a0 + i]; t.clist[i] = prep.cl[a0 + i]; t.hv[i] = prep.hv[a0 + i];
-            t.bot[i] = prep.bot[a0 + i]; t.pq[i] = prep.pq[a0 + i];
+            t.bot[i] = prep.bot[a0 + i]; t.pq[i] = prep.pq[a0 + i]; t.rpos[i] = prep.rpos[a0 + i];
             t.done[i] = 0; t.sready[i] = 0;
         }
         if (tid == 0) { t.cstart[m] = (uint16_t)(m - 1); s_npaths = prep.npaths[net]; }
@@ -877,215 +1073,193 @@ __global__ void __launch_bounds__(32 * kLargeWarps, 1) k_dp_large(GridView g, Ne
     TMARK(2);
     const int npaths = s_npaths;
     // ---------------- values: bottom-up path walks
-#ifdef FGR_TIMING
-    long long vw_wait = 0, vw_nodes = 0, vw_paths = 0, vw_light = 0, vw_t0 = clock64();
-    long long f_rows = 0, f_pref = 0, f_B = 0, f_E = 0, f_fin = 0, f_x;
-#endif
+    // warp 0 walks the root path; the other warps walk the remaining paths (deepest tops
+    // first), then precompute root-path transfer matrices ahead of warp 0 and fill in the
+    // recB/recE of the nodes warp 0 passed with a matrix step.
+    __shared__ int s_K, s_mnext, s_anext, s_acount, s_wdone;
+    __shared__ int sstate[kMR];   // slot state: generation * 4 + {0 free, 1 writing, 2 ready}
+    uint32_t* mslots = reinterpret_cast<uint32_t*>(base + (size_t)kLargeWarps * G * wscr_bytes(LT) +
+                                                   tabs_bytes(m, LT, nH, nV, true));
+    for (int v = tid; v < m; v += T)
+        if (t.rpos[v] != 0xFFFF) t.rp[t.rpos[v]] = (uint16_t)v;
+    if (tid == 0) { s_K = t.rpos[0] + 1; s_mnext = 1; s_anext = 0; s_acount = 0; s_wdone = 0; }
+    if (tid < kMR) sstate[tid] = (tid == 0 ? kMR : tid) * 4;
+    __syncthreads();
+    const int K = s_K;
     if (glane) {
         const uint32_t opp = c.my_dir == 1 ? c.hmask : (~c.hmask & ((1u << LT) - 1u));   // bend partner layers
-        bool first = (warp == 0);   // warp 0 starts on the root path right away
-        for (;;) {
-            int tp;
-            if (first) {
-                tp = 0;
-                first = false;
-            } else {
-                int p = 0;
-                if (gl == 0) p = atomicAdd(&s_ticket, 1);
-                p = __shfl_sync(gmask, p, gbase);
-                if (p >= npaths - 1) break;   // pq[npaths-1] is the root path
-                tp = t.pq[p];
-            }
-            int v = t.bot[tp];
-#ifdef FGR_TIMING
-            vw_paths++;
-#endif
+        if (warp == 0) {
+            // ---- root-path walker
             uint32_t Eprev = FGR_INF;
-            bool has_prev = false;
-            for (;;) {
-                const int hvv = t.hv[v];
-                const int k0 = t.cstart[v], k1 = t.cstart[v + 1];
-                const bool light = (k1 - k0) > 1;
 #ifdef FGR_TIMING
-                vw_nodes++;
+            long long w_slot = 0, w_inline = 0, w_fast = 0, w_x;
 #endif
-                if (light) {
-#ifdef FGR_TIMING
-                    long long q0 = clock64();
-                    vw_light++;
-#endif
-                    for (int k = k0 + gl; k < k1; k += LT) {
-                        const int ch = t.clist[k];
-                        if (ch != hvv) while (ld_flag(&t.done[ch]) == 0) __nanosleep(40);
-                    }
-                    __syncwarp(gmask);
-#ifdef FGR_TIMING
-                    vw_wait += clock64() - q0;
-                    f_x = clock64();
-#endif
-                    __threadfence_block();
-                    // K rows (light children only) -> suffix minima R(lo, b) -> column prefix G(a, b), in w.R
-                    const int lo = gl;
-                    uint32_t acc[LT];
-#pragma unroll
-                    for (int hi = 0; hi < LT; hi++) acc[hi] = hi >= lo ? c.vme[hi] : FGR_INF;
-                    for (int k = k0; k < k1; k++) {
-                        const int ch = t.clist[k];
-                        if (ch == hvv) continue;
-                        const uint32_t* Ec = t.E + (size_t)ch * LT;
-                        uint32_t run = FGR_INF;
-#pragma unroll
-                        for (int hi = 0; hi < LT; hi++) {
-                            const uint32_t e = Ec[hi];
-                            if (hi >= lo) { run = min(run, e); acc[hi] = sat_add(acc[hi], run); }
-                        }
-                    }
-                    unsigned long long run = ~0ull;
-#pragma unroll
-                    for (int hi = LT - 1; hi >= 0; hi--)
-                        if (hi >= lo) {
-                            const unsigned long long key = ((unsigned long long)acc[hi] << 8) | (unsigned)(lo << 4) | (unsigned)hi;
-                            run = key < run ? key : run;
-                            w.R[lo * LT + hi] = run;
-                        }
-                    __syncwarp(gmask);
-#ifdef FGR_TIMING
-                    f_rows += clock64() - f_x; f_x = clock64();
-#endif
-                    const int bcol = gl;
-                    unsigned long long pr = ~0ull;
-#pragma unroll
-                    for (int a = 0; a < LT; a++)
-                        if (a <= bcol) {
-                            const unsigned long long x = w.R[a * LT + bcol];
-                            pr = x < pr ? x : pr;
-                            w.R[a * LT + bcol] = pr;
-                        }
-                    __syncwarp(gmask);
-#ifdef FGR_TIMING
-                    f_pref += clock64() - f_x;
-#endif
-                }
-#ifdef FGR_TIMING
-                f_x = clock64();
-#endif
-                const int plo = t.plo[v], phi = t.phi[v];
+            for (int k = 0; k < K; k++) {
+                const int v = t.rp[k];
                 if (v == 0) {
                     // generalised Eq. (4): min over l of E_h(l) + G(hull({l} + pins)) (any span for a Steiner root)
+                    const bool light = (t.cstart[1] - t.cstart[0]) > 1;
+                    if (light) build_G<LT>(c, t, w, 0, gl, gmask);
+                    const int plo = t.plo[0], phi = t.phi[0];
                     const int ra = plo >= 0 ? plo : LT - 1, rb = plo >= 0 ? phi : 0;
-                    unsigned long long best = ~0ull;
+                    unsigned long long kk[LT];
 #pragma unroll
                     for (int l = 0; l < LT; l++) {
                         const uint32_t e = __shfl_sync(gmask, Eprev, gbase + l);
                         const int a = min(ra, l), b = max(rb, l);
                         const unsigned long long gk = light ? w.R[a * LT + b] : gclosed(h, a, b);
-                        const unsigned long long key = ((unsigned long long)sat_add(e, (uint32_t)(gk >> 8)) << 8) | (gk & 0xFFull);
-                        best = key < best ? key : best;
+                        kk[l] = ((unsigned long long)sat_add(e, (uint32_t)(gk >> 8)) << 8) | (gk & 0xFFull);
                     }
+                    const unsigned long long best = tree_min<LT>(kk);
                     if (gl == 0) { s_root = best; t.span[0] = (uint8_t)(best & 0xFF); }
                     __syncwarp(gmask);
                     __threadfence_block();
                     if (gl == 0) { t.done[0] = 1; *(volatile uint8_t*)&t.sready[0] = 1; }
                     break;
                 }
-                // Eq. (2) in product form, lane = ls
-                const int ls = gl;
-                int a0 = ls, b0 = ls;
-                if (plo >= 0) { a0 = min(a0, plo); b0 = max(b0, phi); }
-                unsigned long long bk = ~0ull;
-                if (light) {
-                    if (!has_prev) bk = w.R[a0 * LT + b0];
-                    else {
-                        unsigned long long gk[LT];
-#pragma unroll
-                        for (int l = 0; l < LT; l++) gk[l] = w.R[min(a0, l) * LT + max(b0, l)];
-#pragma unroll
-                        for (int l = 0; l < LT; l++) {
-                            const uint32_t e = __shfl_sync(gmask, Eprev, gbase + l);
-                            gk[l] = ((unsigned long long)sat_add(e, (uint32_t)(gk[l] >> 8)) << 8) | (gk[l] & 0xFFull);
+                bool fast = false;
+#ifdef FGR_TIMING
+                w_x = clock64();
+#endif
+                if (k > 0) {
+                    const int sl = k % kMR;
+                    for (;;) {
+                        const int st = *(volatile int*)&sstate[sl];
+                        if (st == k * 4 + 2) { fast = true; break; }
+                        if (st == k * 4) {
+                            int old = 0;
+                            if (gl == 0) old = atomicCAS(&sstate[sl], k * 4, (k + kMR) * 4);   // not ready: go inline
+                            old = __shfl_sync(gmask, old, gbase);
+                            if (old == k * 4) break;
+                            continue;
                         }
-                        bk = tree_min<LT>(gk);
+                        // a helper is writing this matrix: busy-wait (a sleeping walker oversleeps)
                     }
-                } else {
-                    // K = V: G(a, b) = (V(a, b), span (zlo[a], b)) in closed form, a = min(a0, l), b = max(b0, l)
-                    uint32_t va0 = 0, vb0 = 0, za0 = 0;
+#ifdef FGR_TIMING
+                    w_slot += clock64() - w_x; w_x = clock64();
+#endif
+                    if (fast) {
+                        __threadfence_block();
+                        const uint32_t* col = mslots + (size_t)sl * LT * MStride<LT>::v + gl * MStride<LT>::v;
+                        unsigned long long dummy;
+                        (void)dummy;
+                        uint32_t ev[LT];
 #pragma unroll
-                    for (int l = 0; l < LT; l++) {
-                        va0 = (l == a0) ? c.vp[l] : va0;
-                        vb0 = (l == b0) ? c.vp[l] : vb0;
-                        za0 = (l == a0) ? c.zl[l] : za0;
-                    }
-                    if (!has_prev) bk = ((unsigned long long)(vb0 - va0) << 8) | (za0 << 4) | (unsigned)b0;
-                    else {
-                        unsigned long long kk[LT];
+                        for (int l = 0; l < LT; l++) ev[l] = sat_add(__shfl_sync(gmask, Eprev, gbase + l), col[l]);
 #pragma unroll
-                        for (int l = 0; l < LT; l++) {
-                            const uint32_t e = __shfl_sync(gmask, Eprev, gbase + l);
-                            const bool la = l < a0, lb = l > b0;
-                            const uint32_t va = la ? c.vp[l] : va0, vb = lb ? c.vp[l] : vb0;
-                            const uint32_t za = la ? c.zl[l] : za0;
-                            const uint32_t bb = lb ? (uint32_t)l : (uint32_t)b0;
-                            kk[l] = ((unsigned long long)sat_add(e, vb - va) << 8) | (za << 4) | bb;
+                        for (int s2 = 1; s2 < LT; s2 <<= 1)
+#pragma unroll
+                            for (int i = 0; i + s2 < LT; i += 2 * s2) ev[i] = min(ev[i], ev[i + s2]);
+                        const uint32_t Ev = ev[0];
+                        t.E[(size_t)v * LT + gl] = Ev;
+                        __syncwarp(gmask);
+                        if (gl == 0) {
+                            *(volatile int*)&sstate[sl] = (k + kMR) * 4;   // slot free for item k + kMR
+                            t.argq[s_acount] = (uint16_t)k;
+                            __threadfence_block();
+                            *(volatile int*)&s_acount = s_acount + 1;
                         }
-                        bk = tree_min<LT>(kk);
+                        Eprev = Ev;
+#ifdef FGR_TIMING
+                        w_fast += clock64() - w_x;
+#endif
+                        continue;
                     }
                 }
-                const uint32_t Bv = (uint32_t)(bk >> 8);
-                t.recB[(size_t)v * LT + ls] = (uint8_t)(bk & 0xFF);
-#ifdef FGR_TIMING
-                f_B += clock64() - f_x; f_x = clock64();
-#endif
-                // Eqs. (1),(3),(5)-(7), lane = lt
-                const int lt = gl;
-                const int u = t.par[v];
-                const int xv = t.x[v], yv = t.y[v], xu = t.x[u], yu = t.y[u];
-                uint32_t best = FGR_INF;
-                int bls = lt;
-                uint32_t Bl[LT];
-#pragma unroll
-                for (int l = 0; l < LT; l++) Bl[l] = __shfl_sync(gmask, Bv, gbase + l);
-                if (yv == yu || xv == xu) {
-                    const int de = (yv == yu) ? 0 : 1;
-                    if (c.my_dir == de) {
-                        const uint32_t leg = de == 0 ? t.legH[(size_t)v * 2 * nH + c.my_slot] : t.legV[(size_t)v * 2 * nV + c.my_slot];
-                        best = sat_add(Bv, leg);
-                    }
-                } else {
-                    const bool b0v = c.my_dir == 1;
-                    const uint32_t leg2 = b0v ? t.legV[((size_t)v * 2 + 1) * nV + c.my_slot] : t.legH[((size_t)v * 2 + 1) * nH + c.my_slot];
-                    const uint32_t* l1 = b0v ? t.legH + (size_t)v * 2 * nH : t.legV + (size_t)v * 2 * nV;
-                    int sidx = 0;
-#pragma unroll
-                    for (int l = 0; l < LT; l++)
-                        if ((opp >> l) & 1u) {
-                            const uint32_t cst = sat_add(sat_add(sat_add(Bl[l], l1[sidx]), c.vme[l]), leg2);
-                            if (cst < best) { best = cst; bls = l; }
-                            sidx++;
-                        }
-                }
-                t.E[(size_t)v * LT + lt] = best;
-                t.recE[(size_t)v * LT + lt] = (uint8_t)bls;
-#ifdef FGR_TIMING
-                f_E += clock64() - f_x; f_x = clock64();
-#endif
+                const bool light = (t.cstart[v + 1] - t.cstart[v]) > 1;
+                if (light) build_G<LT>(c, t, w, v, gl, gmask);
+                Eprev = path_node<LT>(c, t, w, v, Eprev, k > 0, light, gl, gbase, gmask, nH, nV, opp, true);
                 __syncwarp(gmask);
                 __threadfence_block();
-                if (gl == 0) *(volatile uint8_t*)&t.done[v] = 1;
 #ifdef FGR_TIMING
-                f_fin += clock64() - f_x;
+                w_inline += clock64() - w_x;
 #endif
-                if (v == tp) break;
-                Eprev = best;
-                has_prev = true;
-                v = u;
+            }
+            if (gl == 0) *(volatile int*)&s_wdone = 1;
+#ifdef FGR_TIMING
+            if (gl == 0 && m > 880) printf("WALK m=%d K=%d fast=%d t=%lld slot=%lld inline=%lld fastc=%lld\n", m, K, s_acount,
+                                           clock64() - tm[2], w_slot, w_inline, w_fast);
+#endif
+        } else {
+            // ---- the other paths, deepest tops first (pq[npaths-1] is the root path)
+            for (;;) {
+                int p = 0;
+                if (gl == 0) p = atomicAdd(&s_ticket, 1);
+                p = __shfl_sync(gmask, p, gbase);
+                if (p >= npaths - 1) break;
+                const int tp = t.pq[p];
+                int v = t.bot[tp];
+                uint32_t Eprev = FGR_INF;
+                bool has_prev = false;
+                for (;;) {
+                    const bool light = (t.cstart[v + 1] - t.cstart[v]) > 1;
+                    if (light) build_G<LT>(c, t, w, v, gl, gmask);
+                    const uint32_t Ev = path_node<LT>(c, t, w, v, Eprev, has_prev, light, gl, gbase, gmask, nH, nV, opp, true);
+                    if (v == tp) {   // only path tops are read by other warps (as light children)
+                        __syncwarp(gmask);
+                        __threadfence_block();
+                        if (gl == 0) *(volatile uint8_t*)&t.done[v] = 1;
+                        break;
+                    }
+                    Eprev = Ev;
+                    has_prev = true;
+                    v = t.par[v];
+                }
+            }
+            // ---- root-path transfer matrices ahead of the walker
+            for (;;) {
+                int k = 0;
+                if (gl == 0) k = atomicAdd(&s_mnext, 1);
+                k = __shfl_sync(gmask, k, gbase);
+                if (k >= K - 1) break;
+                const int sl = k % kMR;
+                int st;
+                for (;;) {
+                    st = *(volatile int*)&sstate[sl];
+                    if ((st >> 2) >= k) break;
+                    __nanosleep(32);
+                }
+                if (st != k * 4) continue;   // the walker passed this item already
+                const int v = t.rp[k];
+                const bool light = (t.cstart[v + 1] - t.cstart[v]) > 1;
+                if (light) build_G<LT>(c, t, w, v, gl, gmask);   // waits for v's light children
+                int old = 0;
+                if (gl == 0) old = atomicCAS(&sstate[sl], k * 4, k * 4 + 1);
+                old = __shfl_sync(gmask, old, gbase);
+                if (old != k * 4) continue;
+                build_M<LT>(h, c, t, w, v, light, gl, nH, nV, opp, mslots + (size_t)sl * LT * MStride<LT>::v);
+                __syncwarp(gmask);
+                __threadfence_block();
+                if (gl == 0) *(volatile int*)&sstate[sl] = k * 4 + 2;
+            }
+            // ---- recB / recE of the root-path nodes the walker passed with a matrix step
+            for (;;) {
+                int j = 0;
+                if (gl == 0) j = atomicAdd(&s_anext, 1);
+                j = __shfl_sync(gmask, j, gbase);
+                int cnt;
+                bool over = false;
+                for (;;) {
+                    cnt = *(volatile int*)&s_acount;
+                    if (j < cnt) break;
+                    if (*(volatile int*)&s_wdone) {
+                        cnt = *(volatile int*)&s_acount;
+                        if (j >= cnt) over = true;
+                        break;
+                    }
+                    __nanosleep(64);
+                }
+                if (over) break;
+                __threadfence_block();
+                const int k = t.argq[j];
+                const int v = t.rp[k];
+                const uint32_t Eh = t.E[(size_t)t.rp[k - 1] * LT + gl];
+                const bool light = (t.cstart[v + 1] - t.cstart[v]) > 1;
+                if (light) build_G<LT>(c, t, w, v, gl, gmask);
+                path_node<LT>(c, t, w, v, Eh, true, light, gl, gbase, gmask, nH, nV, opp, false);
             }
         }
     }
-#ifdef FGR_TIMING_DETAIL
-    if (gl == 0 && glane && m > 900)
-        printf("VAL m=%d warp=%d paths=%lld nodes=%lld light=%lld wait=%lld total=%lld rows=%lld pref=%lld B=%lld E=%lld fin=%lld\n", m, warp, vw_paths, vw_nodes,
-               vw_light, vw_wait, clock64() - vw_t0, f_rows, f_pref, f_B, f_E, f_fin);
-#endif
     __syncthreads();
     TMARK(3);
     // ---------------- backtrack: top-down path walks (S5)
@@ -1166,7 +1340,7 @@ __global__ void __launch_bounds__(32 * kLargeWarps, 1) k_dp_large(GridView g, Ne
     __syncthreads();
     TMARK(6);
     if (tid == 0 && m > 600)
-        printf("TIMING m=%d maxd=%d paths=%d prologue=%lld gather=%lld dp=%lld backtrack=%lld commit=%lld\n", m, maxd,
+        printf("TIMING m=%d maxd=%d paths=%d prologue=%lld gather=%lld dp=%lld backtrack=%lld commit=%lld\n", m, K - 1,
                npaths, tm[1] - tm[0], tm[2] - tm[1], tm[3] - tm[2], tm[4] - tm[3], tm[6] - tm[5]);
 #endif
     if (tid == 0) {
@@ -1180,7 +1354,7 @@ __global__ void __launch_bounds__(32 * kLargeWarps, 1) k_dp_large(GridView g, Ne
 template <int LT>
 __global__ void __launch_bounds__(32 * kLargeWarps, 1) k_large_prep(GridView g, NetsView nv, const int32_t* __restrict__ list,
                                                                     uint16_t* cs, uint16_t* cl, uint16_t* hv, uint16_t* bot,
-                                                                    uint16_t* pq, int32_t* npaths) {
+                                                                    uint16_t* pq, uint16_t* rpos, int32_t* npaths) {
     extern __shared__ __align__(16) unsigned char smem[];
     __shared__ int s_maxd, s_npaths, s_deep;
     if (threadIdx.x == 0) { s_maxd = 0; s_npaths = 0; }
@@ -1194,7 +1368,7 @@ __global__ void __launch_bounds__(32 * kLargeWarps, 1) k_large_prep(GridView g, 
     __syncthreads();
     for (int i = tid; i < m; i += T) {
         cs[a0 + i] = t.cstart[i]; cl[a0 + i] = t.clist[i]; hv[a0 + i] = t.hv[i];
-        bot[a0 + i] = t.bot[i]; pq[a0 + i] = t.pq[i];
+        bot[a0 + i] = t.bot[i]; pq[a0 + i] = t.pq[i]; rpos[a0 + i] = t.rpos[i];
     }
     if (tid == 0) npaths[net] = s_npaths;
 }
@@ -1387,7 +1561,8 @@ size_t smem_group(int L, int nH, int nV, int mc) {
 }
 
 size_t smem_large(int L, int nH, int nV, int m) {
-    return a16(sizeof(Hdr)) + (size_t)kLargeWarps * wscr_bytes(L) + tabs_bytes(m, L, nH, nV, true);
+    return a16(sizeof(Hdr)) + (size_t)kLargeWarps * wscr_bytes(L) + tabs_bytes(m, L, nH, nV, true) +
+           (size_t)kMR * L * ((L + 3) & ~3) * 4;
 }
 
 template <int LT>
@@ -1491,7 +1666,7 @@ size_t fgr_dp_smem_large(const fgr_grid* g, int m) { return smem_large(g->L, g->
 cudaError_t fgr_launch_dp(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int nlarge, int nmidL,
                           int nmidS, int ntwo, int maxm_large, uint32_t* seg_out, uint32_t* cost_out, uint32_t* rec_seg,
                           const int32_t* rec_off, uint32_t* rec_cost, int list_base, bool commit, const Prep* prep) {
-    const Prep pz = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
+    const Prep pz = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
     const Prep& pp = prep ? *prep : pz;
     Out o;
     o.seg = seg_out; o.cost = cost_out; o.rec_seg = rec_seg; o.rec_off = rec_off; o.rec_cost = rec_cost;
@@ -1508,7 +1683,8 @@ cudaError_t fgr_launch_dp(fgr_grid* g, cudaStream_t st, const NetsView& nv, cons
 namespace {
 template <int LT>
 cudaError_t launch_prep_lt(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int count, int maxm,
-                           uint16_t* cs, uint16_t* cl, uint16_t* hv, uint16_t* bot, uint16_t* pq, int32_t* np) {
+                           uint16_t* cs, uint16_t* cl, uint16_t* hv, uint16_t* bot, uint16_t* pq, uint16_t* rpos,
+                           int32_t* np) {
     cudaFuncAttributes fa;
     cudaError_t e = cudaFuncGetAttributes(&fa, k_large_prep<LT>);
     if (e == cudaSuccess)
@@ -1516,7 +1692,7 @@ cudaError_t launch_prep_lt(fgr_grid* g, cudaStream_t st, const NetsView& nv, con
                                  g->max_smem - (int)fa.sharedSizeBytes);
     if (e != cudaSuccess) return e;
     k_large_prep<LT><<<count, 32 * kLargeWarps, smem_large(LT, g->nH, g->nV, maxm), st>>>(g->view, nv, list, cs, cl, hv,
-                                                                                        bot, pq, np);
+                                                                                        bot, pq, rpos, np);
     g->stats.kernel_launches++;
     return cudaGetLastError();
 }
@@ -1524,10 +1700,10 @@ cudaError_t launch_prep_lt(fgr_grid* g, cudaStream_t st, const NetsView& nv, con
 
 cudaError_t fgr_launch_large_prep(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int count,
                                   int maxm, uint16_t* cs, uint16_t* cl, uint16_t* hv, uint16_t* bot, uint16_t* pq,
-                                  int32_t* np) {
+                                  uint16_t* rpos, int32_t* np) {
     if (count <= 0) return cudaSuccess;
     switch (g->L) {
-#define FGR_LT(n) case n: return launch_prep_lt<n>(g, st, nv, list, count, maxm, cs, cl, hv, bot, pq, np);
+#define FGR_LT(n) case n: return launch_prep_lt<n>(g, st, nv, list, count, maxm, cs, cl, hv, bot, pq, rpos, np);
         FGR_LT(2) FGR_LT(3) FGR_LT(4) FGR_LT(5) FGR_LT(6) FGR_LT(7) FGR_LT(8) FGR_LT(9) FGR_LT(10) FGR_LT(11)
         FGR_LT(12) FGR_LT(13) FGR_LT(14) FGR_LT(15) FGR_LT(16)
 #undef FGR_LT

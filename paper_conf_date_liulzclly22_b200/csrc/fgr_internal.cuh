@@ -82,6 +82,7 @@ struct Prep {
     const uint16_t* bot;   // bottom of the path topped by the node
     const uint16_t* pq;    // path queue (path tops, deepest first)
     const int32_t* npaths; // [num_nets]
+    const uint16_t* rpos;  // index along the root path (0xFFFF off it)
 };
 
 struct PlanCache {
@@ -180,7 +181,7 @@ cudaError_t fgr_launch_dp(fgr_grid* g, cudaStream_t st, const NetsView& nv, cons
                           bool commit, const Prep* prep);
 cudaError_t fgr_launch_large_prep(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int count,
                                   int maxm, uint16_t* cs, uint16_t* cl, uint16_t* hv, uint16_t* bot, uint16_t* pq,
-                                  int32_t* np);
+                                  uint16_t* rpos, int32_t* np);
 cudaError_t fgr_launch_commit(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int count,
                               const uint32_t* rec_seg, const int32_t* rec_off, int list_base);
 size_t fgr_dp_smem_small(const fgr_grid* g);

@@ -147,6 +147,7 @@ __global__ void k_tile_bounds(int T, const unsigned long long* __restrict__ tkey
 #define COLOR_BITS 1024
 #define COLOR_DEFER 128
 #define COLOR_UNROLL 8
+#define COLOR_CHUNK 16
 __device__ __forceinline__ void mark_colour(uint32_t* bw, int c, int wb) {
     c -= wb;
     if (c >= 0 && c < COLOR_BITS) atomicOr(&bw[c >> 5], 1u << (c & 31));
@@ -160,12 +161,33 @@ __global__ void __launch_bounds__(256) k_color(int R, const unsigned long long* 
     __shared__ uint32_t bits[8][COLOR_BITS / 32];
     __shared__ int defer[8][COLOR_DEFER];
     __shared__ int ndefer[8];
+    __shared__ int s_base, s_next;
+    if (threadIdx.x == 0) { s_base = 0; s_next = COLOR_CHUNK; }   // empty block: first taker refills
+    __syncthreads();
     const int w = threadIdx.x >> 5, lane = lane_id();
     uint32_t* bw = bits[w];
     volatile int* vcolor = color;
     for (;;) {
+        // Hierarchical tickets: a CTA takes a block of COLOR_CHUNK consecutive ranks with one
+        // global atomic; its warps take ranks from it in order through a shared counter.
+        // Deadlock-free: the smallest unfinished rank of the earliest unfinished block is
+        // always held by a running warp, and every wait is on a smaller rank.
         int r = 0;
-        if (lane == 0) r = atomicAdd(ticket, 1);
+        if (lane == 0) {
+            for (;;) {
+                const int k = atomicAdd(&s_next, 1);
+                if (k < COLOR_CHUNK) { r = s_base + k; break; }
+                // block exhausted: one warp refills it; the others spin until the new block is published
+                if (k == COLOR_CHUNK) {
+                    const int nb = atomicAdd(ticket, COLOR_CHUNK);
+                    s_base = nb;
+                    __threadfence_block();
+                    atomicExch(&s_next, 0);
+                } else {
+                    while (*(volatile int*)&s_next >= COLOR_CHUNK) __nanosleep(20);
+                }
+            }
+        }
         r = __shfl_sync(0xffffffffu, r, 0);
         if (r >= R) return;
         int x0, y0, x1, y1;

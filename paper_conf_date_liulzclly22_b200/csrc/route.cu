@@ -233,22 +233,23 @@ static fgr_status ensure_prep(fgr_grid* g, const fgr_nets* nets, int B, cudaStre
     const int R = B > 0 ? c.h_off[B] : 0;
     int maxm = 0, nl = 0;
     for (int b = 0; b < B; b++) { maxm = c.h_maxm[b] > maxm ? c.h_maxm[b] : maxm; nl += c.h_nlarge[b]; }
-    if (nl == 0) { c.prep = Prep{nullptr, nullptr, nullptr, nullptr, nullptr, nullptr}; c.prep_valid = true; return FGR_OK; }
+    if (nl == 0) { c.prep = Prep{nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr}; c.prep_valid = true; return FGR_OK; }
     const size_t M = (size_t)nets->num_nodes, N = (size_t)nets->num_nets;
     cudaError_t e;
-    char* p = (char*)fgr_scratch(g->s_prep, 5 * 2 * M + 4 * N + 4 * (size_t)nl + 64 + 5 * 16, &e);
+    char* p = (char*)fgr_scratch(g->s_prep, 6 * 2 * M + 4 * N + 4 * (size_t)nl + 64 + 6 * 16, &e);
     if (e != cudaSuccess) return fgr_cuda_fail(g, e, "prep arrays");
     auto take16 = [&](size_t n) { uint16_t* q = (uint16_t*)p; p += (2 * n + 15) & ~(size_t)15; return q; };
     uint16_t* cs = take16(M); uint16_t* cl = take16(M); uint16_t* hv = take16(M); uint16_t* bot = take16(M);
     uint16_t* pq = take16(M);
+    uint16_t* rpos = take16(M);
     int32_t* np = (int32_t*)p; p += (4 * N + 15) & ~(size_t)15;
     int32_t* list = (int32_t*)p; p += 4 * (size_t)nl;
     int* cnt = (int*)p;
     FGR_CHECK_CUDA(g, cudaMemsetAsync(cnt, 0, sizeof(int), st));
     k_large_list<<<(R + 255) / 256, 256, 0, st>>>(R, c.exec, nets->node_offset, list, cnt);
     FGR_CHECK_CUDA(g, cudaGetLastError());
-    FGR_CHECK_CUDA(g, fgr_launch_large_prep(g, st, fgr_nets_view(nets), list, nl, maxm, cs, cl, hv, bot, pq, np));
-    c.prep = Prep{cs, cl, hv, bot, pq, np};
+    FGR_CHECK_CUDA(g, fgr_launch_large_prep(g, st, fgr_nets_view(nets), list, nl, maxm, cs, cl, hv, bot, pq, rpos, np));
+    c.prep = Prep{cs, cl, hv, bot, pq, np, rpos};
     c.prep_valid = true;
     return FGR_OK;
 }

@@ -11,8 +11,8 @@ ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpuru
     python bench.py --steps 1 --warmup 1 --no-cpu-baseline --no-e2e > /dev/null 2>&1
 ncu --set full --import-source on --clock-control none -k regex:k_dp_large -s 60 -c 1 \
     -o gpurun_out/${TAG}_full_dp_large python tools/prof_step.py t9 > /dev/null 2>&1
-ncu --set full --import-source on --clock-control none -k regex:k_dp_group -s 0 -c 1 \
-    -o gpurun_out/${TAG}_full_dp_group python tools/prof_step.py t9 > /dev/null 2>&1
+ncu --set full --import-source on --clock-control none -k regex:k_dp_two -s 0 -c 1 \
+    -o gpurun_out/${TAG}_full_dp_two python tools/prof_step.py t9 > /dev/null 2>&1
 ncu --set full --import-source on --clock-control none -k regex:k_refresh -s 0 -c 2 \
     -o gpurun_out/${TAG}_full_refresh python tools/prof_step.py t9 > /dev/null 2>&1
 ncu --set full --import-source on --clock-control none -k regex:k_color -s 0 -c 1 \
@@ -20,5 +20,5 @@ ncu --set full --import-source on --clock-control none -k regex:k_color -s 0 -c 
 ls -la gpurun_out/
 # per-launch DRAM traffic of the DP kernels and the refresh over one whole step (for roofline.traffic)
 ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum --clock-control none --csv \
-    -k regex:"k_dp_large|k_dp_group|k_refresh|k_color" --log-file gpurun_out/${TAG}_traffic.csv \
+    -k regex:"k_dp_large|k_dp_group|k_dp_two|k_refresh|k_color" --log-file gpurun_out/${TAG}_traffic.csv \
     python tools/prof_step.py t9 > /dev/null 2>&1
