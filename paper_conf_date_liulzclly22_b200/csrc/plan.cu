@@ -148,12 +148,13 @@ __global__ void k_tile_bounds(int T, const unsigned long long* __restrict__ tkey
 #define COLOR_DEFER 128
 #define COLOR_UNROLL 8
 #define COLOR_CHUNK 16
+#define COLOR_BIG_HPWL 96u   // boxes with HPWL >= this take the CTA-per-net phase
 __device__ __forceinline__ void mark_colour(uint32_t* bw, int c, int wb) {
     c -= wb;
     if (c >= 0 && c < COLOR_BITS) atomicOr(&bw[c >> 5], 1u << (c & 31));
 }
 
-__global__ void __launch_bounds__(256) k_color(int R, const unsigned long long* __restrict__ box_r,
+__global__ void __launch_bounds__(256) k_color(int R, const int* __restrict__ rlim, const unsigned long long* __restrict__ box_r,
                                                const int* __restrict__ tstart, const int* __restrict__ tend,
                                                const uint4* __restrict__ entries, int tiles_x, int* color,
                                                int* __restrict__ ticket, int* __restrict__ nbatches,
@@ -164,6 +165,7 @@ __global__ void __launch_bounds__(256) k_color(int R, const unsigned long long* 
     __shared__ int s_base, s_next;
     if (threadIdx.x == 0) { s_base = 0; s_next = COLOR_CHUNK; }   // empty block: first taker refills
     __syncthreads();
+    R = *rlim;   // phase 1: the ranks below the big-box threshold (k_color_big does the rest)
     const int w = threadIdx.x >> 5, lane = lane_id();
     uint32_t* bw = bits[w];
     volatile int* vcolor = color;
@@ -271,6 +273,120 @@ __global__ void __launch_bounds__(256) k_color(int R, const unsigned long long* 
             atomicMax(nbatches, result + 1);
             atomicAdd(&bcount[result], 1);
         }
+    }
+}
+
+// First rank whose HPWL reaches `hbig` (keys are sorted by HPWL << 32 | id).
+__global__ void k_find_rbig(int R, const unsigned long long* __restrict__ keys_s, unsigned hbig, int* __restrict__ out) {
+    int lo = 0, hi = R;
+    while (lo < hi) {
+        const int mid = (lo + hi) >> 1;
+        if ((unsigned)(keys_s[mid] >> 32) < hbig) lo = mid + 1; else hi = mid;
+    }
+    *out = lo;
+}
+
+// Phase 2 of the colouring: ranks with a big box (the tail of the rank order), one CTA
+// per net, the 8 warps sharing its tile scan; same first-fit rule and dataflow waits.
+#define BIG_DEFER 1024
+__global__ void __launch_bounds__(256) k_color_big(int R, const int* __restrict__ rlim,
+                                                   const unsigned long long* __restrict__ box_r,
+                                                   const int* __restrict__ tstart, const int* __restrict__ tend,
+                                                   const uint4* __restrict__ entries, int tiles_x, int* color,
+                                                   int* __restrict__ ticket, int* __restrict__ nbatches,
+                                                   int* __restrict__ bcount) {
+    __shared__ uint32_t bits[COLOR_BITS / 32];
+    __shared__ int defer[BIG_DEFER];
+    __shared__ int ndefer, s_r, s_res;
+    const int w = threadIdx.x >> 5, lane = lane_id(), tid = threadIdx.x;
+    volatile int* vcolor = color;
+    const int R0 = *rlim;
+    for (;;) {
+        if (tid == 0) s_r = R0 + atomicAdd(ticket, 1);
+        __syncthreads();
+        const int r = s_r;
+        if (r >= R) return;
+        int x0, y0, x1, y1;
+        unpack_box(box_r[r], x0, y0, x1, y1);
+        const int tx0 = x0 >> TILE_SHIFT, ty0 = y0 >> TILE_SHIFT;
+        const int ntx = (x1 >> TILE_SHIFT) - tx0 + 1, nty = (y1 >> TILE_SHIFT) - ty0 + 1;
+        int result = -1;
+        for (int wb = 0; result < 0; wb += COLOR_BITS) {
+            if (tid < COLOR_BITS / 32) bits[tid] = 0;
+            if (tid == 0) { ndefer = 0; s_res = -1; }
+            __syncthreads();
+            for (int ti = w; ti < ntx * nty; ti += 8) {
+                const int tx = tx0 + ti % ntx, ty = ty0 + ti / ntx;
+                const int t = ty * tiles_x + tx;
+                const int s = tstart[t], e = tend[t];
+                for (int base = s; base < e; base += 32 * COLOR_UNROLL) {
+                    int rr[COLOR_UNROLL];
+                    unsigned long long bb[COLOR_UNROLL];
+#pragma unroll
+                    for (int u = 0; u < COLOR_UNROLL; u++) {
+                        const int j = base + u * 32 + lane;
+                        if (j < e) {
+                            const uint4 q = __ldg(entries + j);
+                            rr[u] = (int)q.x;
+                            bb[u] = (unsigned long long)q.y | ((unsigned long long)q.z << 32);
+                        } else {
+                            rr[u] = 0x7FFFFFFF;
+                            bb[u] = 0ull;
+                        }
+                    }
+                    bool stop = false;
+#pragma unroll
+                    for (int u = 0; u < COLOR_UNROLL; u++) {
+                        stop |= (rr[u] != 0x7FFFFFFF && rr[u] >= r);
+                        if (rr[u] < r) {
+                            int a0, b0, a1, b1;
+                            unpack_box(bb[u], a0, b0, a1, b1);
+                            if (!(a1 < x0 || x1 < a0 || b1 < y0 || y1 < b0) &&
+                                (max(a0, x0) >> TILE_SHIFT) == tx && (max(b0, y0) >> TILE_SHIFT) == ty) {
+                                const int c = vcolor[rr[u]];
+                                if (c >= 0) mark_colour(bits, c, wb);
+                                else {
+                                    const int k = atomicAdd(&ndefer, 1);
+                                    if (k < BIG_DEFER) defer[k] = rr[u];
+                                    else {
+                                        int cc;
+                                        while ((cc = vcolor[rr[u]]) < 0) __nanosleep(20);
+                                        mark_colour(bits, cc, wb);
+                                    }
+                                }
+                            }
+                        }
+                    }
+                    if (__any_sync(0xffffffffu, stop)) break;
+                }
+            }
+            __syncthreads();
+            const int nd = min(ndefer, BIG_DEFER);
+            for (int k = tid; k < nd; k += blockDim.x) {
+                int cc;
+                while ((cc = vcolor[defer[k]]) < 0) __nanosleep(20);
+                mark_colour(bits, cc, wb);
+            }
+            __syncthreads();
+            if (w == 0) {
+                const uint32_t freeb = ~bits[lane];
+                const uint32_t any = __ballot_sync(0xffffffffu, freeb != 0);
+                if (any && lane == 0) {
+                    const int ql = __ffs(any) - 1;
+                    const uint32_t fw = ~bits[ql];
+                    s_res = ql * 32 + __ffs(fw) - 1;
+                }
+            }
+            __syncthreads();
+            if (s_res >= 0) result = wb + s_res;
+            __syncthreads();
+        }
+        if (tid == 0) {
+            atomicExch(&color[r], result);
+            atomicMax(nbatches, result + 1);
+            atomicAdd(&bcount[result], 1);
+        }
+        __syncthreads();
     }
 }
 
@@ -469,8 +585,12 @@ extern "C" FGR_API fgr_status fgr_plan(fgr_grid* g, const fgr_nets* nets, int32_
         int need = (R + 7) / 8;
         if (blocks > need) blocks = need;
         ps = fgr_prof_begin(g, PROF_COLOR, st);
-        k_color<<<blocks, 256, 0, st>>>(R, box_r, tstart, tend, entries, tiles_x, color, counters + 3, counters + 4,
-                                        d_bcount);
+        // ranks below the big-box threshold: a warp per net; the big boxes: a CTA per net
+        k_find_rbig<<<1, 1, 0, st>>>(R, keys_s, COLOR_BIG_HPWL, counters + 5);
+        k_color<<<blocks, 256, 0, st>>>(R, counters + 5, box_r, tstart, tend, entries, tiles_x, color, counters + 3,
+                                        counters + 4, d_bcount);
+        k_color_big<<<g->num_sms * 4, 256, 0, st>>>(R, counters + 5, box_r, tstart, tend, entries, tiles_x, color,
+                                                   counters + 6, counters + 4, d_bcount);
         fgr_prof_end(g, ps, st);
         FGR_CHECK_CUDA(g, cudaGetLastError());
         g->stats.kernel_launches++;
