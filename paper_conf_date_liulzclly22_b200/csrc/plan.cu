@@ -148,7 +148,7 @@ __global__ void k_tile_bounds(int T, const unsigned long long* __restrict__ tkey
 #define COLOR_DEFER 128
 #define COLOR_UNROLL 8
 #define COLOR_CHUNK 16
-#define COLOR_BIG_HPWL 96u   // boxes with HPWL >= this take the CTA-per-net phase
+#define COLOR_BIG_HPWL 24u   // boxes with HPWL >= this take the CTA-per-net phase
 __device__ __forceinline__ void mark_colour(uint32_t* bw, int c, int wb) {
     c -= wb;
     if (c >= 0 && c < COLOR_BITS) atomicOr(&bw[c >> 5], 1u << (c & 31));
