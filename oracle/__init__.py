@@ -28,6 +28,23 @@ class _Grid(ctypes.Structure):
     ]
 
 
+class _Pattern(ctypes.Structure):
+    _fields_ = [("hybrid_lo", ctypes.c_int32), ("hybrid_hi", ctypes.c_int32)]
+
+
+def _pat(hybrid):
+    """hybrid = None (L only) or (t1, t2): edges with t1 <= |dx|+|dy| <= t2 take hybrid L+Z patterns."""
+    if hybrid is None:
+        return None
+    p = _Pattern()
+    p.hybrid_lo, p.hybrid_hi = int(hybrid[0]), int(hybrid[1])
+    return p
+
+
+def _pp(p):
+    return ctypes.byref(p) if p is not None else ctypes.c_void_p(0)
+
+
 class _Nets(ctypes.Structure):
     _fields_ = [
         ("num_nets", ctypes.c_int32), ("node_offset", ctypes.c_void_p),
@@ -51,8 +68,13 @@ def _lib():
         lib.orc_commit_net.argtypes = [P, P, ctypes.c_int32, P, P]
         lib.orc_route.argtypes = [P, P, P, ctypes.c_int32, P, P, P, ctypes.c_int, P]
         lib.orc_recost_net.argtypes = [P, P, ctypes.c_int32, P, P, P]
+        lib.orc_route_net_ex.argtypes = [P, P, ctypes.c_int32, P, P, P, P, P]
+        lib.orc_commit_net_ex.argtypes = [P, P, ctypes.c_int32, P, P, P]
+        lib.orc_route_ex.argtypes = [P, P, P, ctypes.c_int32, P, P, P, ctypes.c_int, P, P, P]
+        lib.orc_recost_net_ex.argtypes = [P, P, ctypes.c_int32, P, P, P, P]
         for f in ("orc_cost_table", "orc_validate", "orc_plan", "orc_route_net", "orc_commit_net",
-                  "orc_route", "orc_recost_net"):
+                  "orc_route", "orc_recost_net", "orc_route_net_ex", "orc_commit_net_ex", "orc_route_ex",
+                  "orc_recost_net_ex"):
             getattr(lib, f).restype = ctypes.c_int
         _LIB = lib
     return _LIB
@@ -118,41 +140,53 @@ class Oracle:
             raise ValueError(f"orc_plan rc={rc}")
         return b, int(nb[0])
 
-    def route(self, batch_of_net, num_batches, demand=None, sequential=False, hashes=False):
-        """Batches in sequence -> (seg uint32[M], net_cost uint32[N], demand int32[L,ny,nx][, hashes])."""
+    def route(self, batch_of_net, num_batches, demand=None, sequential=False, hashes=False, hybrid=None,
+              with_zmid=False):
+        """Batches in sequence -> (seg uint32[M], net_cost uint32[N], demand int32[L,ny,nx][, hashes][, zmid]).
+
+        hybrid=(t1, t2) enables the hybrid L+Z patterns on edges with t1 <= |dx|+|dy| <= t2;
+        zmid int32[M] = mid | lb << 16 for edges routed as a Z, -1 elsewhere."""
         dem = self.zero_demand() if demand is None else np.ascontiguousarray(demand, np.int32).copy()
         seg = np.zeros(self.d.num_nodes, np.uint32)
         cost = np.zeros(self.d.num_nets, np.uint32)
+        zmid = np.full(self.d.num_nodes, -1, np.int32)
         bon = np.ascontiguousarray(batch_of_net, np.int32)
         h = np.zeros(max(num_batches, 1), np.uint64) if hashes else None
-        rc = _lib().orc_route(ctypes.byref(self.g), ctypes.byref(self.n), _p(bon), int(num_batches),
-                              _p(dem), _p(seg), _p(cost), int(bool(sequential)), _p(h))
+        pat = _pat(hybrid)
+        rc = _lib().orc_route_ex(ctypes.byref(self.g), ctypes.byref(self.n), _p(bon), int(num_batches),
+                                 _p(dem), _p(seg), _p(cost), int(bool(sequential)), _p(h), _pp(pat), _p(zmid))
         if rc != ORC_OK:
             raise ValueError(f"orc_route rc={rc}")
+        out = [seg, cost, dem]
         if hashes:
-            return seg, cost, dem, h[:num_batches]
-        return seg, cost, dem
+            out.append(h[:num_batches])
+        if with_zmid:
+            out.append(zmid)
+        return tuple(out)
 
-    def route_net(self, net, demand, seg=None):
+    def route_net(self, net, demand, seg=None, hybrid=None, zmid=None):
         """One net's DP on a given demand; returns (seg uint32[M] with this net filled, cost)."""
         if seg is None:
             seg = np.zeros(self.d.num_nodes, np.uint32)
         dem = np.ascontiguousarray(demand, np.int32)
         c = np.zeros(1, np.uint32)
-        rc = _lib().orc_route_net(ctypes.byref(self.g), ctypes.byref(self.n), int(net), _p(dem), _p(seg), _p(c))
+        rc = _lib().orc_route_net_ex(ctypes.byref(self.g), ctypes.byref(self.n), int(net), _p(dem), _p(seg), _p(c),
+                                     _pp(_pat(hybrid)), _p(zmid))
         if rc != ORC_OK:
             raise ValueError(f"orc_route_net rc={rc}")
         return seg, int(c[0])
 
-    def commit_net(self, net, seg, demand):
-        _lib().orc_commit_net(ctypes.byref(self.g), ctypes.byref(self.n), int(net),
-                              _p(np.ascontiguousarray(seg, np.uint32)), _p(demand))
+    def commit_net(self, net, seg, demand, zmid=None):
+        _lib().orc_commit_net_ex(ctypes.byref(self.g), ctypes.byref(self.n), int(net),
+                                 _p(np.ascontiguousarray(seg, np.uint32)),
+                                 _p(None if zmid is None else np.ascontiguousarray(zmid, np.int32)), _p(demand))
 
-    def recost_net(self, net, demand, seg) -> int:
+    def recost_net(self, net, demand, seg, zmid=None) -> int:
         c = np.zeros(1, np.uint64)
-        _lib().orc_recost_net(ctypes.byref(self.g), ctypes.byref(self.n), int(net),
-                              _p(np.ascontiguousarray(demand, np.int32)),
-                              _p(np.ascontiguousarray(seg, np.uint32)), _p(c))
+        _lib().orc_recost_net_ex(ctypes.byref(self.g), ctypes.byref(self.n), int(net),
+                                 _p(np.ascontiguousarray(demand, np.int32)),
+                                 _p(np.ascontiguousarray(seg, np.uint32)),
+                                 _p(None if zmid is None else np.ascontiguousarray(zmid, np.int32)), _p(c))
         return int(c[0])
 
     def run(self):

@@ -207,14 +207,96 @@ int orc_plan(const orc_grid* g, const orc_nets* n, int32_t* batch_of_net, int32_
  *   B[v][ls]   = min over spans [lo,hi] containing ls and the pin span of F_v
  *   root total = min over spans containing the root pin span of F_r   (generalised Eq. (4))
  */
-static int route_net(const cost_ctx* cc, const orc_nets* n, int32_t net, uint32_t* seg, uint32_t* net_cost) {
+/* Hybrid selection (reading R23): a bent tree edge whose
+ * two-pin HPWL |dx|+|dy| lies in [hybrid_lo, hybrid_hi] is a "medium" two-pin
+ * net and takes the hybrid L+Z patterns; every other edge takes the L patterns. */
+static int is_hybrid_edge(const orc_pattern* pat, int xv, int yv, int xu, int yu) {
+    if (!pat || xv == xu || yv == yu) return 0;
+    int h = abs(xv - xu) + abs(yv - yu);
+    return h >= pat->hybrid_lo && h <= pat->hybrid_hi;
+}
+
+/*
+ * c*(Ps,Pt,lt) of one hybrid edge, §III-E/F (Eqs. (8)-(14), L831-1041,
+ * and the hybrid candidate set, L1043-1092): the candidates are the two L
+ * shapes (the bend pairs whose target bend point coincides with Pt, L1062-1068)
+ * and the Z shapes whose bend points lie strictly inside the box (reading R24):
+ *   HVH: Bs = (xm, yv), Bt = (xm, yu) for every xm strictly between xv and xu,
+ *   VHV: Bs = (xv, ym), Bt = (xu, ym) for every ym strictly between yv and yu.
+ * Eq. (8): c = cw(Ps,Bs,ls) + cv(Bs,ls,lb) + cw(Bs,Bt,lb) + cv(Bt,lb,lt) + cw(Bt,Pt,lt),
+ * Eq. (9)/(14): min over ls, lb of cbc(Ps,ls) + c; Eq. (10): min over the candidates.
+ * Tie-break (reading R25): the first minimum in the order (ls, candidate, lb),
+ * candidates = the L shape first, then Z shapes by increasing xm / ym.
+ * Writes E[lt], recE[lt] = ls and recZ[lt] = xm|ym | lb << 16 for a Z (else -1).
+ */
+static void hybrid_edge(const cost_ctx* c, const uint64_t* Bv, int xv, int yv, int xu, int yu,
+                        uint64_t* E, uint8_t* recE, int32_t* recZ) {
+    const orc_grid* g = c->g;
+    int L = g->nlayers;
+    int nxm = abs(xu - xv) - 1, nym = abs(yu - yv) - 1;      /* interior bend positions */
+    int xlo = xv < xu ? xv : xu, ylo = yv < yu ? yv : yu;
+    /* wire costs of the three legs of every Z candidate on every layer, by direct sums */
+    uint64_t* hw = (uint64_t*)malloc(sizeof(uint64_t) * (size_t)(nxm > 0 ? nxm : 1) * L * 3);
+    uint64_t* vw = (uint64_t*)malloc(sizeof(uint64_t) * (size_t)(nym > 0 ? nym : 1) * L * 3);
+    for (int i = 0; i < nxm; i++) {
+        int xm = xlo + 1 + i;
+        for (int l = 0; l < L; l++) {
+            hw[((size_t)i * L + l) * 3 + 0] = wire_cost(c, l, xv, yv, xm, yv);   /* Ps -> Bs */
+            hw[((size_t)i * L + l) * 3 + 1] = wire_cost(c, l, xm, yv, xm, yu);   /* Bs -> Bt */
+            hw[((size_t)i * L + l) * 3 + 2] = wire_cost(c, l, xm, yu, xu, yu);   /* Bt -> Pt */
+        }
+    }
+    for (int i = 0; i < nym; i++) {
+        int ym = ylo + 1 + i;
+        for (int l = 0; l < L; l++) {
+            vw[((size_t)i * L + l) * 3 + 0] = wire_cost(c, l, xv, yv, xv, ym);
+            vw[((size_t)i * L + l) * 3 + 1] = wire_cost(c, l, xv, ym, xu, ym);
+            vw[((size_t)i * L + l) * 3 + 2] = wire_cost(c, l, xu, ym, xu, yu);
+        }
+    }
+    for (int lt = 0; lt < L; lt++) {
+        uint64_t best = INF; int bls = 0; int32_t bz = -1;
+        for (int ls = 0; ls < L; ls++) {
+            if (g->dir[ls] != g->dir[lt]) {
+                /* the L shape: bend 0 = (xu, yv) when leg 1 is horizontal, bend 1 = (xv, yu) */
+                int bx = g->dir[ls] == 0 ? xu : xv, by = g->dir[ls] == 0 ? yv : yu;
+                uint64_t cost = add(add(add(Bv[ls], wire_cost(c, ls, xv, yv, bx, by)), via_stack(g, ls, lt)),
+                                    wire_cost(c, lt, bx, by, xu, yu));
+                if (cost < best) { best = cost; bls = ls; bz = -1; }
+                continue;
+            }
+            int hvh = g->dir[ls] == 0;
+            int nm = hvh ? nxm : nym;
+            const uint64_t* w = hvh ? hw : vw;
+            for (int i = 0; i < nm; i++)
+                for (int lb = 0; lb < L; lb++) {
+                    uint64_t cost = add(Bv[ls], w[((size_t)i * L + ls) * 3 + 0]);   /* Eq. (11) */
+                    cost = add(cost, add(via_stack(g, ls, lb), w[((size_t)i * L + lb) * 3 + 1]));   /* Eq. (12) */
+                    cost = add(cost, add(via_stack(g, lb, lt), w[((size_t)i * L + lt) * 3 + 2]));   /* Eq. (13) */
+                    if (cost < best) {
+                        best = cost; bls = ls;
+                        bz = (int32_t)((hvh ? xlo : ylo) + 1 + i) | (int32_t)(lb << 16);
+                    }
+                }
+        }
+        E[lt] = best;
+        recE[lt] = (uint8_t)bls;
+        recZ[lt] = bz;
+    }
+    free(hw); free(vw);
+}
+
+static int route_net(const cost_ctx* cc, const orc_nets* n, int32_t net, uint32_t* seg, uint32_t* net_cost,
+                     const orc_pattern* pat, int32_t* zmid) {
     const orc_grid* g = cc->g;
     const cost_ctx c = *cc;
     int a = n->node_offset[net], m = n->node_offset[net + 1] - a, L = g->nlayers;
+    if (zmid) for (int v = a; v < a + m; v++) zmid[v] = -1;
     if (m < 2) { if (m == 1) seg[a] = 0xFFFFFFFFu; *net_cost = 0; return ORC_OK; }
 
     uint64_t* E = (uint64_t*)malloc(sizeof(uint64_t) * m * L);   /* c*(v -> parent, lt) */
     uint8_t* recE = (uint8_t*)malloc((size_t)m * L);             /* argmin ls of E[v][lt] */
+    int32_t* recZ = (int32_t*)malloc(sizeof(int32_t) * (size_t)m * L);   /* hybrid: Z bend of E[v][lt] or -1 */
     uint8_t* recLo = (uint8_t*)malloc((size_t)m * L);            /* argmin span of B[v][ls] */
     uint8_t* recHi = (uint8_t*)malloc((size_t)m * L);
     uint64_t* F = (uint64_t*)malloc(sizeof(uint64_t) * L * L);
@@ -279,6 +361,11 @@ static int route_net(const cost_ctx* cc, const orc_nets* n, int32_t net, uint32_
         int u = n->parent[a + v];
         int xv = n->x[a + v], yv = n->y[a + v], xu = n->x[a + u], yu = n->y[a + u];
         int straight = (xv == xu) || (yv == yu);
+        for (int lt = 0; lt < L; lt++) recZ[(int64_t)v * L + lt] = -1;
+        if (is_hybrid_edge(pat, xv, yv, xu, yu)) {
+            hybrid_edge(&c, Bv, xv, yv, xu, yu, E + (int64_t)v * L, recE + (int64_t)v * L, recZ + (int64_t)v * L);
+            continue;
+        }
         for (int lt = 0; lt < L; lt++) {
             uint64_t best = INF; int bls = 0;
             if (straight) {
@@ -314,25 +401,35 @@ static int route_net(const cost_ctx* cc, const orc_nets* n, int32_t net, uint32_
             int xv = n->x[a + v], yv = n->y[a + v], xu = n->x[a + u], yu = n->y[a + u];
             int straight = (xv == xu) || (yv == yu);
             int bend = straight ? 0 : (g->dir[lt] == 1 ? 0 : 1);
+            int32_t z = recZ[(int64_t)v * L + lt];
+            if (z >= 0) {   /* a Z shape (hybrid edges only): 2 = HVH, 3 = VHV */
+                bend = g->dir[ls] == 0 ? 2 : 3;
+                if (zmid) zmid[a + v] = z;
+            }
             seg[a + v] = (uint32_t)bend | ((uint32_t)ls << 8) | ((uint32_t)lt << 16) | ((uint32_t)straight << 24);
             spanLo[v] = recLo[(int64_t)v * L + ls];
             spanHi[v] = recHi[(int64_t)v * L + ls];
         }
     }
-    free(E); free(recE); free(recLo); free(recHi); free(F); free(Bv);
+    free(E); free(recE); free(recZ); free(recLo); free(recHi); free(F); free(Bv);
     free(nchild); free(child); free(spanLo); free(spanHi);
+    return rc;
+}
+
+int orc_route_net_ex(const orc_grid* g, const orc_nets* n, int32_t net, const int32_t* demand,
+                     uint32_t* seg, uint32_t* net_cost, const orc_pattern* pat, int32_t* zmid) {
+    cost_ctx c;
+    c.g = g; c.demand = demand;
+    c.table = (int64_t*)malloc(sizeof(int64_t) * g->nlayers * (2 * g->slack_clamp + 1));
+    orc_cost_table(g, c.table);
+    int rc = route_net(&c, n, net, seg, net_cost, pat, zmid);
+    free(c.table);
     return rc;
 }
 
 int orc_route_net(const orc_grid* g, const orc_nets* n, int32_t net, const int32_t* demand,
                   uint32_t* seg, uint32_t* net_cost) {
-    cost_ctx c;
-    c.g = g; c.demand = demand;
-    c.table = (int64_t*)malloc(sizeof(int64_t) * g->nlayers * (2 * g->slack_clamp + 1));
-    orc_cost_table(g, c.table);
-    int rc = route_net(&c, n, net, seg, net_cost);
-    free(c.table);
-    return rc;
+    return orc_route_net_ex(g, n, net, demand, seg, net_cost, NULL, NULL);
 }
 
 /* +1 track on every unit edge of a leg (reading R16); zero-length legs add nothing. */
@@ -346,28 +443,53 @@ static void commit_leg(const orc_grid* g, int l, int xa, int ya, int xb, int yb,
     }
 }
 
-int orc_commit_net(const orc_grid* g, const orc_nets* n, int32_t net, const uint32_t* seg, int32_t* demand) {
+/* The straight legs of one chosen route v -> u as (layer, xa, ya, xb, yb); returns how many (1..3).
+ * Z shapes (bend 2 = HVH, 3 = VHV) take their middle coordinate and lb from zmid. */
+static int route_legs(uint32_t s, int32_t z, int xv, int yv, int xu, int yu, int legs[3][5]) {
+    int bend = s & 0xFF, ls = (s >> 8) & 0xFF, lt = (s >> 16) & 0xFF, straight = (s >> 24) & 0xFF;
+    if (straight) {
+        int q[5] = {lt, xv, yv, xu, yu};
+        memcpy(legs[0], q, sizeof(q));
+        return 1;
+    }
+    if (bend >= 2) {
+        int mid = z & 0xFFFF, lb = (z >> 16) & 0xFF;
+        int bsx = bend == 2 ? mid : xv, bsy = bend == 2 ? yv : mid;   /* source bend point Bs */
+        int btx = bend == 2 ? mid : xu, bty = bend == 2 ? yu : mid;   /* target bend point Bt */
+        int q0[5] = {ls, xv, yv, bsx, bsy}, q1[5] = {lb, bsx, bsy, btx, bty}, q2[5] = {lt, btx, bty, xu, yu};
+        memcpy(legs[0], q0, sizeof(q0)); memcpy(legs[1], q1, sizeof(q1)); memcpy(legs[2], q2, sizeof(q2));
+        return 3;
+    }
+    int bx = bend == 0 ? xu : xv, by = bend == 0 ? yv : yu;
+    int q0[5] = {ls, xv, yv, bx, by}, q1[5] = {lt, bx, by, xu, yu};
+    memcpy(legs[0], q0, sizeof(q0)); memcpy(legs[1], q1, sizeof(q1));
+    return 2;
+}
+
+int orc_commit_net_ex(const orc_grid* g, const orc_nets* n, int32_t net, const uint32_t* seg, const int32_t* zmid,
+                      int32_t* demand) {
     int a = n->node_offset[net], m = n->node_offset[net + 1] - a;
     for (int v = 1; v < m; v++) {
-        uint32_t s = seg[a + v];
-        int bend = s & 0xFF, ls = (s >> 8) & 0xFF, lt = (s >> 16) & 0xFF, straight = (s >> 24) & 0xFF;
         int u = n->parent[a + v];
-        int xv = n->x[a + v], yv = n->y[a + v], xu = n->x[a + u], yu = n->y[a + u];
-        if (straight) { commit_leg(g, lt, xv, yv, xu, yu, demand); continue; }
-        int bx = bend == 0 ? xu : xv, by = bend == 0 ? yv : yu;
-        commit_leg(g, ls, xv, yv, bx, by, demand);
-        commit_leg(g, lt, bx, by, xu, yu, demand);
+        int legs[3][5];
+        int k = route_legs(seg[a + v], zmid ? zmid[a + v] : -1, n->x[a + v], n->y[a + v], n->x[a + u], n->y[a + u], legs);
+        for (int j = 0; j < k; j++) commit_leg(g, legs[j][0], legs[j][1], legs[j][2], legs[j][3], legs[j][4], demand);
     }
     return ORC_OK;
 }
 
+int orc_commit_net(const orc_grid* g, const orc_nets* n, int32_t net, const uint32_t* seg, int32_t* demand) {
+    return orc_commit_net_ex(g, n, net, seg, NULL, demand);
+}
+
 /*
  * Independent re-costing of a chosen route (used by the invariant tests):
- * wires + one bend via stack per bent edge + at every node the via stack over
- * the hull of {pin span, departure layer ls, arrival layers lt of the children}.
+ * wires + the via stack at every bend point (one per L, two per Z) + at every
+ * node the via stack over the hull of {pin span, departure layer ls, arrival
+ * layers lt of the children}.
  */
-int orc_recost_net(const orc_grid* g, const orc_nets* n, int32_t net, const int32_t* demand,
-                   const uint32_t* seg, uint64_t* cost) {
+int orc_recost_net_ex(const orc_grid* g, const orc_nets* n, int32_t net, const int32_t* demand,
+                      const uint32_t* seg, const int32_t* zmid, uint64_t* cost) {
     int a = n->node_offset[net], m = n->node_offset[net + 1] - a, L = g->nlayers, S = g->slack_clamp;
     cost_ctx c; c.g = g; c.demand = demand;
     c.table = (int64_t*)malloc(sizeof(int64_t) * L * (2 * S + 1));
@@ -381,15 +503,13 @@ int orc_recost_net(const orc_grid* g, const orc_nets* n, int32_t net, const int3
     uint64_t total = 0;
     for (int v = 1; v < m; v++) {
         uint32_t s = seg[a + v];
-        int bend = s & 0xFF, ls = (s >> 8) & 0xFF, lt = (s >> 16) & 0xFF, straight = (s >> 24) & 0xFF;
+        int ls = (s >> 8) & 0xFF, lt = (s >> 16) & 0xFF;
         int u = n->parent[a + v];
-        int xv = n->x[a + v], yv = n->y[a + v], xu = n->x[a + u], yu = n->y[a + u];
-        if (straight) total = add(total, wire_cost(&c, lt, xv, yv, xu, yu));
-        else {
-            int bx = bend == 0 ? xu : xv, by = bend == 0 ? yv : yu;
-            total = add(total, wire_cost(&c, ls, xv, yv, bx, by));
-            total = add(total, via_stack(g, ls, lt));
-            total = add(total, wire_cost(&c, lt, bx, by, xu, yu));
+        int legs[3][5];
+        int k = route_legs(s, zmid ? zmid[a + v] : -1, n->x[a + v], n->y[a + v], n->x[a + u], n->y[a + u], legs);
+        for (int j = 0; j < k; j++) {
+            total = add(total, wire_cost(&c, legs[j][0], legs[j][1], legs[j][2], legs[j][3], legs[j][4]));
+            if (j > 0) total = add(total, via_stack(g, legs[j - 1][0], legs[j][0]));   /* bend point vias */
         }
         if (ls < hlo[v]) hlo[v] = ls;
         if (ls > hhi[v]) hhi[v] = ls;
@@ -401,6 +521,11 @@ int orc_recost_net(const orc_grid* g, const orc_nets* n, int32_t net, const int3
     *cost = total;
     free(c.table); free(hlo); free(hhi);
     return ORC_OK;
+}
+
+int orc_recost_net(const orc_grid* g, const orc_nets* n, int32_t net, const int32_t* demand,
+                   const uint32_t* seg, uint64_t* cost) {
+    return orc_recost_net_ex(g, n, net, demand, seg, NULL, cost);
 }
 
 static uint64_t fnv1a(const int32_t* d, int64_t n) {
@@ -419,6 +544,13 @@ static uint64_t fnv1a(const int32_t* d, int64_t n) {
 int orc_route(const orc_grid* g, const orc_nets* n, const int32_t* batch_of_net, int32_t num_batches,
               int32_t* demand, uint32_t* seg, uint32_t* net_cost, int sequential_within_batch,
               uint64_t* batch_hash) {
+    return orc_route_ex(g, n, batch_of_net, num_batches, demand, seg, net_cost, sequential_within_batch, batch_hash,
+                        NULL, NULL);
+}
+
+int orc_route_ex(const orc_grid* g, const orc_nets* n, const int32_t* batch_of_net, int32_t num_batches,
+                 int32_t* demand, uint32_t* seg, uint32_t* net_cost, int sequential_within_batch,
+                 uint64_t* batch_hash, const orc_pattern* pat, int32_t* zmid) {
     int32_t bad;
     if (orc_validate(g, n, &bad) != ORC_OK) return ORC_INVALID;
     int N = n->num_nets;
@@ -428,7 +560,11 @@ int orc_route(const orc_grid* g, const orc_nets* n, const int32_t* batch_of_net,
     for (int i = 0; i < N; i++) {
         if (batch_of_net[i] >= num_batches) { free(cnt); return ORC_INVALID; }
         if (batch_of_net[i] >= 0) cnt[batch_of_net[i] + 1]++;
-        else { int a = n->node_offset[i]; for (int v = a; v < n->node_offset[i + 1]; v++) seg[v] = 0xFFFFFFFFu; net_cost[i] = 0; }
+        else {
+            int a = n->node_offset[i];
+            for (int v = a; v < n->node_offset[i + 1]; v++) { seg[v] = 0xFFFFFFFFu; if (zmid) zmid[v] = -1; }
+            net_cost[i] = 0;
+        }
     }
     for (int b = 0; b < num_batches; b++) cnt[b + 1] += cnt[b];
     int* lst = (int*)malloc(sizeof(int) * (N > 0 ? N : 1));
@@ -442,11 +578,11 @@ int orc_route(const orc_grid* g, const orc_nets* n, const int32_t* batch_of_net,
     orc_cost_table(g, c.table);
     for (int b = 0; b < num_batches && rc == ORC_OK; b++) {
         for (int k = cnt[b]; k < cnt[b + 1] && rc == ORC_OK; k++) {
-            rc = route_net(&c, n, lst[k], seg, &net_cost[lst[k]]);
-            if (sequential_within_batch) orc_commit_net(g, n, lst[k], seg, demand);
+            rc = route_net(&c, n, lst[k], seg, &net_cost[lst[k]], pat, zmid);
+            if (sequential_within_batch) orc_commit_net_ex(g, n, lst[k], seg, zmid, demand);
         }
         if (!sequential_within_batch)
-            for (int k = cnt[b]; k < cnt[b + 1]; k++) orc_commit_net(g, n, lst[k], seg, demand);
+            for (int k = cnt[b]; k < cnt[b + 1]; k++) orc_commit_net_ex(g, n, lst[k], seg, zmid, demand);
         if (batch_hash) batch_hash[b] = fnv1a(demand, dsize);
     }
     free(c.table); free(cnt); free(lst); free(pos);

@@ -12,7 +12,10 @@
  *   wire edge (x,y)-(x+1,y) (x = nx-1 unused); for a V layer, entry (y,x) is the
  *   wire edge (x,y)-(x,y+1) (y = ny-1 unused).
  *   seg[node] (node = global node index of the child endpoint of a tree edge):
- *   bend | ls<<8 | lt<<16 | straight<<24; roots get 0xFFFFFFFF.
+ *   bend | ls<<8 | lt<<16 | straight<<24; roots get 0xFFFFFFFF.  bend 0/1 = the
+ *   two L shapes; with hybrid patterns also 2 = Z HVH, 3 = Z VHV, whose middle
+ *   coordinate (xm for HVH, ym for VHV) and middle layer lb are in
+ *   zmid[node] = mid | lb << 16 (-1 for every non-Z edge).
  */
 #ifndef FGR_ORACLE_H
 #define FGR_ORACLE_H
@@ -40,6 +43,14 @@ typedef struct {
     const int32_t* parent;          /* net-local; parent[i] < i; -1 at local 0 */
 } orc_nets;
 
+/* Hybrid L+Z selection (§III-F and §IV-D):
+ * bent tree edges with hybrid_lo <= |dx|+|dy| <= hybrid_hi take the hybrid
+ * patterns (the paper's "medium" two-pin nets, t1 = 100, t2 = 500); all other
+ * edges the L patterns.  NULL pattern (or lo > hi) = L only (FastGRL). */
+typedef struct {
+    int32_t hybrid_lo, hybrid_hi;
+} orc_pattern;
+
 #define ORC_OK 0
 #define ORC_INVALID 1
 #define ORC_RANGE 2
@@ -55,5 +66,15 @@ int orc_route(const orc_grid* g, const orc_nets* n, const int32_t* batch_of_net,
               uint64_t* batch_hash /* [num_batches] or NULL */);
 int orc_recost_net(const orc_grid* g, const orc_nets* n, int32_t net, const int32_t* demand,
                    const uint32_t* seg, uint64_t* cost);
+
+int orc_route_net_ex(const orc_grid* g, const orc_nets* n, int32_t net, const int32_t* demand,
+                     uint32_t* seg, uint32_t* net_cost, const orc_pattern* pat, int32_t* zmid);
+int orc_commit_net_ex(const orc_grid* g, const orc_nets* n, int32_t net, const uint32_t* seg, const int32_t* zmid,
+                      int32_t* demand);
+int orc_route_ex(const orc_grid* g, const orc_nets* n, const int32_t* batch_of_net, int32_t num_batches,
+                 int32_t* demand, uint32_t* seg, uint32_t* net_cost, int sequential_within_batch,
+                 uint64_t* batch_hash, const orc_pattern* pat, int32_t* zmid);
+int orc_recost_net_ex(const orc_grid* g, const orc_nets* n, int32_t net, const int32_t* demand,
+                      const uint32_t* seg, const int32_t* zmid, uint64_t* cost);
 
 #endif

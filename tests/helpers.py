@@ -51,11 +51,20 @@ def make_seg(bend, ls, lt, straight):
     return bend | (ls << 8) | (lt << 16) | (straight << 24)
 
 
-def legs_of_edge(xv, yv, xu, yu, seg):
-    """[(layer, xa, ya, xb, yb)] of a chosen route for tree edge v -> u (include/fastgr.h semantics)."""
+def legs_of_edge(xv, yv, xu, yu, seg, z=-1):
+    """[(layer, xa, ya, xb, yb)] of a chosen route for tree edge v -> u (include/fastgr.h semantics).
+
+    bend 2 / 3 = Z shape HVH / VHV (§III-E) with z = mid | lb << 16."""
     f = seg_fields(seg)
     if f["straight"]:
         return [(f["lt"], xv, yv, xu, yu)]
+    if f["bend"] >= 2:
+        mid, lb = z & 0xFFFF, (z >> 16) & 0xFF
+        if f["bend"] == 2:
+            bs, bt = (mid, yv), (mid, yu)
+        else:
+            bs, bt = (xv, mid), (xu, mid)
+        return [(f["ls"], xv, yv) + bs, (lb,) + bs + bt, (f["lt"],) + bt + (xu, yu)]
     if f["bend"] == 0:
         bx, by = xu, yv
     else:
@@ -63,14 +72,15 @@ def legs_of_edge(xv, yv, xu, yu, seg):
     return [(f["ls"], xv, yv, bx, by), (f["lt"], bx, by, xu, yu)]
 
 
-def recount_demand(d: Design, seg, base=None):
+def recount_demand(d: Design, seg, base=None, zmid=None):
     """Demand = base + sum over committed legs (independent recount from seg)."""
     dem = np.zeros((d.nlayers, d.ny, d.nx), np.int64) if base is None else base.astype(np.int64).copy()
     for n in range(d.num_nets):
         a, b = d.node_offset[n], d.node_offset[n + 1]
         for v in range(a + 1, b):
             u = a + d.parent[v]
-            for (l, xa, ya, xb, yb) in legs_of_edge(int(d.x[v]), int(d.y[v]), int(d.x[u]), int(d.y[u]), seg[v]):
+            z = -1 if zmid is None else int(zmid[v])
+            for (l, xa, ya, xb, yb) in legs_of_edge(int(d.x[v]), int(d.y[v]), int(d.x[u]), int(d.y[u]), seg[v], z):
                 if ya == yb:
                     for x in range(min(xa, xb), max(xa, xb)):
                         dem[l, ya, x] += 1
@@ -145,8 +155,10 @@ class PyCost:
         return int(sum(int(self.d.via_cost[k]) for k in range(lo, hi)))
 
 
-def route_cost(d: Design, pc: PyCost, n, segs):
-    """Cost of a complete assignment: wires + bend vias + node via hulls (None if illegal)."""
+def route_cost(d: Design, pc: PyCost, n, segs, zs=None):
+    """Cost of a complete assignment: wires + bend-point vias + node via hulls (None if illegal).
+
+    segs[i] / zs[i] = the route of local node i's edge (zs: Z middle, see legs_of_edge)."""
     a, b = d.node_offset[n], d.node_offset[n + 1]
     m = b - a
     L = d.nlayers
@@ -156,13 +168,15 @@ def route_cost(d: Design, pc: PyCost, n, segs):
     for i in range(1, m):
         v, u = a + i, a + int(d.parent[a + i])
         f = seg_fields(segs[i])
-        for (l, xa, ya, xb, yb) in legs_of_edge(int(d.x[v]), int(d.y[v]), int(d.x[u]), int(d.y[u]), segs[i]):
+        legs = legs_of_edge(int(d.x[v]), int(d.y[v]), int(d.x[u]), int(d.y[u]), segs[i],
+                            -1 if zs is None else zs[i])
+        for k, (l, xa, ya, xb, yb) in enumerate(legs):
             w = pc.wire(l, xa, ya, xb, yb)
             if w is None:
                 return None
             total += w
-        if not f["straight"]:
-            total += pc.via(f["ls"], f["lt"])
+            if k > 0:
+                total += pc.via(legs[k - 1][0], l)
         ui = int(d.parent[a + i])
         lo[i] = min(lo[i], f["ls"]); hi[i] = max(hi[i], f["ls"])
         lo[ui] = min(lo[ui], f["lt"]); hi[ui] = max(hi[ui], f["lt"])
@@ -172,7 +186,9 @@ def route_cost(d: Design, pc: PyCost, n, segs):
     return total
 
 
-def edge_options(d: Design, n, i):
+def edge_options(d: Design, n, i, hybrid=None):
+    """Every route of local node i's edge: [(seg, z)].  With hybrid=(t1, t2) and t1 <= HPWL <= t2
+    (bent edges only), every Z shape with both bend points strictly inside the box is added."""
     a = d.node_offset[n]
     v, u = a + i, a + int(d.parent[a + i])
     xv, yv, xu, yu = int(d.x[v]), int(d.y[v]), int(d.x[u]), int(d.y[u])
@@ -180,20 +196,27 @@ def edge_options(d: Design, n, i):
     H = [l for l in range(L) if d.dir[l] == 0]
     V = [l for l in range(L) if d.dir[l] == 1]
     if yv == yu:
-        return [make_seg(0, l, l, 1) for l in H]
+        return [(make_seg(0, l, l, 1), -1) for l in H]
     if xv == xu:
-        return [make_seg(0, l, l, 1) for l in V]
-    return [make_seg(0, ls, lt, 0) for ls in H for lt in V] + [make_seg(1, ls, lt, 0) for ls in V for lt in H]
+        return [(make_seg(0, l, l, 1), -1) for l in V]
+    out = [(make_seg(0, ls, lt, 0), -1) for ls in H for lt in V] + [(make_seg(1, ls, lt, 0), -1) for ls in V for lt in H]
+    h = abs(xv - xu) + abs(yv - yu)
+    if hybrid is not None and hybrid[0] <= h <= hybrid[1]:
+        for xm in range(min(xv, xu) + 1, max(xv, xu)):
+            out += [(make_seg(2, ls, lt, 0), xm | (lb << 16)) for ls in H for lb in V for lt in H]
+        for ym in range(min(yv, yu) + 1, max(yv, yu)):
+            out += [(make_seg(3, ls, lt, 0), ym | (lb << 16)) for ls in V for lb in H for lt in V]
+    return out
 
 
-def brute_force_min(d: Design, n, demand):
-    """Min over every per-edge (bend, ls, lt) assignment of the full route cost."""
+def brute_force_min(d: Design, n, demand, hybrid=None):
+    """Min over every per-edge route assignment of the full route cost."""
     pc = PyCost(d, demand)
     m = d.node_offset[n + 1] - d.node_offset[n]
-    opts = [edge_options(d, n, i) for i in range(1, m)]
+    opts = [edge_options(d, n, i, hybrid) for i in range(1, m)]
     best = None
     for combo in itertools.product(*opts):
-        c = route_cost(d, pc, n, [None] + list(combo))
+        c = route_cost(d, pc, n, [None] + [s for s, _ in combo], [None] + [z for _, z in combo])
         if c is not None and (best is None or c < best):
             best = c
     return best
