@@ -148,6 +148,32 @@ FGR_API fgr_status fgr_route_batch(fgr_grid* grid, const fgr_nets* nets, const i
                                    uint32_t* seg_out, uint32_t* net_cost, void* stream);
 
 /*
+ * fgr_set_pattern — candidate pattern set of later fgr_route_* / fgr_run_host_ex
+ * calls on this grid.  A bent tree edge v -> u whose two-pin half perimeter
+ * |x_v - x_u| + |y_v - y_u| lies in [hybrid_t1, hybrid_t2] takes the HYBRID
+ * L+Z patterns (§III-E/F, L758-1092: the two L shapes plus every Z
+ * shape whose two bend points lie strictly inside the edge's box; Eq. (8) path
+ * cost, Eqs. (9)-(14) candidate flows, Eq. (10) merge); every other edge takes
+ * the L patterns.  This is the paper's selection technique (§IV-D;
+ * FastGRH uses t1 = 100, t2 = 500).  hybrid_t1 > hybrid_t2 (the default,
+ * 1 > 0) = L patterns only (FastGRL).  A chosen Z is reported as seg bend 2
+ * (HVH: leg 1 horizontal on ls along row y_v to x = mid, leg 2 vertical on lb
+ * along column mid, leg 3 horizontal on lt along row y_u) or bend 3 (VHV: leg 1
+ * vertical on ls along column x_v to y = mid, leg 2 horizontal on lb along row
+ * mid, leg 3 vertical on lt along column x_u), with mid | lb << 16 in zmid_out.
+ * Tie order of equal costs: smallest ls, then the L shape, then Z by increasing
+ * mid, then smallest lb (R25).  Errors: INVALID (window outside
+ * [0, 65534] when enabled).  Host-only; takes effect at the next route call.
+ */
+FGR_API fgr_status fgr_set_pattern(fgr_grid* grid, int32_t hybrid_t1, int32_t hybrid_t2);
+
+/* fgr_route_batch with the Z middles: zmid_out [num_nodes] DEVICE out (may be NULL):
+ * for the listed nets' nodes, mid | lb << 16 of an edge routed as a Z shape
+ * (seg bend 2 or 3), -1 otherwise.  Same synchronisation and errors. */
+FGR_API fgr_status fgr_route_batch_ex(fgr_grid* grid, const fgr_nets* nets, const int32_t* net_ids, int32_t count,
+                                      uint32_t* seg_out, int32_t* zmid_out, uint32_t* net_cost, void* stream);
+
+/*
  * fgr_route_all — the pattern-routing stage: batches in sequence (PAPER.md
  * L504-512, Fig. 7), each routed on the demand left by all earlier batches.
  * order/batch_offset/num_batches as returned by fgr_plan for the same nets.
@@ -162,6 +188,13 @@ FGR_API fgr_status fgr_route_batch(fgr_grid* grid, const fgr_nets* nets, const i
 FGR_API fgr_status fgr_route_all(fgr_grid* grid, const fgr_nets* nets, const int32_t* order,
                                  const int32_t* batch_offset, int32_t num_batches, uint32_t* seg_out,
                                  uint32_t* net_cost, void* stream);
+
+/* fgr_route_all with the Z middles: zmid_out [num_nodes] DEVICE out (may be NULL),
+ * fully written: mid | lb << 16 for edges routed as a Z shape, -1 elsewhere.
+ * With hybrid patterns on, one host synchronisation per new (plan, window). */
+FGR_API fgr_status fgr_route_all_ex(fgr_grid* grid, const fgr_nets* nets, const int32_t* order,
+                                    const int32_t* batch_offset, int32_t num_batches, uint32_t* seg_out,
+                                    int32_t* zmid_out, uint32_t* net_cost, void* stream);
 
 /* The multi-GPU split rule fgr_route_all applies to one batch (host-only, no GPU):
  * the batch's `count` nets are ordered large nets first (`nlarge` of them); rank r
@@ -186,6 +219,11 @@ FGR_API fgr_status fgr_run_host(fgr_grid* grid, int32_t num_nets, int32_t num_no
                                 const int16_t* x, const int16_t* y, const int8_t* pin_lo, const int8_t* pin_hi,
                                 const int32_t* parent, uint32_t* seg_out, uint32_t* net_cost,
                                 int32_t* num_batches, void* stream);
+/* fgr_run_host with the Z middles (zmid_out [num_nodes] HOST out, may be NULL). */
+FGR_API fgr_status fgr_run_host_ex(fgr_grid* grid, int32_t num_nets, int32_t num_nodes, const int32_t* node_offset,
+                                   const int16_t* x, const int16_t* y, const int8_t* pin_lo, const int8_t* pin_hi,
+                                   const int32_t* parent, uint32_t* seg_out, int32_t* zmid_out, uint32_t* net_cost,
+                                   int32_t* num_batches, void* stream);
 
 /* Counters of the last fgr_route_all (for the byte model in DESIGN.md §5). */
 typedef struct {
@@ -201,13 +239,14 @@ FGR_API fgr_status fgr_get_stats(fgr_grid* grid, fgr_stats* out);
  * Per-kernel-class device timing (CUDA events recorded on the caller's stream
  * around every launch of the class while enabled).  Classes:
  *   0 refresh, 1 dp_small (warp per net), 2 dp_large (CTA per net), 3 commit,
- *   4 plan_preprocess, 5 plan_sort (CUB), 6 plan_color, 7 plan_other, 8 exchange (NCCL)
+ *   4 plan_preprocess, 5 plan_sort (CUB), 6 plan_color, 7 plan_other, 8 exchange (NCCL),
+ *   9 hybrid (Z transfer matrices)
  * fgr_profile_read synchronises, then returns the summed milliseconds and the
  * number of launches per class since the last enable, and clears the counters.
  */
-#define FGR_PROF_CLASSES 9
+#define FGR_PROF_CLASSES 10
 FGR_API fgr_status fgr_profile_enable(fgr_grid* grid, int enable);
-FGR_API fgr_status fgr_profile_read(fgr_grid* grid, double* ms /* [9] */, int64_t* launches /* [9] */);
+FGR_API fgr_status fgr_profile_read(fgr_grid* grid, double* ms /* [10] */, int64_t* launches /* [10] */);
 
 #ifdef __cplusplus
 }

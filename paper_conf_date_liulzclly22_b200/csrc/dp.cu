@@ -153,7 +153,7 @@ struct Out {
     int list_base;
 };
 
-// Per-lane constants of the group lane that owns layer `gl` (= lo in span_rows, = lt in edge_table).
+// Per-lane constants of the group lane that owns layer `gl` (= lo in the K rows, = lt in the edge step).
 template <int LT>
 struct LaneConst {
     uint32_t vme[LT];      // V(min(l, gl), max(l, gl)): via stack between layer l and this lane's layer
@@ -221,106 +221,21 @@ __device__ __forceinline__ void gather_task(const GridView& g, const Tabs& t, in
 }
 
 // ------------------------------------------------------------- DP steps (one group of LT lanes)
-// F_v(lo, hi) for the group lane lo, reduced to suffix minima R(lo, b) of the packed keys.
-template <int LT, bool CTA>
-__device__ __forceinline__ void span_rows(const LaneConst<LT>& c, const Tabs& t, const WScr& w, int v, int lo, bool act) {
-    if (!act) return;
-    uint32_t acc[LT];
-#pragma unroll
-    for (int hi = 0; hi < LT; hi++) acc[hi] = hi >= lo ? c.vme[hi] : FGR_INF;   // lo == this lane's layer
-    auto add_child = [&](int ch) {
-        const uint32_t* Ec = t.E + (size_t)ch * LT;
-        uint32_t run = FGR_INF;
-#pragma unroll
-        for (int hi = 0; hi < LT; hi++) {
-            const uint32_t e = Ec[hi];
-            if (hi >= lo) { run = min(run, e); acc[hi] = sat_add(acc[hi], run); }
-        }
-    };
-    if (CTA) {
-        const int k1 = t.cstart[v + 1];
-        for (int k = t.cstart[v]; k < k1; k++) add_child(t.clist[k]);
-    } else {
-        uint32_t cm = t.aux[v];
-        while (cm) {
-            const int ch = __ffs(cm) - 1;
-            cm &= cm - 1;
-            add_child(ch);
-        }
-    }
-    unsigned long long run = ~0ull;
-#pragma unroll
-    for (int hi = LT - 1; hi >= 0; hi--)
-        if (hi >= lo) {
-            const unsigned long long key = ((unsigned long long)acc[hi] << 8) | (unsigned)(lo << 4) | (unsigned)hi;
-            run = key < run ? key : run;
-            w.R[lo * LT + hi] = run;
-        }
+// Bend field of a chosen route: 0/1 = the L shapes (bend 0 when lt is vertical); a
+// departure and arrival layer of the same direction on a bent edge is a Z shape of a
+// hybrid edge: 2 = HVH, 3 = VHV (§III-E).
+__device__ __forceinline__ uint32_t seg_bend(int dls, int dlt, bool straight) {
+    if (straight) return 0u;
+    if (dls == dlt) return dls == 0 ? 2u : 3u;
+    return dlt == 1 ? 0u : 1u;
 }
 
-// Eq. (2) per ls: min over lo <= a = min(ls, pin_lo) of R(lo, b), b = max(ls, pin_hi);
-// the packed key carries the (value, lo, hi) lexicographic tie-break of R11.
-template <int LT>
-__device__ __forceinline__ void node_table(const Tabs& t, const WScr& w, int v, int ls, bool act) {
-    if (!act) return;
-    int a = ls, b = ls;
-    const int plo = t.plo[v], phi = t.phi[v];
-    if (plo >= 0) { a = min(a, plo); b = max(b, phi); }
-    unsigned long long best = ~0ull;
-#pragma unroll
-    for (int lo = 0; lo < LT; lo++)
-        if (lo <= a) {
-            const unsigned long long k = w.R[lo * LT + b];
-            best = k < best ? k : best;
-        }
-    w.B[ls] = (uint32_t)(best >> 8);
-    t.recB[(size_t)v * LT + ls] = (uint8_t)(best & 0xFF);
-}
-
-// Eqs. (1),(3),(5)-(7): E_v(lt) = min_ls [B_v(ls) + leg1(ls) + V(ls,lt) + leg2(lt)], lane = lt.
-template <int LT>
-__device__ __forceinline__ void edge_table(const LaneConst<LT>& c, const Tabs& t, const WScr& w, int v, int lt,
-                                           int nH, int nV, bool act) {
-    if (!act) return;
-    const int u = t.par[v];
-    const int xv = t.x[v], yv = t.y[v], xu = t.x[u], yu = t.y[u];
-    uint32_t best = FGR_INF;
-    int bls = lt;
-    if (yv == yu || xv == xu) {                   // straight: one leg on ls = lt (R7)
-        const int de = (yv == yu) ? 0 : 1;
-        if (c.my_dir == de) {
-            const uint32_t leg = de == 0 ? t.legH[(size_t)v * 2 * nH + c.my_slot] : t.legV[(size_t)v * 2 * nV + c.my_slot];
-            best = sat_add(w.B[lt], leg);
-        }
-    } else {
-        // bend 0 (lt vertical): leg 1 H on row y_v, leg 2 V on col x_u;
-        // bend 1 (lt horizontal): leg 1 V on col x_v, leg 2 H on row y_u
-        const bool b0 = c.my_dir == 1;
-        const uint32_t leg2 = b0 ? t.legV[((size_t)v * 2 + 1) * nV + c.my_slot] : t.legH[((size_t)v * 2 + 1) * nH + c.my_slot];
-        const uint32_t* l1 = b0 ? t.legH + (size_t)v * 2 * nH : t.legV + (size_t)v * 2 * nV;
-        const uint32_t opp = b0 ? c.hmask : ~c.hmask;
-        int s = 0;
-#pragma unroll
-        for (int ls = 0; ls < LT; ls++)
-            if ((opp >> ls) & 1u) {
-                const uint32_t via = c.vme[ls];   // lt == this lane's layer
-                const uint32_t cst = sat_add(sat_add(sat_add(w.B[ls], l1[s]), via), leg2);
-                if (cst < best) { best = cst; bls = ls; }
-                s++;
-            }
-    }
-    t.E[(size_t)v * LT + lt] = best;
-    t.recE[(size_t)v * LT + lt] = (uint8_t)bls;
-}
-
-// Generalised Eq. (4): candidate of lane lo for the min over spans containing the root pin span.
-template <int LT>
-__device__ __forceinline__ unsigned long long root_cand(const Tabs& t, const WScr& w, int lo, bool act) {
-    if (!act) return ~0ull;
-    const int plo = t.plo[0], phi = t.phi[0];
-    const int a = plo >= 0 ? plo : LT - 1;     // Steiner root: any span
-    const int b = plo >= 0 ? phi : 0;
-    return lo <= a ? w.R[lo * LT + max(lo, b)] : ~0ull;
+// Z argmin (mid | lb << 16) of a chosen Z route of global node gv, or 0 for an L shape.
+__device__ __forceinline__ uint32_t hyb_z(const HybView& hy, int gv, uint32_t seg, int L) {
+    if ((seg & 0xFF) < 2 || !hy.net) return 0u;
+    const int s = hy.slot[gv];
+    const int ls = (seg >> 8) & 0xFF, lt = (seg >> 16) & 0xFF;
+    return hy.A[((size_t)s * L + lt) * L + ls];
 }
 
 // S5: child layer = smallest l in the parent's span minimising E_v(l) (R11).
@@ -338,7 +253,7 @@ __device__ __forceinline__ uint32_t backtrack_node(const Hdr* h, const Tabs& t, 
     const int ls = t.recE[(size_t)v * LT + lt];
     t.span[v] = t.recB[(size_t)v * LT + ls];
     const bool straight = (t.x[v] == t.x[u]) || (t.y[v] == t.y[u]);
-    const uint32_t bend = straight ? 0u : (h->dir[lt] == 1 ? 0u : 1u);
+    const uint32_t bend = seg_bend(h->dir[ls], h->dir[lt], straight);
     return bend | ((uint32_t)ls << 8) | ((uint32_t)lt << 16) | ((uint32_t)straight << 24);
 }
 
@@ -354,11 +269,25 @@ __device__ __forceinline__ void commit_leg(const GridView& g, const DirView& d, 
     g.dline[d.line_base + line] = 1;
 }
 
-__device__ __forceinline__ void commit_edge(const GridView& g, const Hdr* h, int xv, int yv, int xu, int yu, uint32_t seg) {
+__device__ __forceinline__ void commit_edge(const GridView& g, const Hdr* h, int xv, int yv, int xu, int yu, uint32_t seg,
+                                            uint32_t z) {
     const int bend = seg & 0xFF, ls = (seg >> 8) & 0xFF, lt = (seg >> 16) & 0xFF, straight = (seg >> 24) & 0xFF;
     if (straight) {
         if (yv == yu) commit_leg(g, g.h, yv, min(xv, xu), max(xv, xu), h->slot[lt]);
         else commit_leg(g, g.v, xv, min(yv, yu), max(yv, yu), h->slot[lt]);
+        return;
+    }
+    if (bend >= 2) {   // Z shape (hybrid edge): three legs through Bs and Bt, middle layer lb
+        const int mid = (int)(z & 0xFFFF), lb = (int)((z >> 16) & 0xFF);
+        if (bend == 2) {   // HVH: row y_v to xm (ls), column xm (lb), row y_u from xm (lt)
+            commit_leg(g, g.h, yv, min(xv, mid), max(xv, mid), h->slot[ls]);
+            commit_leg(g, g.v, mid, min(yv, yu), max(yv, yu), h->slot[lb]);
+            commit_leg(g, g.h, yu, min(mid, xu), max(mid, xu), h->slot[lt]);
+        } else {           // VHV: column x_v to ym (ls), row ym (lb), column x_u from ym (lt)
+            commit_leg(g, g.v, xv, min(yv, mid), max(yv, mid), h->slot[ls]);
+            commit_leg(g, g.h, mid, min(xv, xu), max(xv, xu), h->slot[lb]);
+            commit_leg(g, g.v, xu, min(mid, yu), max(mid, yu), h->slot[lt]);
+        }
         return;
     }
     if (bend == 0) {   // H on row y_v (layer ls), V on col x_u (layer lt)
@@ -393,7 +322,8 @@ __device__ __forceinline__ unsigned long long tree_min(unsigned long long (&k)[N
 template <int LT>
 __device__ __forceinline__ unsigned long long node_step_group(const Hdr* h, const LaneConst<LT>& c, const Tabs& t,
                                                               const WScr& w, int v, bool act, bool is_root, int gl,
-                                                              int gbase, int nH, int nV, uint32_t opp) {
+                                                              int gbase, int nH, int nV, uint32_t opp,
+                                                              const uint32_t* hm) {
     const uint32_t cm = act ? t.aux[v] : 0u;
     const int hc = cm ? 31 - __clz(cm) : -1;
     const uint32_t lm = hc >= 0 ? (cm & ~(1u << hc)) : 0u;
@@ -477,7 +407,13 @@ __device__ __forceinline__ unsigned long long node_step_group(const Hdr* h, cons
     const int xv = t.x[v], yv = t.y[v], xu = t.x[u], yu = t.y[u];
     uint32_t best = FGR_INF;
     int bls = gl;
-    if (yv == yu || xv == xu) {                   // straight: one leg on ls = lt (R7)
+    if (hm) {                                     // hybrid edge: E_v(lt) = min_ls [B_v(ls) + M_e(ls, lt)]
+#pragma unroll
+        for (int l = 0; l < LT; l++) {
+            const uint32_t cst = sat_add(Bl[l], hm[l]);
+            if (cst < best) { best = cst; bls = l; }
+        }
+    } else if (yv == yu || xv == xu) {            // straight: one leg on ls = lt (R7)
         const int de = (yv == yu) ? 0 : 1;
         if (c.my_dir == de) {
             const uint32_t leg = de == 0 ? t.legH[(size_t)v * 2 * nH + c.my_slot] : t.legV[(size_t)v * 2 * nV + c.my_slot];
@@ -528,7 +464,7 @@ struct Flat {
 
 template <int LT, int kMC>
 __global__ void __launch_bounds__(32 * kGroupWarps) k_dp_group(GridView g, NetsView nv, const int32_t* __restrict__ list,
-                                                               int count, Out o, int commit) {
+                                                               int count, Out o, int commit, HybView hy) {
     constexpr int G = groups_of(LT);
     extern __shared__ __align__(16) unsigned char smem[];
     Hdr* h = reinterpret_cast<Hdr*>(smem);
@@ -547,18 +483,24 @@ __global__ void __launch_bounds__(32 * kGroupWarps) k_dp_group(GridView g, NetsV
     LaneConst<LT> c;
     c.load(h, gl);
     // nets of the G groups
-    int net_l = -1, a0_l = 0, m_l = 0;
+    int net_l = -1, a0_l = 0, m_l = 0, hn_l = -1;
     if (lane < G && idx0 + lane < count) {
         net_l = list[idx0 + lane];
         a0_l = nv.off[net_l];
         m_l = nv.off[net_l + 1] - a0_l;
+        if (hy.net) hn_l = hy.net[net_l];
     }
     int mq[G], aq[G];
 #pragma unroll
     for (int q = 0; q < G; q++) { mq[q] = __shfl_sync(0xffffffffu, m_l, q); aq[q] = __shfl_sync(0xffffffffu, a0_l, q); }
-    int my_m = 0;
+    int my_m = 0, my_a = 0, my_hn = -1;
 #pragma unroll
-    for (int q = 0; q < G; q++) my_m = (gi == q) ? mq[q] : my_m;
+    for (int q = 0; q < G; q++) {
+        const int hq = __shfl_sync(0xffffffffu, hn_l, q);
+        my_m = (gi == q) ? mq[q] : my_m;
+        my_a = (gi == q) ? aq[q] : my_a;
+        my_hn = (gi == q) ? hq : my_hn;
+    }
     Flat<G> nodes;
     nodes.build(mq);
     // node data, zeroed child masks
@@ -600,13 +542,18 @@ __global__ void __launch_bounds__(32 * kGroupWarps) k_dp_group(GridView g, NetsV
     const int gbase = (gi < G ? gi : 0) * LT;
     for (int k = 0; k + 1 < maxm; k++) {
         const int v = my_m - 1 - k;
-        node_step_group<LT>(h, c, t, w, v, glane && v >= 1, false, gl, gbase, nH, nV, opp);
+        const uint32_t* hm = nullptr;   // hybrid edge: its transfer matrix column for lt = gl
+        if (my_hn >= 0 && glane && v >= 1) {
+            const int hs = hy.slot[my_a + v];
+            if (hs >= 0) hm = hy.M + ((size_t)hs * LT + gl) * LT;
+        }
+        node_step_group<LT>(h, c, t, w, v, glane && v >= 1, false, gl, gbase, nH, nV, opp, hm);
         __syncwarp();
     }
     // root (generalised Eq. (4))
     {
         const bool act = glane && my_m >= 2;
-        const unsigned long long rk = node_step_group<LT>(h, c, t, w, 0, act, true, gl, gbase, nH, nV, opp);
+        const unsigned long long rk = node_step_group<LT>(h, c, t, w, 0, act, true, gl, gbase, nH, nV, opp, nullptr);
         if (act && gl == 0) { t.span[0] = (uint8_t)(rk & 0xFF); rootkey = rk; }
         __syncwarp();
     }
@@ -675,7 +622,7 @@ __global__ void __launch_bounds__(32 * kGroupWarps) k_dp_group(GridView g, NetsV
         else o.seg[a + i] = s;
         if (commit && i > 0) {
             const int u = tt.par[i];
-            commit_edge(g, h, tt.x[i], tt.y[i], tt.x[u], tt.y[u], s);
+            commit_edge(g, h, tt.x[i], tt.y[i], tt.x[u], tt.y[u], s, hyb_z(hy, a + i, s, LT));
         }
     }
     if (glane && gl == 0 && my_m >= 1) {
@@ -888,7 +835,7 @@ __device__ __forceinline__ void build_G(const LaneConst<LT>& c, const Tabs& t, c
 template <int LT>
 __device__ __forceinline__ uint32_t path_node(const LaneConst<LT>& c, const Tabs& t, const WScr& w, int v, uint32_t Eprev,
                                               bool has_prev, bool light, int gl, int gbase, unsigned gmask, int nH,
-                                              int nV, uint32_t opp, bool store_E) {
+                                              int nV, uint32_t opp, bool store_E, const uint32_t* hm) {
     const int plo = t.plo[v], phi = t.phi[v];
     const int ls = gl;
     int a0 = ls, b0 = ls;
@@ -940,7 +887,13 @@ __device__ __forceinline__ uint32_t path_node(const LaneConst<LT>& c, const Tabs
     uint32_t Bl[LT];
 #pragma unroll
     for (int l = 0; l < LT; l++) Bl[l] = __shfl_sync(gmask, Bv, gbase + l);
-    if (yv == yu || xv == xu) {
+    if (hm) {                                     // hybrid edge: min-plus with the precomputed M_e
+#pragma unroll
+        for (int l = 0; l < LT; l++) {
+            const uint32_t cst = sat_add(Bl[l], hm[l]);
+            if (cst < best) { best = cst; bls = l; }
+        }
+    } else if (yv == yu || xv == xu) {
         const int de = (yv == yu) ? 0 : 1;
         if (c.my_dir == de) {
             const uint32_t leg = de == 0 ? t.legH[(size_t)v * 2 * nH + c.my_slot] : t.legV[(size_t)v * 2 * nV + c.my_slot];
@@ -969,7 +922,8 @@ __device__ __forceinline__ uint32_t path_node(const LaneConst<LT>& c, const Tabs
 // Exact: min-plus distributes over the saturating sums.  Lane lt writes column lt.
 template <int LT>
 __device__ __forceinline__ void build_M(const Hdr* h, const LaneConst<LT>& c, const Tabs& t, const WScr& w, int v,
-                                        bool light, int gl, int nH, int nV, uint32_t opp, uint32_t* col) {
+                                        bool light, int gl, int nH, int nV, uint32_t opp, uint32_t* col,
+                                        const uint32_t* hm) {
     const int plo = t.plo[v], phi = t.phi[v];
     const int lt = gl;
     const int u = t.par[v];
@@ -987,7 +941,16 @@ __device__ __forceinline__ void build_M(const Hdr* h, const LaneConst<LT>& c, co
     }
     for (int l = 0; l < LT; l++) {
         uint32_t best = FGR_INF;
-        if (straight) {
+        if (hm) {   // hybrid edge: W_v(ls, lt) = M_e(ls, lt)
+#pragma unroll
+            for (int ls = 0; ls < LT; ls++) {
+                int a = ls, b = ls;
+                if (plo >= 0) { a = min(a, plo); b = max(b, phi); }
+                a = min(a, l); b = max(b, l);
+                const uint32_t cv = light ? (uint32_t)(w.R[a * LT + b] >> 8) : h->viapre[b] - h->viapre[a];
+                best = min(best, sat_add(cv, hm[ls]));
+            }
+        } else if (straight) {
             if (legS != FGR_INF) {
                 int a = lt, b = lt;
                 if (plo >= 0) { a = min(a, plo); b = max(b, phi); }
@@ -1023,7 +986,8 @@ __device__ __forceinline__ void build_M(const Hdr* h, const LaneConst<LT>& c, co
 
 template <int LT>
 __global__ void __launch_bounds__(32 * kLargeWarps, 1) k_dp_large(GridView g, NetsView nv, const int32_t* __restrict__ list,
-                                                                  int count, Out o, int commit, Prep prep) {
+                                                                  int count, Out o, int commit, Prep prep,
+                                                                  HybView hy) {
     constexpr int G = 1;   // one lane group per warp: a path walk never shares its warp's issue slots
     extern __shared__ __align__(16) unsigned char smem[];
     Hdr* h = reinterpret_cast<Hdr*>(smem);
@@ -1046,6 +1010,13 @@ __global__ void __launch_bounds__(32 * kLargeWarps, 1) k_dp_large(GridView g, Ne
     const int net = list[idx];
     const int a0 = nv.off[net];
     const int m = nv.off[net + 1] - a0;
+    const int hnet = hy.net ? hy.net[net] : -1;
+    // hybrid edge of node v: its transfer matrix column for lt = gl (nullptr for an L edge)
+    auto hmat = [&](int v) -> const uint32_t* {
+        if (hnet < 0) return nullptr;
+        const int hs = hy.slot[a0 + v];
+        return hs >= 0 ? hy.M + ((size_t)hs * LT + gl) * LT : nullptr;
+    };
     unsigned char* base = smem + a16(sizeof(Hdr));
     const WScr w = carve_wscr(base + ((size_t)warp * G + (gi < G ? gi : 0)) * wscr_bytes(LT), LT);
     const Tabs t = carve_tabs(base + (size_t)kLargeWarps * G * wscr_bytes(LT), m, LT, nH, nV, true);
@@ -1168,7 +1139,7 @@ __global__ void __launch_bounds__(32 * kLargeWarps, 1) k_dp_large(GridView g, Ne
                 }
                 const bool light = (t.cstart[v + 1] - t.cstart[v]) > 1;
                 if (light) build_G<LT>(c, t, w, v, gl, gmask);
-                Eprev = path_node<LT>(c, t, w, v, Eprev, k > 0, light, gl, gbase, gmask, nH, nV, opp, true);
+                Eprev = path_node<LT>(c, t, w, v, Eprev, k > 0, light, gl, gbase, gmask, nH, nV, opp, true, hmat(v));
                 __syncwarp(gmask);
                 __threadfence_block();
 #ifdef FGR_TIMING
@@ -1194,7 +1165,8 @@ __global__ void __launch_bounds__(32 * kLargeWarps, 1) k_dp_large(GridView g, Ne
                 for (;;) {
                     const bool light = (t.cstart[v + 1] - t.cstart[v]) > 1;
                     if (light) build_G<LT>(c, t, w, v, gl, gmask);
-                    const uint32_t Ev = path_node<LT>(c, t, w, v, Eprev, has_prev, light, gl, gbase, gmask, nH, nV, opp, true);
+                    const uint32_t Ev = path_node<LT>(c, t, w, v, Eprev, has_prev, light, gl, gbase, gmask, nH, nV, opp, true,
+                                                      hmat(v));
                     if (v == tp) {   // only path tops are read by other warps (as light children)
                         __syncwarp(gmask);
                         __threadfence_block();
@@ -1227,7 +1199,7 @@ __global__ void __launch_bounds__(32 * kLargeWarps, 1) k_dp_large(GridView g, Ne
                 if (gl == 0) old = atomicCAS(&sstate[sl], k * 4, k * 4 + 1);
                 old = __shfl_sync(gmask, old, gbase);
                 if (old != k * 4) continue;
-                build_M<LT>(h, c, t, w, v, light, gl, nH, nV, opp, mslots + (size_t)sl * LT * MStride<LT>::v);
+                build_M<LT>(h, c, t, w, v, light, gl, nH, nV, opp, mslots + (size_t)sl * LT * MStride<LT>::v, hmat(v));
                 __syncwarp(gmask);
                 __threadfence_block();
                 if (gl == 0) *(volatile int*)&sstate[sl] = k * 4 + 2;
@@ -1256,7 +1228,7 @@ __global__ void __launch_bounds__(32 * kLargeWarps, 1) k_dp_large(GridView g, Ne
                 const uint32_t Eh = t.E[(size_t)t.rp[k - 1] * LT + gl];
                 const bool light = (t.cstart[v + 1] - t.cstart[v]) > 1;
                 if (light) build_G<LT>(c, t, w, v, gl, gmask);
-                path_node<LT>(c, t, w, v, Eh, true, light, gl, gbase, gmask, nH, nV, opp, false);
+                path_node<LT>(c, t, w, v, Eh, true, light, gl, gbase, gmask, nH, nV, opp, false, hmat(v));
             }
         }
     }
@@ -1304,7 +1276,7 @@ __global__ void __launch_bounds__(32 * kLargeWarps, 1) k_dp_large(GridView g, Ne
                     const int ls = t.recE[(size_t)v * LT + lt];
                     t.span[v] = t.recB[(size_t)v * LT + ls];
                     const bool straight = (t.x[v] == t.x[u]) || (t.y[v] == t.y[u]);
-                    const uint32_t bend = straight ? 0u : (h->dir[lt] == 1 ? 0u : 1u);
+                    const uint32_t bend = seg_bend(h->dir[ls], h->dir[lt], straight);
                     const uint32_t sg = bend | ((uint32_t)ls << 8) | ((uint32_t)lt << 16) | ((uint32_t)straight << 24);
                     t.legH[(size_t)v * 2 * nH] = sg;   // the leg costs are dead now: keep the route (shared memory only)
                 }
@@ -1333,7 +1305,7 @@ __global__ void __launch_bounds__(32 * kLargeWarps, 1) k_dp_large(GridView g, Ne
         else o.seg[a0 + i] = s;
         if (commit) {
             const int u = t.par[i];
-            commit_edge(g, h, t.x[i], t.y[i], t.x[u], t.y[u], s);
+            commit_edge(g, h, t.x[i], t.y[i], t.x[u], t.y[u], s, hyb_z(hy, a0 + i, s, LT));
         }
     }
 #ifdef FGR_TIMING
@@ -1403,7 +1375,7 @@ __device__ __forceinline__ void leg_cost_col(const DirView& d, int line, int a, 
 
 template <int LT>
 __global__ void __launch_bounds__(kTwoThreads) k_dp_two(GridView g, NetsView nv, const int32_t* __restrict__ list,
-                                                        int count, Out o, int commit) {
+                                                        int count, Out o, int commit, HybView hy) {
     __shared__ Hdr hs;
     __shared__ uint32_t legs[4 * 16 * kTwoThreads];   // [leg][slot][thread]
     init_hdr(&hs, g);
@@ -1426,6 +1398,7 @@ __global__ void __launch_bounds__(kTwoThreads) k_dp_two(GridView g, NetsView nv,
         return;
     }
     const int x0 = nv.x[a0], y0 = nv.y[a0], x1 = nv.x[a0 + 1], y1 = nv.y[a0 + 1];
+    const int hslot = hy.net ? hy.net[net] : -1;   // a 2-node net's first slot is its only edge
     const int plo0 = nv.plo[a0], phi0 = nv.phi[a0], plo1 = nv.plo[a0 + 1], phi1 = nv.phi[a0 + 1];
     const bool sh = (y0 == y1), sv = (x0 == x1), straight = sh || sv;
     uint32_t* col = legs + tid;
@@ -1475,7 +1448,14 @@ __global__ void __launch_bounds__(kTwoThreads) k_dp_two(GridView g, NetsView nv,
         const bool hlt = (hmask >> lt) & 1u;
         uint32_t best = FGR_INF;
         int bls = lt;
-        if (straight) {
+        if (hslot >= 0) {   // hybrid edge: min-plus with the precomputed transfer matrix
+            const uint32_t* hm = hy.M + ((size_t)hslot * LT + lt) * LT;
+#pragma unroll
+            for (int ls = 0; ls < LT; ls++) {
+                const uint32_t cst = sat_add(Bv[ls], hm[ls]);
+                if (cst < best) { best = cst; bls = ls; }
+            }
+        } else if (straight) {
             if ((hlt ? 0 : 1) == de) best = sat_add(Bv[lt], c1[lt]);
         } else {
 #pragma unroll
@@ -1522,7 +1502,7 @@ __global__ void __launch_bounds__(kTwoThreads) k_dp_two(GridView g, NetsView nv,
     for (int l = 0; l < LT; l++)
         if (l >= lo && l <= hi && E[l] < be) { be = E[l]; lt = l; ls = recE[l]; }
     (void)recB;
-    const uint32_t bend = straight ? 0u : (((hmask >> lt) & 1u) ? 1u : 0u);
+    const uint32_t bend = seg_bend(((hmask >> ls) & 1u) ? 0 : 1, ((hmask >> lt) & 1u) ? 0 : 1, straight);
     const uint32_t sg = bend | ((uint32_t)ls << 8) | ((uint32_t)lt << 16) | ((uint32_t)(straight ? 1 : 0) << 24);
     if (o.rec_seg) {
         uint32_t* rs = o.rec_seg + o.rec_off[o.list_base + idx];
@@ -1532,13 +1512,13 @@ __global__ void __launch_bounds__(kTwoThreads) k_dp_two(GridView g, NetsView nv,
         o.seg[a0] = 0xFFFFFFFFu; o.seg[a0 + 1] = sg;
         o.cost[net] = (uint32_t)(rk >> 8);
     }
-    if (commit) commit_edge(g, &hs, x1, y1, x0, y0, sg);
+    if (commit) commit_edge(g, &hs, x1, y1, x0, y0, sg, hyb_z(hy, a0 + 1, sg, LT));
 }
 
 // Commit from route records (multi-GPU: after the exchange every rank commits every net).
 __global__ void __launch_bounds__(256) k_commit_records(GridView g, NetsView nv, const int32_t* __restrict__ list, int count,
                                                         const uint32_t* __restrict__ rec_seg,
-                                                        const int32_t* __restrict__ rec_off, int list_base) {
+                                                        const int32_t* __restrict__ rec_off, int list_base, HybView hy) {
     __shared__ Hdr hs;
     init_hdr(&hs, g);
     __syncthreads();
@@ -1550,7 +1530,7 @@ __global__ void __launch_bounds__(256) k_commit_records(GridView g, NetsView nv,
         const uint32_t* rs = rec_seg + rec_off[list_base + idx];
         for (int i = 1 + lane_id(); i < m; i += 32) {
             const int u = nv.par[a0 + i];
-            commit_edge(g, &hs, nv.x[a0 + i], nv.y[a0 + i], nv.x[a0 + u], nv.y[a0 + u], rs[i]);
+            commit_edge(g, &hs, nv.x[a0 + i], nv.y[a0 + i], nv.x[a0 + u], nv.y[a0 + u], rs[i], hyb_z(hy, a0 + i, rs[i], g.L));
         }
     }
 }
@@ -1591,6 +1571,7 @@ cudaError_t launch_lt(fgr_grid* g, cudaStream_t st, const NetsView& nv, const in
         configured = true;
     }
     const GridView& v = g->view;
+    const HybView hyv = g->hy.view();
     // The four size classes of one batch are independent: each non-empty class gets its
     // own stream (forked from and joined back into the caller's stream).
     const int cls_n[4] = {nlarge, nmidL, nmidS, ntwo};
@@ -1625,22 +1606,22 @@ cudaError_t launch_lt(fgr_grid* g, cudaStream_t st, const NetsView& nv, const in
                 at[0].val.programmaticStreamSerializationAllowed = 1;
                 cfg.attrs = at;
                 cfg.numAttrs = 1;
-                e = cudaLaunchKernelEx(&cfg, k_dp_large<LT>, v, nv, l, n, os, commit ? 1 : 0, prep);
+                e = cudaLaunchKernelEx(&cfg, k_dp_large<LT>, v, nv, l, n, os, commit ? 1 : 0, prep, hyv);
                 if (e != cudaSuccess) return e;
             }
             else if (k == 1) {
                 const int per_cta = kGroupWarps * groups_of(LT);
                 k_dp_group<LT, FGR_SMALL_NET><<<(n + per_cta - 1) / per_cta, 32 * kGroupWarps,
                                                  smem_group(LT, g->nH, g->nV, FGR_SMALL_NET), sk[k]>>>(v, nv, l, n, os,
-                                                                                                      commit ? 1 : 0);
+                                                                                                      commit ? 1 : 0, hyv);
             } else if (k == 2) {
                 const int per_cta = kGroupWarps * groups_of(LT);
                 k_dp_group<LT, FGR_MID_NET><<<(n + per_cta - 1) / per_cta, 32 * kGroupWarps,
                                                smem_group(LT, g->nH, g->nV, FGR_MID_NET), sk[k]>>>(v, nv, l, n, os,
-                                                                                                  commit ? 1 : 0);
+                                                                                                  commit ? 1 : 0, hyv);
             } else {
                 k_dp_two<LT><<<(n + kTwoThreads - 1) / kTwoThreads, kTwoThreads, 0, sk[k]>>>(v, nv, l, n, os,
-                                                                                              commit ? 1 : 0);
+                                                                                              commit ? 1 : 0, hyv);
             }
             fgr_prof_end(g, ps, sk[k]);
             g->stats.kernel_launches++;
@@ -1718,7 +1699,7 @@ cudaError_t fgr_launch_commit(fgr_grid* g, cudaStream_t st, const NetsView& nv, 
     if (blocks > g->num_sms * 8) blocks = g->num_sms * 8;
     if (blocks < 1) blocks = 1;
     const int ps = fgr_prof_begin(g, PROF_COMMIT, st);
-    k_commit_records<<<blocks, 256, 0, st>>>(v, nv, list, count, rec_seg, rec_off, list_base);
+    k_commit_records<<<blocks, 256, 0, st>>>(v, nv, list, count, rec_seg, rec_off, list_base, g->hy.view());
     fgr_prof_end(g, ps, st);
     g->stats.kernel_launches++;
     return cudaGetLastError();

@@ -21,6 +21,7 @@
 #include <stdint.h>
 
 #include <string>
+#include <vector>
 
 #include "fastgr.h"
 
@@ -83,6 +84,37 @@ struct Prep {
     const uint16_t* pq;    // path queue (path tops, deepest first)
     const int32_t* npaths; // [num_nets]
     const uint16_t* rpos;  // index along the root path (0xFFFF off it)
+};
+
+// Hybrid L+Z tables of the current route call (hybrid.cu).  Slots number the hybrid
+// edges; M[s][lt][ls] is the edge's transfer cost from layer ls at the child to lt at
+// the parent (legs + bend vias, FGR_INF if no candidate), A[s][lt][ls] its Z argmin
+// (mid | lb << 16) or 0xFFFFFFFF for the L shape.
+struct HybView {
+    const int32_t* net;    // [num_nets] first slot of the net, -1 = no hybrid edge (NULL = L only)
+    const int32_t* slot;   // [num_nodes] slot of the node's edge, -1 = L edge (valid in nets with net >= 0)
+    const uint32_t* M;
+    const uint32_t* A;
+};
+
+struct HybState {
+    bool active = false;
+    int nslots = 0;
+    int32_t* net = nullptr;
+    int32_t* slot = nullptr;
+    int32_t* list = nullptr;   // [nslots] global child node of the edge
+    int32_t* par = nullptr;    // [nslots] global parent node
+    uint32_t* M = nullptr;
+    uint32_t* A = nullptr;
+    std::vector<int> boff;     // host: slot offsets per batch
+    bool cached = false;       // tables valid for (key_exec, key_t1, key_t2) of fgr_route_all
+    const int32_t* key_exec = nullptr;
+    int key_t1 = 0, key_t2 = 0;
+    HybView view() const {
+        HybView v;
+        v.net = active ? net : nullptr; v.slot = slot; v.M = M; v.A = A;
+        return v;
+    }
 };
 
 struct PlanCache {
@@ -152,13 +184,17 @@ struct fgr_grid {
     Profiler prof;
     cudaStream_t side[3] = {nullptr, nullptr, nullptr};   // size classes of one batch run side by side
     cudaEvent_t ev_fork = nullptr, ev_join[3] = {nullptr, nullptr, nullptr};
+    // hybrid L+Z pattern routing (fgr_set_pattern): edges with t1 <= HPWL <= t2; t1 > t2 = L only
+    int hyb_t1 = 1, hyb_t2 = 0;
+    HybState hy;
+    Scratch s_hyb[3];
 };
 
 // Profiling brackets around a launch (no-ops unless fgr_profile_enable(grid, 1)).
 int fgr_prof_begin(fgr_grid* g, int cls, cudaStream_t st);
 void fgr_prof_end(fgr_grid* g, int slot, cudaStream_t st);
 enum { PROF_REFRESH = 0, PROF_DP_SMALL, PROF_DP_LARGE, PROF_COMMIT, PROF_PRE, PROF_SORT, PROF_COLOR, PROF_PLAN_OTHER,
-       PROF_EXCHANGE };
+       PROF_EXCHANGE, PROF_HYBRID };
 
 // ------------------------------------------------------------------ host helpers
 fgr_status fgr_set_error(fgr_status s, const char* fmt, ...);
@@ -185,6 +221,10 @@ cudaError_t fgr_launch_large_prep(fgr_grid* g, cudaStream_t st, const NetsView& 
 cudaError_t fgr_launch_commit(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int count,
                               const uint32_t* rec_seg, const int32_t* rec_off, int list_base);
 size_t fgr_dp_smem_small(const fgr_grid* g);
+fgr_status fgr_hyb_prepare(fgr_grid* g, cudaStream_t st, const NetsView& nv, int num_nets, int num_nodes,
+                           const int32_t* exec, int R, const int32_t* boff, int nb, int32_t* zmid);
+cudaError_t fgr_launch_hyb_tm(fgr_grid* g, cudaStream_t st, const NetsView& nv, int slot0, int n);
+cudaError_t fgr_launch_hyb_zmid(fgr_grid* g, cudaStream_t st, const uint32_t* seg, int32_t* zmid);
 size_t fgr_dp_smem_large(const fgr_grid* g, int m);
 
 static inline NetsView fgr_nets_view(const fgr_nets* n) {

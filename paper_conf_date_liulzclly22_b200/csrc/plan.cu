@@ -89,7 +89,7 @@ __global__ void k_preprocess(PlanParams p, NetsView nv, unsigned long long* __re
     if (trivial) atomicAdd(&counters[0], 1);
     if (!bad && !trivial) {
         // R19: worst case of any route = every unit edge at max cost + every via stack at max
-        const unsigned long long bound = wl * p.max_ec + (unsigned long long)(2 * m) * p.vmax;
+        const unsigned long long bound = wl * p.max_ec + (unsigned long long)(3 * m) * p.vmax;   // Z: 2 bend stacks per edge
         if (bound >= (unsigned long long)FGR_INF || m > p.max_nodes_large) atomicMin(&counters[2], net);
     }
     const unsigned hpwl = trivial ? 0xFFFFu : (unsigned)((x1 - x0) + (y1 - y0));
@@ -482,6 +482,7 @@ extern "C" FGR_API fgr_status fgr_plan(fgr_grid* g, const fgr_nets* nets, int32_
         FGR_CHECK_CUDA(g, cudaStreamSynchronize(st));
         g->cache.valid = true;
         g->cache.prep_valid = false;
+        g->hy.cached = false;
         g->cache.exec = order;
         g->cache.nets = *nets; g->cache.order = order; g->cache.batch_offset = batch_offset; g->cache.num_batches = 0;
         return FGR_OK;
@@ -645,6 +646,7 @@ extern "C" FGR_API fgr_status fgr_plan(fgr_grid* g, const fgr_nets* nets, int32_
     }
     c.valid = true;
     c.prep_valid = false;
+    g->hy.cached = false;
     c.exec = order;
     c.nets = *nets;
     c.order = order;

@@ -131,8 +131,23 @@ extern "C" FGR_API fgr_status fgr_split_batch(int32_t count, int32_t nlarge, int
     return FGR_OK;
 }
 
+extern "C" FGR_API fgr_status fgr_set_pattern(fgr_grid* g, int32_t hybrid_t1, int32_t hybrid_t2) {
+    if (!g) return fgr_set_error(FGR_ERR_INVALID, "grid is NULL");
+    if (hybrid_t1 <= hybrid_t2 && (hybrid_t1 < 0 || hybrid_t2 > 2 * 32767))
+        return fgr_set_error(FGR_ERR_INVALID, "hybrid window [%d, %d] out of range", hybrid_t1, hybrid_t2);
+    g->hyb_t1 = hybrid_t1;
+    g->hyb_t2 = hybrid_t2;
+    g->hy.cached = false;
+    return FGR_OK;
+}
+
 extern "C" FGR_API fgr_status fgr_route_batch(fgr_grid* g, const fgr_nets* nets, const int32_t* net_ids, int32_t count,
                                               uint32_t* seg_out, uint32_t* net_cost, void* stream) {
+    return fgr_route_batch_ex(g, nets, net_ids, count, seg_out, nullptr, net_cost, stream);
+}
+
+extern "C" FGR_API fgr_status fgr_route_batch_ex(fgr_grid* g, const fgr_nets* nets, const int32_t* net_ids, int32_t count,
+                                                 uint32_t* seg_out, int32_t* zmid_out, uint32_t* net_cost, void* stream) {
     if (!g || !nets) return fgr_set_error(FGR_ERR_INVALID, "NULL argument");
     if (g->broken) return fgr_set_error(FGR_ERR_STATE, "grid unusable after an earlier CUDA/NCCL error");
     if (count < 0) return fgr_set_error(FGR_ERR_INVALID, "count < 0");
@@ -152,10 +167,15 @@ extern "C" FGR_API fgr_status fgr_route_batch(fgr_grid* g, const fgr_nets* nets,
     int hc[8];
     FGR_CHECK_CUDA(g, cudaMemcpyAsync(hc, ctr, sizeof(hc), cudaMemcpyDeviceToHost, st));
     FGR_CHECK_CUDA(g, cudaStreamSynchronize(st));
-    FGR_CHECK_CUDA(g, refresh_before_dp(g, st, g->total_segs));
     const NetsView nv = fgr_nets_view(nets);
+    g->hy.cached = false;   // the hybrid tables below cover this batch only
+    fgr_status s = fgr_hyb_prepare(g, st, nv, nets->num_nets, nets->num_nodes, list, count, nullptr, 1, zmid_out);
+    if (s != FGR_OK) return s;
+    FGR_CHECK_CUDA(g, refresh_before_dp(g, st, g->total_segs));
+    FGR_CHECK_CUDA(g, fgr_launch_hyb_tm(g, st, nv, 0, g->hy.nslots));
     FGR_CHECK_CUDA(g, fgr_launch_dp(g, st, nv, list, hc[0], hc[1], hc[2], hc[3], hc[4], seg_out, net_cost, nullptr,
                                     nullptr, nullptr, 0, true, nullptr));
+    FGR_CHECK_CUDA(g, fgr_launch_hyb_zmid(g, st, seg_out, zmid_out));
     return FGR_OK;
 }
 
@@ -218,6 +238,7 @@ static fgr_status batch_info(fgr_grid* g, const fgr_nets* nets, const int32_t* o
     FGR_CHECK_CUDA(g, cudaStreamSynchronize(st));
     c.valid = true;
     c.prep_valid = false;
+    g->hy.cached = false;
     c.exec = exec;
     c.nets = *nets;
     c.order = order;
@@ -257,6 +278,28 @@ static fgr_status ensure_prep(fgr_grid* g, const fgr_nets* nets, int B, cudaStre
 extern "C" FGR_API fgr_status fgr_route_all(fgr_grid* g, const fgr_nets* nets, const int32_t* order,
                                             const int32_t* batch_offset, int32_t num_batches, uint32_t* seg_out,
                                             uint32_t* net_cost, void* stream) {
+    return fgr_route_all_ex(g, nets, order, batch_offset, num_batches, seg_out, nullptr, net_cost, stream);
+}
+
+// Hybrid tables for the stage (cached with the plan: same nets, exec order and window).
+static fgr_status ensure_hyb(fgr_grid* g, const fgr_nets* nets, const int32_t* batch_offset, int B, cudaStream_t st) {
+    HybState& h = g->hy;
+    const PlanCache& c = g->cache;
+    if (h.cached && h.key_exec == c.exec && h.key_t1 == g->hyb_t1 && h.key_t2 == g->hyb_t2) return FGR_OK;
+    const int R = B > 0 ? c.h_off[B] : 0;
+    fgr_status s = fgr_hyb_prepare(g, st, fgr_nets_view(nets), nets->num_nets, nets->num_nodes, c.exec, R, batch_offset,
+                                   B, nullptr);
+    if (s != FGR_OK) return s;
+    h.cached = true;
+    h.key_exec = c.exec;
+    h.key_t1 = g->hyb_t1;
+    h.key_t2 = g->hyb_t2;
+    return FGR_OK;
+}
+
+extern "C" FGR_API fgr_status fgr_route_all_ex(fgr_grid* g, const fgr_nets* nets, const int32_t* order,
+                                               const int32_t* batch_offset, int32_t num_batches, uint32_t* seg_out,
+                                               int32_t* zmid_out, uint32_t* net_cost, void* stream) {
     if (!g || !nets) return fgr_set_error(FGR_ERR_INVALID, "NULL argument");
     if (g->broken) return fgr_set_error(FGR_ERR_STATE, "grid unusable after an earlier CUDA/NCCL error");
     const int B = num_batches, N = nets->num_nets, M = nets->num_nodes;
@@ -269,8 +312,12 @@ extern "C" FGR_API fgr_status fgr_route_all(fgr_grid* g, const fgr_nets* nets, c
     if (s != FGR_OK) return s;
     s = ensure_prep(g, nets, B, st);
     if (s != FGR_OK) return s;
+    s = ensure_hyb(g, nets, batch_offset, B, st);
+    if (s != FGR_OK) return s;
     const PlanCache& c = g->cache;
+    const HybState& hy = g->hy;
     if (M > 0) FGR_CHECK_CUDA(g, cudaMemsetAsync(seg_out, 0xFF, sizeof(uint32_t) * (size_t)M, st));
+    if (M > 0 && zmid_out) FGR_CHECK_CUDA(g, cudaMemsetAsync(zmid_out, 0xFF, sizeof(int32_t) * (size_t)M, st));
     if (N > 0) FGR_CHECK_CUDA(g, cudaMemsetAsync(net_cost, 0, sizeof(uint32_t) * (size_t)N, st));
     const NetsView nv = fgr_nets_view(nets);
     g->stats.num_batches = B;
@@ -283,10 +330,12 @@ extern "C" FGR_API fgr_status fgr_route_all(fgr_grid* g, const fgr_nets* nets, c
         for (int b = 0; b < B; b++) {
             const long long bound = b > 0 ? c.h_segb[b - 1] : (long long)g->total_segs;
             FGR_CHECK_CUDA(g, refresh_before_dp(g, st, bound));
+            if (hy.active) FGR_CHECK_CUDA(g, fgr_launch_hyb_tm(g, st, nv, hy.boff[b], hy.boff[b + 1] - hy.boff[b]));
             const int o0 = c.h_off[b], cnt = c.h_off[b + 1] - o0, nl = c.h_nlarge[b], n2 = c.h_ntwo[b], n9 = c.h_n9[b];
             FGR_CHECK_CUDA(g, fgr_launch_dp(g, st, nv, c.exec + o0, nl, n9, cnt - nl - n9 - n2, n2, c.h_maxm[b],
                                             seg_out, net_cost, nullptr, nullptr, nullptr, 0, true, &c.prep));
-                }
+        }
+        FGR_CHECK_CUDA(g, fgr_launch_hyb_zmid(g, st, seg_out, zmid_out));
         return FGR_OK;
     }
     // ---- multi-GPU: split each batch, exchange route records, commit everywhere
@@ -319,6 +368,9 @@ extern "C" FGR_API fgr_status fgr_route_all(fgr_grid* g, const fgr_nets* nets, c
         const long long bound = b > 0 ? c.h_segb[b - 1] : (long long)g->total_segs;
         cudaError_t ce = refresh_before_dp(g, st, bound);
         if (ce != cudaSuccess) { rs = fgr_cuda_fail(g, ce, "refresh"); break; }
+        // every rank builds the batch's hybrid matrices: the commit of remote routes reads their Z argmins
+        if (hy.active) ce = fgr_launch_hyb_tm(g, st, nv, hy.boff[b], hy.boff[b + 1] - hy.boff[b]);
+        if (ce != cudaSuccess) { rs = fgr_cuda_fail(g, ce, "hybrid"); break; }
         const int o0 = c.h_off[b], cnt = c.h_off[b + 1] - o0, nl = c.h_nlarge[b], n2 = c.h_ntwo[b], n9 = c.h_n9[b];
         int32_t sp[4];
         fgr_split_batch(cnt, nl, g->rank, g->world, sp);
@@ -360,6 +412,7 @@ extern "C" FGR_API fgr_status fgr_route_all(fgr_grid* g, const fgr_nets* nets, c
                                                                                      net_cost);
         FGR_CHECK_CUDA(g, cudaGetLastError());
     }
+    FGR_CHECK_CUDA(g, fgr_launch_hyb_zmid(g, st, seg_out, zmid_out));
     return FGR_OK;
 }
 
@@ -392,6 +445,13 @@ extern "C" FGR_API fgr_status fgr_run_host(fgr_grid* g, int32_t N, int32_t M, co
                                            const int16_t* h_y, const int8_t* h_plo, const int8_t* h_phi,
                                            const int32_t* h_par, uint32_t* h_seg, uint32_t* h_cost,
                                            int32_t* h_nb, void* stream) {
+    return fgr_run_host_ex(g, N, M, h_off, h_x, h_y, h_plo, h_phi, h_par, h_seg, nullptr, h_cost, h_nb, stream);
+}
+
+extern "C" FGR_API fgr_status fgr_run_host_ex(fgr_grid* g, int32_t N, int32_t M, const int32_t* h_off,
+                                              const int16_t* h_x, const int16_t* h_y, const int8_t* h_plo,
+                                              const int8_t* h_phi, const int32_t* h_par, uint32_t* h_seg,
+                                              int32_t* h_zmid, uint32_t* h_cost, int32_t* h_nb, void* stream) {
     if (!g) return fgr_set_error(FGR_ERR_INVALID, "grid is NULL");
     if (g->broken) return fgr_set_error(FGR_ERR_STATE, "grid unusable after an earlier CUDA/NCCL error");
     if (N < 0 || M < 0 || (N > 0 && (!h_off || !h_x || !h_y || !h_plo || !h_phi || !h_par)))

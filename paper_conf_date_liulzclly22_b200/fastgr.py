@@ -25,9 +25,12 @@ STATUS_NAMES = ["OK", "INVALID", "RANGE", "OOM", "CUDA", "NCCL", "STATE"]
 EXPORTS = ["fgr_last_error", "fgr_version", "fgr_cost_table", "fgr_grid_create", "fgr_grid_destroy",
            "fgr_grid_set_demand", "fgr_grid_get_demand", "fgr_plan", "fgr_route_batch", "fgr_route_all",
            "fgr_comm_unique_id", "fgr_comm_init", "fgr_run_host", "fgr_get_stats", "fgr_profile_enable",
-           "fgr_profile_read", "fgr_split_batch"]
+           "fgr_profile_read", "fgr_split_batch", "fgr_set_pattern", "fgr_route_batch_ex", "fgr_route_all_ex",
+           "fgr_run_host_ex"]
 PROF_CLASSES = ["refresh", "dp_small", "dp_large", "commit", "plan_preprocess", "plan_sort", "plan_color",
-                "plan_other", "exchange"]
+                "plan_other", "exchange", "hybrid"]
+# the paper's FastGRH selection window: hybrid L+Z on two-pin HPWL in [100, 500]
+HYBRID_PAPER = (100, 500)
 
 
 class FgrError(RuntimeError):
@@ -82,6 +85,10 @@ def lib():
             "fgr_profile_enable": ([P, S], S),
             "fgr_profile_read": ([P, P, P], S),
             "fgr_split_batch": ([I, I, I, I, P], S),
+            "fgr_set_pattern": ([P, I, I], S),
+            "fgr_route_batch_ex": ([P, P, P, I, P, P, P, P], S),
+            "fgr_route_all_ex": ([P, P, P, P, I, P, P, P, P], S),
+            "fgr_run_host_ex": ([P, I, I, P, P, P, P, P, P, P, P, P, P, P], S),
         }
         for name, (args, res) in sig.items():
             f = getattr(L, name)
@@ -173,6 +180,20 @@ def fgr_route_all(h, nets, order, batch_offset, num_batches, seg_out, net_cost, 
                                _ptr(seg_out), _ptr(net_cost), _stream(stream)))
 
 
+def fgr_set_pattern(h, hybrid_t1, hybrid_t2):
+    _check(lib().fgr_set_pattern(h, int(hybrid_t1), int(hybrid_t2)))
+
+
+def fgr_route_batch_ex(h, nets, net_ids, count, seg_out, zmid_out, net_cost, stream=None):
+    _check(lib().fgr_route_batch_ex(h, ctypes.byref(nets), _ptr(net_ids), int(count), _ptr(seg_out), _ptr(zmid_out),
+                                    _ptr(net_cost), _stream(stream)))
+
+
+def fgr_route_all_ex(h, nets, order, batch_offset, num_batches, seg_out, zmid_out, net_cost, stream=None):
+    _check(lib().fgr_route_all_ex(h, ctypes.byref(nets), _ptr(order), _ptr(batch_offset), int(num_batches),
+                                  _ptr(seg_out), _ptr(zmid_out), _ptr(net_cost), _stream(stream)))
+
+
 def fgr_comm_unique_id() -> bytes:
     buf = ctypes.create_string_buffer(128)
     _check(lib().fgr_comm_unique_id(buf))
@@ -191,6 +212,17 @@ def fgr_run_host(h, node_offset, x, y, pin_lo, pin_hi, parent, seg_out=None, net
     M = len(x)
     _check(lib().fgr_run_host(h, N, M, _ptr(node_offset), _ptr(x), _ptr(y), _ptr(pin_lo), _ptr(pin_hi),
                               _ptr(parent), _ptr(seg_out), _ptr(net_cost), ctypes.byref(nb), _stream(stream)))
+    return nb.value
+
+
+def fgr_run_host_ex(h, node_offset, x, y, pin_lo, pin_hi, parent, seg_out=None, zmid_out=None, net_cost=None,
+                    stream=None) -> int:
+    nb = ctypes.c_int32(0)
+    N = len(node_offset) - 1
+    M = len(x)
+    _check(lib().fgr_run_host_ex(h, N, M, _ptr(node_offset), _ptr(x), _ptr(y), _ptr(pin_lo), _ptr(pin_hi),
+                                 _ptr(parent), _ptr(seg_out), _ptr(zmid_out), _ptr(net_cost), ctypes.byref(nb),
+                                 _stream(stream)))
     return nb.value
 
 
@@ -222,7 +254,7 @@ def fgr_profile_read(h) -> dict:
 class Router:
     """Owns a grid handle plus device copies of one design's nets (torch tensors)."""
 
-    def __init__(self, design, device: int = 0, stream=None):
+    def __init__(self, design, device: int = 0, stream=None, hybrid=None):
         import torch
         if not torch.cuda.is_available():
             raise RuntimeError("fastgr needs a CUDA device (no CPU fallback)")
@@ -237,6 +269,9 @@ class Router:
                               design.slack_clamp, ecap)
         self.h = fgr_grid_create(self.desc, device, stream)
         torch.cuda.synchronize(self.dev)
+        self.hybrid = hybrid
+        if hybrid is not None:
+            fgr_set_pattern(self.h, hybrid[0], hybrid[1])
         self._ecap = ecap
         t = lambda a: torch.from_numpy(np.ascontiguousarray(a)).to(self.dev)
         self.t_off, self.t_x, self.t_y = t(design.node_offset), t(design.x), t(design.y)
@@ -249,6 +284,7 @@ class Router:
         self.order = torch.empty(max(N, 1), dtype=i32, device=self.dev)
         self.batch_offset = torch.empty(N + 1, dtype=i32, device=self.dev)
         self.seg = torch.empty(max(M, 1), dtype=i32, device=self.dev)
+        self.zmid = torch.full((max(M, 1),), -1, dtype=i32, device=self.dev)
         self.cost = torch.empty(max(N, 1), dtype=i32, device=self.dev)
         self.num_batches = 0
 
@@ -271,10 +307,19 @@ class Router:
         return self.num_batches
 
     def route_all(self, stream=None):
-        fgr_route_all(self.h, self.nets, self.order, self.batch_offset, self.num_batches, self.seg, self.cost, stream)
+        if self.hybrid is None:
+            fgr_route_all(self.h, self.nets, self.order, self.batch_offset, self.num_batches, self.seg, self.cost,
+                          stream)
+        else:
+            fgr_route_all_ex(self.h, self.nets, self.order, self.batch_offset, self.num_batches, self.seg, self.zmid,
+                             self.cost, stream)
 
     def route_batch(self, net_ids, stream=None):
-        fgr_route_batch(self.h, self.nets, net_ids, int(net_ids.numel()), self.seg, self.cost, stream)
+        if self.hybrid is None:
+            fgr_route_batch(self.h, self.nets, net_ids, int(net_ids.numel()), self.seg, self.cost, stream)
+        else:
+            fgr_route_batch_ex(self.h, self.nets, net_ids, int(net_ids.numel()), self.seg, self.zmid, self.cost,
+                               stream)
 
     def demand(self, stream=None):
         out = self.torch.empty((self.d.nlayers, self.d.ny, self.d.nx), dtype=self.torch.int32, device=self.dev)
@@ -294,3 +339,8 @@ class Router:
         return (self.batch_of_net[:N].cpu().numpy(), self.num_batches,
                 self.seg[:M].cpu().numpy().view(np.uint32), self.cost[:N].cpu().numpy().view(np.uint32),
                 self.demand().cpu().numpy())
+
+    def zmids(self):
+        """zmid int32[M] (mid | lb << 16 of Z routes, -1 elsewhere) of the last hybrid route call."""
+        self.torch.cuda.synchronize(self.dev)
+        return self.zmid[:self.d.num_nodes].cpu().numpy()
