@@ -80,6 +80,19 @@ def design_stats(d):
                 nodes_large=int(sizes[sizes > 32].sum()), nets_large=int((sizes > 32).sum()))
 
 
+def hybrid_edges(d, w):
+    """Bent tree edges whose two-pin HPWL lies in the hybrid window (reading R23)."""
+    sizes = d.net_sizes()
+    nid = np.repeat(np.arange(d.num_nets), sizes)
+    off = d.node_offset[:-1].astype(np.int64)[nid]
+    ch = d.parent >= 0
+    p = off[ch] + d.parent[ch]
+    dx = np.abs(d.x[ch].astype(np.int64) - d.x[p])
+    dy = np.abs(d.y[ch].astype(np.int64) - d.y[p])
+    h = dx + dy
+    return int(((h >= w[0]) & (h <= w[1]) & (dx > 0) & (dy > 0)).sum())
+
+
 def dp_bytes(M, E, WL, N):
     """SURVEY.md §8(d) per-net figure: 12 B/node input + 8 gathered 32-B sectors per
     tree edge + 4 B/edge segment out + 4 B/net cost + 8 B per committed unit edge."""
@@ -161,13 +174,13 @@ def run_reference(args, rank):
     print(json.dumps(line), flush=True)
 
 
-def cpu_baseline(d, config, budget_s=20.0):
+def cpu_baseline(d, config, budget_s=20.0, hybrid=None):
     """The oracle as it stands, on this host, single thread: whole design if it fits the budget."""
     from oracle import Oracle
     o = Oracle(d)
     t0 = time.perf_counter()
     b, nb = o.plan()
-    o.route(b, nb)
+    o.route(b, nb, hybrid=hybrid)
     t = time.perf_counter() - t0
     routed = int((d.net_sizes() >= 2).sum())
     return {"value": routed / t, "unit": "nets/s", "cores": 1, "kind": "oracle",
@@ -195,6 +208,8 @@ def main():
     ap.add_argument("--ref-fraction", type=float, default=0.25)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--hybrid", default=None,
+                    help="T1,T2: hybrid L+Z patterns on tree edges with T1 <= HPWL <= T2 (FastGRH; default L only)")
     args = ap.parse_args()
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -214,7 +229,8 @@ def main():
     dev = torch.device("cuda", local)
     d = gen.make_config(args.config)
     ds = design_stats(d)
-    r = Router(d, device=local)
+    hybrid = tuple(int(v) for v in args.hybrid.split(",")) if args.hybrid else None
+    r = Router(d, device=local, hybrid=hybrid)
     if world > 1:
         uid = [F.fgr_comm_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(uid, src=0)
@@ -304,16 +320,23 @@ def main():
         h = [pin(d.node_offset), pin(d.x), pin(d.y), pin(d.pin_lo), pin(d.pin_hi), pin(d.parent)]
         seg_h = torch.empty(d.num_nodes, dtype=torch.int32).pin_memory()
         cost_h = torch.empty(d.num_nets, dtype=torch.int32).pin_memory()
+        zmid_h = torch.empty(d.num_nodes, dtype=torch.int32).pin_memory() if hybrid else None
         h2d = sum(t.numel() * t.element_size() for t in h)
-        d2h = seg_h.numel() * 4 + cost_h.numel() * 4
+        d2h = seg_h.numel() * 4 + cost_h.numel() * 4 + (zmid_h.numel() * 4 if hybrid else 0)
+
+        def run_host():
+            if hybrid:
+                F.fgr_run_host_ex(r.h, *h, seg_out=seg_h, zmid_out=zmid_h, net_cost=cost_h)
+            else:
+                F.fgr_run_host(r.h, *h, seg_out=seg_h, net_cost=cost_h)
         for _ in range(max(1, args.warmup)):
-            F.fgr_run_host(r.h, *h, seg_out=seg_h, net_cost=cost_h)
+            run_host()
         times = []
         for _ in range(max(3, min(args.steps, 5))):
             flush.zero_()
             a = torch.cuda.Event(enable_timing=True); b = torch.cuda.Event(enable_timing=True)
             a.record(stream)
-            F.fgr_run_host(r.h, *h, seg_out=seg_h, net_cost=cost_h)
+            run_host()
             b.record(stream)
             b.synchronize()
             times.append(a.elapsed_time(b))
@@ -324,7 +347,7 @@ def main():
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        cpu = cpu_baseline(d, args.config)
+        cpu = cpu_baseline(d, args.config, hybrid=hybrid)
 
     if rank == 0:
         line = {
@@ -335,7 +358,10 @@ def main():
                        "nets_total": ds["nets_total"], "nets_routed": ds["nets_routed"], "nodes": ds["nodes"],
                        "tree_edges": ds["edges"], "batches": r.num_batches,
                        "l2": "flushed between steps (256 MiB write, outside the step events)",
-                       "parallelism": f"grid replicated, batches split over {world} rank(s)"},
+                       "parallelism": f"grid replicated, batches split over {world} rank(s)",
+                       "pattern": ("L shapes (FastGRL)" if hybrid is None else
+                                   f"hybrid L+Z on tree edges with {hybrid[0]} <= HPWL <= {hybrid[1]} (FastGRH), "
+                                   f"{hybrid_edges(d, hybrid)} hybrid edges")},
             "plan_ms": statistics.mean(plan_ms), "route_ms": statistics.mean(route_ms),
             "clocks": clk, "e2e": e2e, "gpu_launches": int(launches_total // max(1, steps)),
             "gpu_launches_note": "library kernels per step (CUB sort kernels counted as one launch each call)",

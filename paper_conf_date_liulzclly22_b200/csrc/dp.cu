@@ -1234,67 +1234,52 @@ __global__ void __launch_bounds__(32 * kLargeWarps, 1) k_dp_large(GridView g, Ne
     }
     __syncthreads();
     TMARK(3);
-    // ---------------- backtrack: top-down path walks (S5)
-#ifdef FGR_TIMING
-    long long bt_wait = 0, bt_walk = 0, bt_nodes = 0, bt_paths = 0;
-#endif
-    if (glane) {
-        for (;;) {
-            int p = 0;
-            if (gl == 0) p = atomicAdd(&s_ticket2, 1);   // ticket 0 = the root path (shallowest top)
-            p = __shfl_sync(gmask, p, gbase);
-            if (p >= npaths) break;
-            const int tp = t.pq[npaths - 1 - p];
-            int v;
-#ifdef FGR_TIMING
-            long long w0 = clock64();
-#endif
-            if (tp == 0) v = t.hv[0];
-            else {
-                while (ld_flag(&t.sready[t.par[tp]]) == 0) __nanosleep(40);
+    // ---------------- backtrack: top-down path walks (S5), one lane per path
+    // A walk is a scalar chain (span of u -> lt -> ls -> span of v), so lane 0 of a warp
+    // walks a path with the parent's span in a register (no shuffles, no per-node warp
+    // synchronisation); a path whose top hangs off another path waits for that node's span
+    // (sready).  Warps take paths by ticket, shallowest top first, so every awaited path is
+    // already held by a running warp (no deadlock).
+    for (;;) {
+        int p = 0;
+        if (lane == 0) p = atomicAdd(&s_ticket2, 1);
+        p = __shfl_sync(0xffffffffu, p, 0);
+        if (p >= npaths) break;
+        if (lane != 0) continue;
+        const int tp = t.pq[npaths - 1 - p];
+        int v, sp;
+        if (tp == 0) { v = t.hv[0]; sp = t.span[0]; }
+        else {
+            const int u0 = t.par[tp];
+            while (ld_flag(&t.sready[u0]) == 0) __nanosleep(32);
+            __threadfence_block();
+            v = tp;
+            sp = t.span[u0];
+        }
+        while (v != 0xFFFF) {
+            const int u = t.par[v];
+            const int lo = sp >> 4, hi = sp & 15;
+            uint32_t ev[LT];
+#pragma unroll
+            for (int l = 0; l < LT; l++) ev[l] = t.E[(size_t)v * LT + l];
+            uint32_t be = 0xFFFFFFFFu;
+            int lt = lo;
+#pragma unroll
+            for (int l = 0; l < LT; l++)
+                if (l >= lo && l <= hi && ev[l] < be) { be = ev[l]; lt = l; }   // smallest l attaining the min (R11)
+            const int ls = t.recE[(size_t)v * LT + lt];
+            sp = t.recB[(size_t)v * LT + ls];
+            t.span[v] = (uint8_t)sp;
+            const bool straight = (t.x[v] == t.x[u]) || (t.y[v] == t.y[u]);
+            const uint32_t bend = seg_bend(h->dir[ls], h->dir[lt], straight);
+            t.legH[(size_t)v * 2 * nH] = bend | ((uint32_t)ls << 8) | ((uint32_t)lt << 16) | ((uint32_t)straight << 24);
+            if (t.cstart[v + 1] - t.cstart[v] > 1) {   // light children wait for this span
                 __threadfence_block();
-                v = tp;
+                *(volatile uint8_t*)&t.sready[v] = 1;
             }
-#ifdef FGR_TIMING
-            long long w1 = clock64();
-            bt_wait += w1 - w0;
-            bt_paths++;
-#endif
-            while (v != 0xFFFF) {
-#ifdef FGR_TIMING
-                bt_nodes++;
-#endif
-                const int u = t.par[v];
-                const int sp = t.span[u];
-                const int lo = sp >> 4, hi = sp & 15;
-                const int l = gl;
-                const uint32_t cand = (l >= lo && l <= hi) ? t.E[(size_t)v * LT + l] : 0xFFFFFFFFu;
-                const uint32_t mn = __reduce_min_sync(gmask, cand);
-                const unsigned bal = __ballot_sync(gmask, cand == mn) >> gbase;   // smallest l attaining the min (R11)
-                if (gl == 0) {
-                    const int lt = __ffs(bal) - 1;
-                    const int ls = t.recE[(size_t)v * LT + lt];
-                    t.span[v] = t.recB[(size_t)v * LT + ls];
-                    const bool straight = (t.x[v] == t.x[u]) || (t.y[v] == t.y[u]);
-                    const uint32_t bend = seg_bend(h->dir[ls], h->dir[lt], straight);
-                    const uint32_t sg = bend | ((uint32_t)ls << 8) | ((uint32_t)lt << 16) | ((uint32_t)straight << 24);
-                    t.legH[(size_t)v * 2 * nH] = sg;   // the leg costs are dead now: keep the route (shared memory only)
-                }
-                __syncwarp(gmask);
-                __threadfence_block();
-                if (gl == 0) *(volatile uint8_t*)&t.sready[v] = 1;
-                v = t.hv[v];
-            }
-#ifdef FGR_TIMING
-            bt_walk += clock64() - w1;
-#endif
+            v = t.hv[v];
         }
     }
-#ifdef FGR_TIMING_DETAIL
-    if (gl == 0 && glane && m > 900)
-        printf("BT m=%d warp=%d paths=%lld nodes=%lld wait=%lld walk=%lld per_node=%lld\n", m, warp, bt_paths, bt_nodes,
-               bt_wait, bt_walk, bt_nodes ? bt_walk / bt_nodes : 0);
-#endif
     __syncthreads();
     TMARK(4);
     TMARK(5);
