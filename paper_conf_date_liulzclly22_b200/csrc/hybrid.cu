@@ -96,88 +96,125 @@ __global__ void k_hyb_boff(int n, const int32_t* __restrict__ boff, const int32_
     if (i < n) out[i] = base[boff[i]];
 }
 
-constexpr int kTmWarps = 4;
+constexpr int kTmThreads = 128;
+constexpr int kTmTile = 64;     // candidates whose legs are staged in shared memory at a time
 
 // Transfer matrices M[s][lt][ls] (values) and A[s][lt][ls] (Z argmin mid | lb << 16, 0xFFFFFFFF = the L shape
-// or no candidate) of the hybrid edges s = slot0 .. slot0 + gridDim.x - 1.
+// or no candidate) of the hybrid edges s = slot0 .. slot0 + gridDim.x - 1, one CTA per edge.
+// Per family (HVH: ls, lt horizontal; VHV: ls, lt vertical) the candidates are processed in tiles:
+// the CTA first stages the three leg costs of every layer for a tile of bend positions in shared
+// memory (each leg one prefix difference), then every thread owns one (ls, lt) entry (or a share of
+// one) and scans the tile: value = leg1(ls) + min_lb [V(ls,lb) + leg2(lb) + V(lb,lt)] + leg3(lt)
+// (Eqs. (11)-(14)); the running minimum of the packed (value, mid, lb) key is Eq. (10)'s merge.
 template <int LT>
-__global__ void __launch_bounds__(32 * kTmWarps) k_hyb_tm(GridView g, NetsView nv, const int32_t* __restrict__ hlist,
-                                                         const int32_t* __restrict__ hpar, int slot0,
-                                                         uint32_t* __restrict__ M, uint32_t* __restrict__ A) {
+__global__ void __launch_bounds__(kTmThreads) k_hyb_tm(GridView g, NetsView nv, const int32_t* __restrict__ hlist,
+                                                      const int32_t* __restrict__ hpar, int slot0,
+                                                      uint32_t* __restrict__ M, uint32_t* __restrict__ A) {
+    __shared__ uint32_t legs[kTmTile][3][LT];
+    __shared__ unsigned long long best_s[LT * LT];
     const int s = slot0 + blockIdx.x;
     const int gv = hlist[s], gu = hpar[s];
     const int xv = nv.x[gv], yv = nv.y[gv], xu = nv.x[gu], yu = nv.y[gu];
-    const int warp = threadIdx.x >> 5, lane = lane_id();
+    const int t = threadIdx.x;
     uint32_t vp[LT];
     int dl[LT], sl[LT];
 #pragma unroll
     for (int l = 0; l < LT; l++) { vp[l] = g.viapre[l]; dl[l] = g.dir[l]; sl[l] = g.slot[l]; }
-    auto via = [&](int a, int b) -> uint32_t {   // V(min, max) for compile-time-unrolled indices
-        return vp[a] > vp[b] ? vp[a] - vp[b] : vp[b] - vp[a];
-    };
     uint32_t* Ms = M + (size_t)s * LT * LT;
     uint32_t* As = A + (size_t)s * LT * LT;
+    const int xlo = min(xv, xu), ylo = min(yv, yu);
+    // the L shape for every (ls, lt) of opposite directions (bend 0 if leg 1 is horizontal)
+    for (int e = t; e < LT * LT; e += kTmThreads) {
+        const int ls = e % LT, lt = e / LT;
+        best_s[e] = ~0ull;
+        const int dls = g.dir[ls], dlt = g.dir[lt];
+        if (dls != dlt) {
+            const int sls = g.slot[ls], slt = g.slot[lt];
+            const uint32_t l1 = dls == 0 ? leg_of(g.h, yv, xv, xu, sls) : leg_of(g.v, xv, yv, yu, sls);
+            const uint32_t l2 = dls == 0 ? leg_of(g.v, xu, yv, yu, slt) : leg_of(g.h, yu, xv, xu, slt);
+            const uint32_t vv = g.viapre[max(ls, lt)] - g.viapre[min(ls, lt)];
+            Ms[lt * LT + ls] = l1 + vv + l2;
+            As[lt * LT + ls] = 0xFFFFFFFFu;
+        }
+    }
+    for (int f = 0; f < 2; f++) {   // f = 0: HVH (ls, lt horizontal), f = 1: VHV
+        const int nmid = f == 0 ? abs(xu - xv) - 1 : abs(yu - yv) - 1;
+        int nf = 0;
 #pragma unroll
-    for (int ls = 0; ls < LT; ls++) {
-        if (ls % kTmWarps != warp) continue;
-        const int dls = dl[ls];
-        // the L shape for every lt of the other direction (bend 0 if leg 1 is horizontal)
+        for (int l = 0; l < LT; l++) nf += dl[l] == f ? 1 : 0;
+        const int nE = nf * nf;
+        if (nmid <= 0 || nE == 0) continue;
+        const int tpe = nE <= kTmThreads ? kTmThreads / nE : 1;   // threads sharing one entry
+        // this thread's entries (at most 2: nE <= 15 * 15)
+        int ls_[2] = {-1, -1}, lt_[2] = {-1, -1};
+        uint32_t vsum[2][LT];
+        unsigned long long best[2] = {~0ull, ~0ull};
+        const int sub = t % tpe;
+        for (int k = 0; k < 2; k++) {
+            const int e = t / tpe + k * (kTmThreads / tpe);
+            if (e >= nE || (k == 1 && tpe > 1)) break;
+            int a = e / nf, b = e % nf, ls = -1, lt = -1;
 #pragma unroll
-        for (int lt = 0; lt < LT; lt++)
-            if (lane == lt && dl[lt] != dls) {
-                const uint32_t l1 = dls == 0 ? leg_of(g.h, yv, xv, xu, sl[ls]) : leg_of(g.v, xv, yv, yu, sl[ls]);
-                const uint32_t l2 = dls == 0 ? leg_of(g.v, xu, yv, yu, sl[lt]) : leg_of(g.h, yu, xv, xu, sl[lt]);
-                Ms[lt * LT + ls] = l1 + via(ls, lt) + l2;
-                As[lt * LT + ls] = 0xFFFFFFFFu;
+            for (int l = 0; l < LT; l++)
+                if (dl[l] == f) { if (a == 0) ls = l; if (b == 0) lt = l; a--; b--; }
+            ls_[k] = ls; lt_[k] = lt;
+            uint32_t vls = 0, vlt = 0;
+#pragma unroll
+            for (int l = 0; l < LT; l++) { vls = l == ls ? vp[l] : vls; vlt = l == lt ? vp[l] : vlt; }
+#pragma unroll
+            for (int lb = 0; lb < LT; lb++) {
+                const uint32_t a1 = vp[lb] > vls ? vp[lb] - vls : vls - vp[lb];
+                const uint32_t a2 = vp[lb] > vlt ? vp[lb] - vlt : vlt - vp[lb];
+                vsum[k][lb] = a1 + a2;   // V(ls, lb) + V(lb, lt)
             }
-        // Z shapes (lt in the direction of ls): candidate flows over the interior bend positions
-        const bool hvh = dls == 0;
-        const int p0 = hvh ? min(xv, xu) + 1 : min(yv, yu) + 1;
-        const int p1 = hvh ? max(xv, xu) - 1 : max(yv, yu) - 1;
-        unsigned long long best[LT];
-#pragma unroll
-        for (int lt = 0; lt < LT; lt++) best[lt] = ~0ull;
-        for (int mid = p0 + lane; mid <= p1; mid += 32) {
-            // Eq. (11): leg 1 on ls;  Eq. (12): bend via + leg 2 on lb;  Eq. (13): bend via + leg 3 on lt
-            const uint32_t w1 = hvh ? leg_of(g.h, yv, xv, mid, sl[ls]) : leg_of(g.v, xv, yv, mid, sl[ls]);
-            uint32_t t2v[LT];
-#pragma unroll
-            for (int lb = 0; lb < LT; lb++)
-                if (dl[lb] != dls)
-                    t2v[lb] = via(ls, lb) + (hvh ? leg_of(g.v, mid, yv, yu, sl[lb]) : leg_of(g.h, mid, xv, xu, sl[lb]));
-#pragma unroll
-            for (int lt = 0; lt < LT; lt++)
-                if (dl[lt] == dls) {
+        }
+        const int base = f == 0 ? xlo + 1 : ylo + 1;
+        for (int c0 = 0; c0 < nmid; c0 += kTmTile) {
+            const int nt = min(kTmTile, nmid - c0);
+            __syncthreads();
+            for (int it = t; it < nt * LT; it += kTmThreads) {
+                const int i = it / LT, l = it % LT;
+                const int mid = base + c0 + i;
+                const int sll = g.slot[l];
+                if (g.dir[l] == f) {
+                    legs[i][0][l] = f == 0 ? leg_of(g.h, yv, xv, mid, sll) : leg_of(g.v, xv, yv, mid, sll);
+                    legs[i][2][l] = f == 0 ? leg_of(g.h, yu, mid, xu, sll) : leg_of(g.v, xu, mid, yu, sll);
+                } else {
+                    legs[i][1][l] = f == 0 ? leg_of(g.v, mid, yv, yu, sll) : leg_of(g.h, mid, xv, xu, sll);
+                }
+            }
+            __syncthreads();
+            for (int k = 0; k < 2; k++) {
+                if (ls_[k] < 0) break;
+                const int ls = ls_[k], lt = lt_[k];
+                for (int i = sub; i < nt; i += tpe) {
                     uint32_t bv = 0xFFFFFFFFu;
                     int blb = 0;
 #pragma unroll
                     for (int lb = 0; lb < LT; lb++)
-                        if (dl[lb] != dls) {
-                            const uint32_t c = t2v[lb] + via(lb, lt);
+                        if (dl[lb] != f) {
+                            const uint32_t c = vsum[k][lb] + legs[i][1][lb];
                             if (c < bv) { bv = c; blb = lb; }   // first minimum: smallest lb (R25)
                         }
-                    const uint32_t w3 = hvh ? leg_of(g.h, yu, mid, xu, sl[lt]) : leg_of(g.v, xu, mid, yu, sl[lt]);
+                    const uint32_t val = legs[i][0][ls] + bv + legs[i][2][lt];
                     const unsigned long long key =
-                        ((unsigned long long)(w1 + bv + w3) << 32) | ((unsigned)mid << 4) | (unsigned)blb;
-                    best[lt] = key < best[lt] ? key : best[lt];
-                }
-        }
-        // merge step, Eq. (10): warp minimum of the packed (value, mid, lb) keys
-#pragma unroll
-        for (int lt = 0; lt < LT; lt++)
-            if (dl[lt] == dls) {
-                unsigned long long k = best[lt];
-#pragma unroll
-                for (int off = 16; off; off >>= 1) {
-                    const unsigned long long o = __shfl_xor_sync(0xffffffffu, k, off);
-                    k = o < k ? o : k;
-                }
-                if (lane == 0) {
-                    const bool none = k == ~0ull;
-                    Ms[lt * LT + ls] = none ? FGR_INF : (uint32_t)(k >> 32);
-                    As[lt * LT + ls] = none ? 0xFFFFFFFFu : ((uint32_t)((k >> 4) & 0xFFFF) | ((uint32_t)(k & 15) << 16));
+                        ((unsigned long long)val << 32) | ((unsigned)(base + c0 + i) << 4) | (unsigned)blb;
+                    best[k] = key < best[k] ? key : best[k];
                 }
             }
+        }
+        for (int k = 0; k < 2; k++)
+            if (ls_[k] >= 0) atomicMin(&best_s[lt_[k] * LT + ls_[k]], best[k]);
+    }
+    __syncthreads();
+    for (int e = t; e < LT * LT; e += kTmThreads) {
+        const int ls = e % LT, lt = e / LT;
+        if (g.dir[ls] == g.dir[lt]) {
+            const unsigned long long k = best_s[lt * LT + ls];
+            const bool none = k == ~0ull;
+            Ms[lt * LT + ls] = none ? FGR_INF : (uint32_t)(k >> 32);
+            As[lt * LT + ls] = none ? 0xFFFFFFFFu : ((uint32_t)((k >> 4) & 0xFFFF) | ((uint32_t)(k & 15) << 16));
+        }
     }
 }
 
@@ -196,7 +233,7 @@ __global__ void k_hyb_zmid(int n, int L, const int32_t* __restrict__ hlist, cons
 
 template <int LT>
 cudaError_t launch_tm_lt(fgr_grid* g, cudaStream_t st, const NetsView& nv, int slot0, int n) {
-    k_hyb_tm<LT><<<n, 32 * kTmWarps, 0, st>>>(g->view, nv, g->hy.list, g->hy.par, slot0, g->hy.M, g->hy.A);
+    k_hyb_tm<LT><<<n, kTmThreads, 0, st>>>(g->view, nv, g->hy.list, g->hy.par, slot0, g->hy.M, g->hy.A);
     return cudaGetLastError();
 }
 
