@@ -72,9 +72,11 @@ def _lib():
         lib.orc_commit_net_ex.argtypes = [P, P, ctypes.c_int32, P, P, P]
         lib.orc_route_ex.argtypes = [P, P, P, ctypes.c_int32, P, P, P, ctypes.c_int, P, P, P]
         lib.orc_recost_net_ex.argtypes = [P, P, ctypes.c_int32, P, P, P, P]
+        lib.orc_overflow.argtypes = [P, P, P, P, P, P, P]
+        lib.orc_task_graph.argtypes = [P, P, P, ctypes.c_int32, P, P, P, P, ctypes.c_int64, P]
         for f in ("orc_cost_table", "orc_validate", "orc_plan", "orc_route_net", "orc_commit_net",
                   "orc_route", "orc_recost_net", "orc_route_net_ex", "orc_commit_net_ex", "orc_route_ex",
-                  "orc_recost_net_ex"):
+                  "orc_recost_net_ex", "orc_overflow", "orc_task_graph"):
             getattr(lib, f).restype = ctypes.c_int
         _LIB = lib
     return _LIB
@@ -188,6 +190,34 @@ class Oracle:
                                  _p(np.ascontiguousarray(seg, np.uint32)),
                                  _p(None if zmid is None else np.ascontiguousarray(zmid, np.int32)), _p(c))
         return int(c[0])
+
+    def overflow(self, seg, demand, zmid=None):
+        """Rip-up set on a final demand -> (violating uint8[N], (overflowed edges, total overflow))."""
+        viol = np.zeros(max(self.d.num_nets, 1), np.uint8)
+        tot = np.zeros(2, np.int64)
+        _lib().orc_overflow(ctypes.byref(self.g), ctypes.byref(self.n), _p(np.ascontiguousarray(seg, np.uint32)),
+                            _p(None if zmid is None else np.ascontiguousarray(zmid, np.int32)),
+                            _p(np.ascontiguousarray(demand, np.int32)), _p(viol), _p(tot))
+        return viol[:self.d.num_nets], (int(tot[0]), int(tot[1]))
+
+    def task_graph(self, tasks):
+        """Ordered task graph of net ids `tasks` -> (order, is_root, succ_offset, succ) (task-ID indexed)."""
+        tasks = np.ascontiguousarray(tasks, np.int32)
+        R = len(tasks)
+        order = np.zeros(max(R, 1), np.int32)
+        root = np.zeros(max(R, 1), np.uint8)
+        off = np.zeros(R + 1, np.int32)
+        ne = np.zeros(1, np.int64)
+        cap = 0
+        while True:
+            succ = np.zeros(max(cap, 1), np.int32)
+            rc = _lib().orc_task_graph(ctypes.byref(self.g), ctypes.byref(self.n), _p(tasks), R, _p(order),
+                                       _p(root), _p(off), _p(succ), int(cap), _p(ne))
+            if rc == ORC_OK:
+                return order[:R], root[:R], off, succ[:int(ne[0])]
+            if rc != ORC_RANGE:
+                raise ValueError(f"orc_task_graph rc={rc}")
+            cap = int(ne[0])
 
     def run(self):
         """Whole stage: plan + route from zero demand."""

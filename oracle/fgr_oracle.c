@@ -588,3 +588,114 @@ int orc_route_ex(const orc_grid* g, const orc_nets* n, const int32_t* batch_of_n
     free(c.table); free(cnt); free(lst); free(pos);
     return rc;
 }
+
+/* ------------------------------------------- overflow extraction (NEXT #3) */
+
+/*
+ * Rip-up set after the pattern-routing stage (§III-A: "we first
+ * extract the nets to rip up"; §III-G: "rewire the nets with violations").
+ * Reading R26: a wire edge is overflowed when its demand exceeds its capacity; a net
+ * is violating when one of its committed legs covers an overflowed edge.
+ * totals[0] = overflowed wire edges, totals[1] = sum of (demand - capacity) over them.
+ */
+int orc_overflow(const orc_grid* g, const orc_nets* n, const uint32_t* seg, const int32_t* zmid,
+                 const int32_t* demand, uint8_t* violating, int64_t* totals) {
+    int L = g->nlayers;
+    int64_t cnt = 0, sum = 0;
+    for (int l = 0; l < L; l++)
+        for (int y = 0; y < g->ny; y++)
+            for (int x = 0; x < g->nx; x++) {
+                if (g->dir[l] == 0 && x == g->nx - 1) continue;   /* no wire edge there */
+                if (g->dir[l] == 1 && y == g->ny - 1) continue;
+                int64_t over = (int64_t)demand[((int64_t)l * g->ny + y) * g->nx + x] - capacity_at(g, l, y, x);
+                if (over > 0) { cnt++; sum += over; }
+            }
+    totals[0] = cnt;
+    totals[1] = sum;
+    for (int i = 0; i < n->num_nets; i++) {
+        int a = n->node_offset[i], m = n->node_offset[i + 1] - a, bad = 0;
+        for (int v = 1; v < m && !bad; v++) {
+            int u = n->parent[a + v];
+            int legs[3][5];
+            int k = route_legs(seg[a + v], zmid ? zmid[a + v] : -1, n->x[a + v], n->y[a + v], n->x[a + u],
+                               n->y[a + u], legs);
+            for (int j = 0; j < k && !bad; j++) {
+                int l = legs[j][0], xa = legs[j][1], ya = legs[j][2], xb = legs[j][3], yb = legs[j][4];
+                if (ya == yb) {
+                    for (int x = (xa < xb ? xa : xb); x < (xa < xb ? xb : xa); x++)
+                        if (demand[((int64_t)l * g->ny + ya) * g->nx + x] > capacity_at(g, l, ya, x)) { bad = 1; break; }
+                } else {
+                    for (int y = (ya < yb ? ya : yb); y < (ya < yb ? yb : ya); y++)
+                        if (demand[((int64_t)l * g->ny + y) * g->nx + xa] > capacity_at(g, l, y, xa)) { bad = 1; break; }
+                }
+            }
+        }
+        violating[i] = (uint8_t)bad;
+    }
+    return ORC_OK;
+}
+
+/*
+ * Ordered task graph of a set of routing tasks (§III-B, Fig. 6):
+ *   task IDs = the tasks sorted by (HPWL, net id) ("the task ID indicates the sorting
+ *   result", L461-462; sort key as reading R12);
+ *   conflict = closed bounding boxes share a G-cell (reading R13);
+ *   root task batch = one pass of Algorithm 1 over the sorted tasks (L432-448);
+ *   every conflicting pair is ordered root -> non-root (L454-456), else from the
+ *   smaller task ID to the larger (L457-459).
+ * Outputs: order[t] = net id of task t; is_root[t]; successors in CSR by task ID,
+ * ascending.  ORC_RANGE (with *num_edges set) when the edges exceed `cap`.
+ */
+int orc_task_graph(const orc_grid* g, const orc_nets* n, const int32_t* tasks, int32_t count, int32_t* order,
+                   uint8_t* is_root, int32_t* succ_off, int32_t* succ, int64_t cap, int64_t* num_edges) {
+    keyed* t = (keyed*)malloc(sizeof(keyed) * (count > 0 ? count : 1));
+    int* bx = (int*)malloc(sizeof(int) * 4 * (count > 0 ? count : 1));
+    for (int i = 0; i < count; i++) {
+        int x0, y0, x1, y1;
+        net_bbox(n, tasks[i], &x0, &y0, &x1, &y1);
+        t[i].key = (int64_t)(x1 - x0) + (y1 - y0);
+        t[i].id = tasks[i];
+    }
+    qsort(t, count, sizeof(keyed), cmp_keyed);
+    for (int i = 0; i < count; i++) {
+        order[i] = t[i].id;
+        net_bbox(n, t[i].id, &bx[4 * i], &bx[4 * i + 1], &bx[4 * i + 2], &bx[4 * i + 3]);
+    }
+    /* root batch: Algorithm 1 lines 1-8, literally (occupancy bitmap of the batch) */
+    uint8_t* occ = (uint8_t*)calloc((size_t)g->nx * g->ny, 1);
+    for (int i = 0; i < count; i++) {
+        int conflict = 0;
+        for (int y = bx[4 * i + 1]; y <= bx[4 * i + 3] && !conflict; y++)
+            for (int x = bx[4 * i]; x <= bx[4 * i + 2]; x++)
+                if (occ[(int64_t)y * g->nx + x]) { conflict = 1; break; }
+        is_root[i] = (uint8_t)!conflict;
+        if (!conflict)
+            for (int y = bx[4 * i + 1]; y <= bx[4 * i + 3]; y++)
+                for (int x = bx[4 * i]; x <= bx[4 * i + 2]; x++) occ[(int64_t)y * g->nx + x] = 1;
+    }
+    free(occ);
+    /* every conflicting pair, oriented; CSR by source, successors ascending */
+    int64_t ne = 0;
+    for (int i = 0; i <= count; i++) succ_off[i] = 0;
+    for (int pass = 0; pass < 2; pass++) {
+        int64_t k = 0;
+        for (int a = 0; a < count; a++) {
+            if (pass == 1) succ_off[a] = (int32_t)k;
+            for (int b = 0; b < count; b++) {
+                if (a == b) continue;
+                int touch = !(bx[4 * a + 2] < bx[4 * b] || bx[4 * b + 2] < bx[4 * a] ||
+                              bx[4 * a + 3] < bx[4 * b + 1] || bx[4 * b + 3] < bx[4 * a + 1]);
+                if (!touch) continue;
+                int a_first = is_root[a] ? 1 : (is_root[b] ? 0 : a < b);
+                if (!a_first) continue;                       /* the edge is b -> a */
+                if (pass == 1 && k < cap) succ[k] = b;
+                k++;
+            }
+        }
+        if (pass == 1) succ_off[count] = (int32_t)k;
+        ne = k;
+    }
+    *num_edges = ne;
+    free(t); free(bx);
+    return ne > cap ? ORC_RANGE : ORC_OK;
+}

@@ -76,5 +76,11 @@ int orc_route_ex(const orc_grid* g, const orc_nets* n, const int32_t* batch_of_n
                  uint64_t* batch_hash, const orc_pattern* pat, int32_t* zmid);
 int orc_recost_net_ex(const orc_grid* g, const orc_nets* n, int32_t net, const int32_t* demand,
                       const uint32_t* seg, const int32_t* zmid, uint64_t* cost);
+/* rip-up set extraction (violating nets) and overflow totals on a final demand */
+int orc_overflow(const orc_grid* g, const orc_nets* n, const uint32_t* seg, const int32_t* zmid,
+                 const int32_t* demand, uint8_t* violating, int64_t* totals /* [2] */);
+/* ordered task graph of a task set (net ids): task order, root batch, successor CSR */
+int orc_task_graph(const orc_grid* g, const orc_nets* n, const int32_t* tasks, int32_t count, int32_t* order,
+                   uint8_t* is_root, int32_t* succ_off, int32_t* succ, int64_t cap, int64_t* num_edges);
 
 #endif
