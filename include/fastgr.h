@@ -225,6 +225,44 @@ FGR_API fgr_status fgr_run_host_ex(fgr_grid* grid, int32_t num_nets, int32_t num
                                    const int32_t* parent, uint32_t* seg_out, int32_t* zmid_out, uint32_t* net_cost,
                                    int32_t* num_batches, void* stream);
 
+/*
+ * fgr_overflow — rip-up set extraction after a routing stage (§III-A
+ * L398-402 "we first extract the nets to rip up"; §III-G "rewire the
+ * nets with violations").  On the grid's current demand, a wire edge is
+ * overflowed when demand > capacity, and a net is violating when a committed leg
+ * of its route (seg / zmid as written by fgr_route_all(_ex) for `nets`) covers an
+ * overflowed edge (R26).
+ *   seg [num_nodes], zmid [num_nodes] DEVICE in (zmid may be NULL only while the
+ *       grid's pattern is L-only)
+ *   violating [num_nets] DEVICE out: 1 / 0 per net
+ *   rip_ids [num_nets] DEVICE out: the violating net ids, ascending; *num_rip (host) of them
+ *   totals [2] HOST out: overflowed wire edges, sum of (demand - capacity) over them
+ * Synchronises `stream`.  Errors: INVALID, CUDA.  Demand is not modified.
+ */
+FGR_API fgr_status fgr_overflow(fgr_grid* grid, const fgr_nets* nets, const uint32_t* seg, const int32_t* zmid,
+                                uint8_t* violating, int32_t* rip_ids, int32_t* num_rip, int64_t* totals, void* stream);
+
+/*
+ * fgr_task_graph — the ordered task graph of a set of routing tasks (PAPER.md
+ * §III-B, Fig. 6; used for the rip-up tasks, §III-G).
+ * Task IDs are the tasks sorted by (HPWL over all tree nodes, net id) (R12);
+ * two tasks conflict when their closed bounding boxes share a G-cell (R13); the
+ * root task batch is one pass of Algorithm 1 over the task IDs; every
+ * conflicting pair is ordered from the root task to the non-root one, else from
+ * the smaller task ID to the larger (R27).  The result is acyclic.
+ *   tasks [count] DEVICE in: net ids (distinct, any order)
+ *   order [count] DEVICE out: net id of task t
+ *   is_root [count] DEVICE out: 1 if task t is in the root batch
+ *   succ_offset [count+1], succ [capacity] DEVICE out: successors of task t are
+ *       succ[succ_offset[t] .. succ_offset[t+1]), task IDs ascending
+ *   *num_edges (host) = number of directed edges; RANGE if it exceeds capacity
+ *       (succ untouched, succ_offset valid — call again with a larger buffer).
+ * Synchronises `stream`.  Errors: INVALID, RANGE, CUDA.
+ */
+FGR_API fgr_status fgr_task_graph(fgr_grid* grid, const fgr_nets* nets, const int32_t* tasks, int32_t count,
+                                  int32_t* order, uint8_t* is_root, int32_t* succ_offset, int32_t* succ,
+                                  int64_t capacity, int64_t* num_edges, void* stream);
+
 /* Counters of the last fgr_route_all (for the byte model in DESIGN.md §5). */
 typedef struct {
     int64_t refresh_segments;          /* 32-position row/column segments rescanned            */

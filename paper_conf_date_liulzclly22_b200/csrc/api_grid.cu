@@ -243,6 +243,7 @@ extern "C" FGR_API fgr_status fgr_grid_destroy(fgr_grid* g) {
     for (auto& s : g->s_rec) cudaFree(s.p);
     cudaFree(g->s_prep.p);
     for (auto& s : g->s_hyb) cudaFree(s.p);
+    for (auto& s : g->s_rip) cudaFree(s.p);
     for (auto e : g->prof.pool) cudaEventDestroy(e);
     for (int i = 0; i < 3; i++) {
         if (g->side[i]) cudaStreamDestroy(g->side[i]);

@@ -188,6 +188,7 @@ struct fgr_grid {
     int hyb_t1 = 1, hyb_t2 = 0;
     HybState hy;
     Scratch s_hyb[3];
+    Scratch s_rip[6];          // rip-up extraction and task graph (ripup.cu)
 };
 
 // Profiling brackets around a launch (no-ops unless fgr_profile_enable(grid, 1)).

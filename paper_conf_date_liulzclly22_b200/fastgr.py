@@ -26,7 +26,7 @@ EXPORTS = ["fgr_last_error", "fgr_version", "fgr_cost_table", "fgr_grid_create",
            "fgr_grid_set_demand", "fgr_grid_get_demand", "fgr_plan", "fgr_route_batch", "fgr_route_all",
            "fgr_comm_unique_id", "fgr_comm_init", "fgr_run_host", "fgr_get_stats", "fgr_profile_enable",
            "fgr_profile_read", "fgr_split_batch", "fgr_set_pattern", "fgr_route_batch_ex", "fgr_route_all_ex",
-           "fgr_run_host_ex"]
+           "fgr_run_host_ex", "fgr_overflow", "fgr_task_graph"]
 PROF_CLASSES = ["refresh", "dp_small", "dp_large", "commit", "plan_preprocess", "plan_sort", "plan_color",
                 "plan_other", "exchange", "hybrid"]
 # the paper's FastGRH selection window: hybrid L+Z on two-pin HPWL in [100, 500]
@@ -89,6 +89,8 @@ def lib():
             "fgr_route_batch_ex": ([P, P, P, I, P, P, P, P], S),
             "fgr_route_all_ex": ([P, P, P, P, I, P, P, P, P], S),
             "fgr_run_host_ex": ([P, I, I, P, P, P, P, P, P, P, P, P, P, P], S),
+            "fgr_overflow": ([P, P, P, P, P, P, P, P, P], S),
+            "fgr_task_graph": ([P, P, P, I, P, P, P, P, ctypes.c_int64, P, P], S),
         }
         for name, (args, res) in sig.items():
             f = getattr(L, name)
@@ -226,6 +228,23 @@ def fgr_run_host_ex(h, node_offset, x, y, pin_lo, pin_hi, parent, seg_out=None, 
     return nb.value
 
 
+def fgr_overflow(h, nets, seg, zmid, violating, rip_ids, stream=None):
+    """-> (num_rip, (overflowed edges, total overflow)); violating / rip_ids filled on the device."""
+    nr = ctypes.c_int32(0)
+    tot = np.zeros(2, np.int64)
+    _check(lib().fgr_overflow(h, ctypes.byref(nets), _ptr(seg), _ptr(zmid), _ptr(violating), _ptr(rip_ids),
+                              ctypes.byref(nr), tot.ctypes.data, _stream(stream)))
+    return nr.value, (int(tot[0]), int(tot[1]))
+
+
+def fgr_task_graph(h, nets, tasks, count, order, is_root, succ_offset, succ, capacity, stream=None) -> int:
+    """-> number of directed edges (raises FGR_ERR_RANGE when it exceeds capacity)."""
+    ne = ctypes.c_int64(0)
+    _check(lib().fgr_task_graph(h, ctypes.byref(nets), _ptr(tasks), int(count), _ptr(order), _ptr(is_root),
+                                _ptr(succ_offset), _ptr(succ), int(capacity), ctypes.byref(ne), _stream(stream)))
+    return ne.value
+
+
 def fgr_get_stats(h) -> dict:
     s = fgr_stats()
     _check(lib().fgr_get_stats(h, ctypes.byref(s)))
@@ -339,6 +358,36 @@ class Router:
         return (self.batch_of_net[:N].cpu().numpy(), self.num_batches,
                 self.seg[:M].cpu().numpy().view(np.uint32), self.cost[:N].cpu().numpy().view(np.uint32),
                 self.demand().cpu().numpy())
+
+    def overflow(self, stream=None):
+        """Rip-up set of the last route call -> (violating uint8[N], rip_ids int32[R], totals) on the host."""
+        torch = self.torch
+        N = self.d.num_nets
+        viol = torch.empty(max(N, 1), dtype=torch.uint8, device=self.dev)
+        rip = torch.empty(max(N, 1), dtype=torch.int32, device=self.dev)
+        nr, tot = fgr_overflow(self.h, self.nets, self.seg, self.zmid if self.hybrid is not None else None, viol, rip,
+                               stream)
+        return viol[:N].cpu().numpy(), rip[:nr].cpu().numpy(), tot
+
+    def task_graph(self, tasks, stream=None):
+        """Ordered task graph of net ids `tasks` (host array) -> (order, is_root, succ_offset, succ) on the host."""
+        torch = self.torch
+        t = torch.from_numpy(np.ascontiguousarray(tasks, np.int32)).to(self.dev)
+        R = int(t.numel())
+        order = torch.empty(max(R, 1), dtype=torch.int32, device=self.dev)
+        root = torch.empty(max(R, 1), dtype=torch.uint8, device=self.dev)
+        off = torch.empty(R + 1, dtype=torch.int32, device=self.dev)
+        cap = 1 << 16
+        while True:
+            succ = torch.empty(cap, dtype=torch.int32, device=self.dev)
+            try:
+                ne = fgr_task_graph(self.h, self.nets, t, R, order, root, off, succ, cap, stream)
+                break
+            except FgrError as e:
+                if e.status != FGR_ERR_RANGE:
+                    raise
+                cap *= 4
+        return (order[:R].cpu().numpy(), root[:R].cpu().numpy(), off.cpu().numpy(), succ[:ne].cpu().numpy())
 
     def zmids(self):
         """zmid int32[M] (mid | lb << 16 of Z routes, -1 elsewhere) of the last hybrid route call."""
