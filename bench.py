@@ -345,6 +345,35 @@ def main():
                "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h),
                "call": "fgr_run_host (pinned host nets in -> plan -> route_all -> seg/cost out)"}
 
+    # rip-up extraction on the final demand (NEXT #3): the overflow scan streams the whole
+    # demand + capacity arrays once (an HBM-bound kernel), then one warp per net checks its legs
+    ripup = None
+    if world == 1:
+        N = d.num_nets
+        viol = torch.empty(max(N, 1), dtype=torch.uint8, device=dev)
+        rip = torch.empty(max(N, 1), dtype=torch.int32, device=dev)
+        zm = r.zmid if hybrid else None
+        F.fgr_overflow(r.h, r.nets, r.seg, zm, viol, rip)
+        times = []
+        for _ in range(5):
+            flush.zero_()
+            a = torch.cuda.Event(enable_timing=True); b = torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            nr, tot = F.fgr_overflow(r.h, r.nets, r.seg, zm, viol, rip)
+            b.record(stream)
+            b.synchronize()
+            times.append(a.elapsed_time(b))
+        grid_bytes = 0
+        for dr, cnt in ((0, int((d.dir == 0).sum())), (1, int((d.dir == 1).sum()))):
+            W = 4
+            while W < cnt:
+                W *= 2
+            lines, ln = (d.ny, d.nx) if dr == 0 else (d.nx, d.ny)
+            grid_bytes += lines * ln * W * 5   # int32 demand + uint8 capacity per slot
+        ms = statistics.median(times)
+        ripup = {"ms": ms, "violating_nets": nr, "overflowed_edges": tot[0], "total_overflow": tot[1],
+                 "scan_bytes": grid_bytes, "note": "fgr_overflow device time incl. the per-net check and compaction"}
+
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         cpu = cpu_baseline(d, args.config, hybrid=hybrid)
@@ -369,6 +398,7 @@ def main():
             "kernels_ms_per_step": {c: v[0] / steps for c, v in prof.items() if v[1]},
             "kernels_launches_per_step": {c: v[1] / steps for c, v in prof.items() if v[1]},
             "refresh_segments_per_step": stats["refresh_segments"],
+            "ripup": ripup,
             "wall_s": t_wall,
         }
         print(json.dumps(line), flush=True)
