@@ -17,9 +17,11 @@ CFLAGS  := -O2 -std=c11 -fPIC -Wall -Wextra -Wno-unused-parameter
 
 KERN_SRC := $(wildcard $(CSRC)/*.cu)
 KERN_HDR := $(wildcard $(CSRC)/*.cuh) include/fastgr.h
-KERN_OBJ := $(patsubst $(CSRC)/%.cu,build/%.o,$(KERN_SRC))
+BUILD   ?= build
+LIB     ?= $(PKG)/libfastgr.so
+KERN_OBJ := $(patsubst $(CSRC)/%.cu,$(BUILD)/%.o,$(KERN_SRC))
 
-all: gen/libfgrgen.so oracle/liboracle.so $(PKG)/libfastgr.so
+all: gen/libfgrgen.so oracle/liboracle.so $(LIB)
 
 gen/libfgrgen.so: gen/fgr_gen.c
 	$(CC) $(CFLAGS) -shared -o $@ $< -lm
@@ -27,11 +29,11 @@ gen/libfgrgen.so: gen/fgr_gen.c
 oracle/liboracle.so: oracle/fgr_oracle.c oracle/fgr_oracle.h
 	$(CC) $(CFLAGS) -shared -o $@ oracle/fgr_oracle.c -lm
 
-build/%.o: $(CSRC)/%.cu $(KERN_HDR)
-	@mkdir -p build
-	$(NVCC) $(NVFLAGS) -c -o $@ $< 2> build/$*.ptxas.txt || (cat build/$*.ptxas.txt; false)
+$(BUILD)/%.o: $(CSRC)/%.cu $(KERN_HDR)
+	@mkdir -p $(BUILD)
+	$(NVCC) $(NVFLAGS) -c -o $@ $< 2> $(BUILD)/$*.ptxas.txt || (cat $(BUILD)/$*.ptxas.txt; false)
 
-$(PKG)/libfastgr.so: $(KERN_OBJ)
+$(LIB): $(KERN_OBJ)
 	$(NVCC) $(ARCH) -shared -o $@ $(KERN_OBJ) -L$(NCCL_LIB) -l:libnccl.so.2 \
 	    -Xlinker -rpath=$(NCCL_LIB) -Xcompiler -fPIC
 

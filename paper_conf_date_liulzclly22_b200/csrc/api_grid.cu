@@ -218,7 +218,7 @@ extern "C" FGR_API fgr_status fgr_grid_create(const fgr_grid_desc* d, int device
     if (e != cudaSuccess) { fgr_grid_destroy(g); return fgr_cuda_fail(nullptr, e, "grid init"); }
     g->full_dirty = true;
     bool sok = cudaEventCreateWithFlags(&g->ev_fork, cudaEventDisableTiming) == cudaSuccess;
-    for (int i = 0; i < 3 && sok; i++)
+    for (int i = 0; i < FGR_SIDE_STREAMS && sok; i++)
         sok = cudaStreamCreateWithFlags(&g->side[i], cudaStreamNonBlocking) == cudaSuccess &&
               cudaEventCreateWithFlags(&g->ev_join[i], cudaEventDisableTiming) == cudaSuccess;
     if (!sok) {
@@ -245,7 +245,7 @@ extern "C" FGR_API fgr_status fgr_grid_destroy(fgr_grid* g) {
     for (auto& s : g->s_hyb) cudaFree(s.p);
     for (auto& s : g->s_rip) cudaFree(s.p);
     for (auto e : g->prof.pool) cudaEventDestroy(e);
-    for (int i = 0; i < 3; i++) {
+    for (int i = 0; i < FGR_SIDE_STREAMS; i++) {
         if (g->side[i]) cudaStreamDestroy(g->side[i]);
         if (g->ev_join[i]) cudaEventDestroy(g->ev_join[i]);
     }
@@ -256,6 +256,7 @@ extern "C" FGR_API fgr_status fgr_grid_destroy(fgr_grid* g) {
     free(g->cache.h_segb);
     free(g->cache.h_ntwo);
     free(g->cache.h_n9);
+    free(g->cache.h_lsplit);
     delete g;
     return FGR_OK;
 }

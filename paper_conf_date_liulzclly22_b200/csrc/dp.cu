@@ -24,22 +24,15 @@
 // All prefix gathers of a net are issued up front (costs are fixed during the
 // DP); the per-node tables live in shared memory; each min-plus step is a DPX
 // VIADDMNMX (sat_add).  Tie-breaks follow reading R11 exactly.
-#include "fgr_internal.cuh"
+#include "dp_common.cuh"
 
 namespace {
 
 constexpr int kGroupWarps = 4;              // warps per CTA in k_dp_group
-constexpr int kLargeWarps = 16;             // warps per CTA in k_dp_large (one path-walking group each)
+constexpr int kLargeWarps = 16;
+constexpr int kFlowMax = 128;               // largest net of the dataflow kernel by default             // warps per CTA in k_dp_large (one path-walking group each)
 
-__host__ __device__ constexpr int groups_of(int LT) { return (32 / LT) < 4 ? (32 / LT) : 4; }
-__host__ __device__ inline size_t a16(size_t b) { return (b + 15) & ~(size_t)15; }
 
-struct Hdr {                  // per-block constants copied to shared memory
-    uint32_t viapre[FGR_MAXL + 1];
-    uint8_t dir[FGR_MAXL];
-    uint8_t slot[FGR_MAXL];
-    uint8_t zlo[FGR_MAXL];    // smallest lo with V(lo, a) == 0 (zero-cost via run below a)
-};
 
 struct Tabs {
     uint32_t* E;      // [m][LT]      E_v(lt) = c*(v -> parent, lt)
@@ -133,25 +126,7 @@ __device__ inline WScr carve_wscr(unsigned char* p, int L) {
     return w;
 }
 
-__device__ inline void init_hdr(Hdr* h, const GridView& g) {
-    for (int i = threadIdx.x; i <= FGR_MAXL; i += blockDim.x) h->viapre[i] = g.viapre[i];
-    for (int i = threadIdx.x; i < FGR_MAXL; i += blockDim.x) {
-        h->dir[i] = g.dir[i];
-        h->slot[i] = g.slot[i];
-        int z = i;
-        while (z > 0 && g.viapre[z - 1] == g.viapre[i]) z--;
-        h->zlo[i] = (uint8_t)z;
-    }
-}
 
-struct Out {
-    uint32_t* seg;        // [num_nodes] by global node index (direct mode)
-    uint32_t* cost;       // [num_nets] by net id (direct mode)
-    uint32_t* rec_seg;    // record mode: rec_seg[rec_off[list_base + idx] + local]
-    const int32_t* rec_off;
-    uint32_t* rec_cost;   // record mode: rec_cost[list_base + idx]
-    int list_base;
-};
 
 // Per-lane constants of the group lane that owns layer `gl` (= lo in the K rows, = lt in the edge step).
 template <int LT>
@@ -179,29 +154,6 @@ struct LaneConst {
     }
 };
 
-// ------------------------------------------------------------- leg gathers
-// Cost of the leg from position a to b (a < b) on `line` for every slot:
-// (SB[seg(b)] + P[b]) - (SB[seg(a)] + P[a]), exact in uint32 (R19).
-__device__ __forceinline__ void leg_cost(const DirView& d, int line, int a, int b, uint32_t* out) {
-    const size_t pa = ((size_t)line * d.len + a) * d.W, pb = ((size_t)line * d.len + b) * d.W;
-    const size_t sa = ((size_t)line * d.nseg + (a >> FGR_SEG_SHIFT)) * d.W;
-    const size_t sb = ((size_t)line * d.nseg + (b >> FGR_SEG_SHIFT)) * d.W;
-    const int nq = d.W >> 2;
-#pragma unroll
-    for (int q = 0; q < 4; q++) {
-        if (q < nq) {
-            uint4 Pa = __ldg(reinterpret_cast<const uint4*>(d.P + pa) + q);
-            uint4 Pb = __ldg(reinterpret_cast<const uint4*>(d.P + pb) + q);
-            uint4 Sa = __ldg(reinterpret_cast<const uint4*>(d.SB + sa) + q);
-            uint4 Sb = __ldg(reinterpret_cast<const uint4*>(d.SB + sb) + q);
-            uint32_t r[4] = {(Sb.x + Pb.x) - (Sa.x + Pa.x), (Sb.y + Pb.y) - (Sa.y + Pa.y),
-                             (Sb.z + Pb.z) - (Sa.z + Pa.z), (Sb.w + Pb.w) - (Sa.w + Pa.w)};
-#pragma unroll
-            for (int k = 0; k < 4; k++)
-                if (4 * q + k < d.cnt) out[4 * q + k] = r[k];
-        }
-    }
-}
 
 // task = 4*(i-1) + type for node i >= 1: 0 = H row y_v, 1 = H row y_u, 2 = V col x_v, 3 = V col x_u
 __device__ __forceinline__ void gather_task(const GridView& g, const Tabs& t, int task) {
@@ -221,22 +173,6 @@ __device__ __forceinline__ void gather_task(const GridView& g, const Tabs& t, in
 }
 
 // ------------------------------------------------------------- DP steps (one group of LT lanes)
-// Bend field of a chosen route: 0/1 = the L shapes (bend 0 when lt is vertical); a
-// departure and arrival layer of the same direction on a bent edge is a Z shape of a
-// hybrid edge: 2 = HVH, 3 = VHV (§III-E).
-__device__ __forceinline__ uint32_t seg_bend(int dls, int dlt, bool straight) {
-    if (straight) return 0u;
-    if (dls == dlt) return dls == 0 ? 2u : 3u;
-    return dlt == 1 ? 0u : 1u;
-}
-
-// Z argmin (mid | lb << 16) of a chosen Z route of global node gv, or 0 for an L shape.
-__device__ __forceinline__ uint32_t hyb_z(const HybView& hy, int gv, uint32_t seg, int L) {
-    if ((seg & 0xFF) < 2 || !hy.net) return 0u;
-    const int s = hy.slot[gv];
-    const int ls = (seg >> 8) & 0xFF, lt = (seg >> 16) & 0xFF;
-    return hy.A[((size_t)s * L + lt) * L + ls];
-}
 
 // S5: child layer = smallest l in the parent's span minimising E_v(l) (R11).
 template <int LT>
@@ -257,47 +193,6 @@ __device__ __forceinline__ uint32_t backtrack_node(const Hdr* h, const Tabs& t, 
     return bend | ((uint32_t)ls << 8) | ((uint32_t)lt << 16) | ((uint32_t)straight << 24);
 }
 
-// S6: +1 on every unit edge of a leg (fire-and-forget RED), and mark the touched
-// 32-position segments and their line stale for the next refresh (plain byte stores).
-__device__ __forceinline__ void commit_leg(const GridView& g, const DirView& d, int line, int a, int b, int sl) {
-    if (a >= b) return;
-    int32_t* D = d.D + (size_t)line * d.len * d.W + sl;
-    for (int p = a; p < b; p++) atomicAdd(D + (size_t)p * d.W, 1);
-    const int s0 = a >> FGR_SEG_SHIFT, s1 = (b - 1) >> FGR_SEG_SHIFT;
-    uint8_t* f = g.dseg + d.seg_base + (size_t)line * d.nseg;
-    for (int s = s0; s <= s1; s++) f[s] = 1;
-    g.dline[d.line_base + line] = 1;
-}
-
-__device__ __forceinline__ void commit_edge(const GridView& g, const Hdr* h, int xv, int yv, int xu, int yu, uint32_t seg,
-                                            uint32_t z) {
-    const int bend = seg & 0xFF, ls = (seg >> 8) & 0xFF, lt = (seg >> 16) & 0xFF, straight = (seg >> 24) & 0xFF;
-    if (straight) {
-        if (yv == yu) commit_leg(g, g.h, yv, min(xv, xu), max(xv, xu), h->slot[lt]);
-        else commit_leg(g, g.v, xv, min(yv, yu), max(yv, yu), h->slot[lt]);
-        return;
-    }
-    if (bend >= 2) {   // Z shape (hybrid edge): three legs through Bs and Bt, middle layer lb
-        const int mid = (int)(z & 0xFFFF), lb = (int)((z >> 16) & 0xFF);
-        if (bend == 2) {   // HVH: row y_v to xm (ls), column xm (lb), row y_u from xm (lt)
-            commit_leg(g, g.h, yv, min(xv, mid), max(xv, mid), h->slot[ls]);
-            commit_leg(g, g.v, mid, min(yv, yu), max(yv, yu), h->slot[lb]);
-            commit_leg(g, g.h, yu, min(mid, xu), max(mid, xu), h->slot[lt]);
-        } else {           // VHV: column x_v to ym (ls), row ym (lb), column x_u from ym (lt)
-            commit_leg(g, g.v, xv, min(yv, mid), max(yv, mid), h->slot[ls]);
-            commit_leg(g, g.h, mid, min(xv, xu), max(xv, xu), h->slot[lb]);
-            commit_leg(g, g.v, xu, min(mid, yu), max(mid, yu), h->slot[lt]);
-        }
-        return;
-    }
-    if (bend == 0) {   // H on row y_v (layer ls), V on col x_u (layer lt)
-        commit_leg(g, g.h, yv, min(xv, xu), max(xv, xu), h->slot[ls]);
-        commit_leg(g, g.v, xu, min(yv, yu), max(yv, yu), h->slot[lt]);
-    } else {           // V on col x_v (layer ls), H on row y_u (layer lt)
-        commit_leg(g, g.v, xv, min(yv, yu), max(yv, yu), h->slot[ls]);
-        commit_leg(g, g.h, yu, min(xv, xu), max(xv, xu), h->slot[lt]);
-    }
-}
 
 // Packed G entry of a node without light children (K = V): value V(a,b), span (zlo[a], b).
 __device__ __forceinline__ unsigned long long gclosed(const Hdr* h, int a, int b) {
@@ -438,29 +333,6 @@ __device__ __forceinline__ unsigned long long node_step_group(const Hdr* h, cons
 }
 
 // ------------------------------------------------------------- group kernel (nets <= 32 nodes)
-// Flattened (group, item) iteration: item counts per group n[q]; returns the group of item `it`.
-template <int G>
-struct Flat {
-    int pre[G + 1];
-    __device__ __forceinline__ void build(const int (&n)[G]) {
-        pre[0] = 0;
-#pragma unroll
-        for (int q = 0; q < G; q++) pre[q + 1] = pre[q] + n[q];
-    }
-    __device__ __forceinline__ int total() const { return pre[G]; }
-    __device__ __forceinline__ int group(int it) const {
-        int q = 0;
-#pragma unroll
-        for (int k = 1; k < G; k++) q += (it >= pre[k]) ? 1 : 0;
-        return q;
-    }
-    __device__ __forceinline__ int base(int q) const {
-        int b = 0;
-#pragma unroll
-        for (int k = 0; k < G; k++) b = (k == q) ? pre[k] : b;
-        return b;
-    }
-};
 
 template <int LT, int kMC>
 __global__ void __launch_bounds__(32 * kGroupWarps) k_dp_group(GridView g, NetsView nv, const int32_t* __restrict__ list,
@@ -1530,9 +1402,29 @@ size_t smem_large(int L, int nH, int nV, int m) {
            (size_t)kMR * L * ((L + 3) & ~3) * 4;
 }
 
+// FGR_LARGE_KERNEL=old / FGR_GROUP_KERNEL=old select the previous lane-group kernel for nets of 3..32 nodes (A/B runs).
+bool use_old_large() {
+    static int v = -1;
+    if (v < 0) {
+        const char* s = getenv("FGR_LARGE_KERNEL");
+        v = (s && s[0] == 'o') ? 1 : 0;
+    }
+    return v == 1;
+}
+
+bool use_old_group() {
+    static int v = -1;
+    if (v < 0) {
+        const char* s = getenv("FGR_GROUP_KERNEL");
+        v = (s && s[0] == 'o') ? 1 : 0;
+    }
+    return v == 1;
+}
+
 template <int LT>
 cudaError_t launch_lt(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int nlarge, int nmidL,
-                      int nmidS, int ntwo, int maxm_large, const Out& o, bool commit, const Prep& prep) {
+                      int nmidS, int ntwo, int maxm_large, const Out& o, bool commit, const Prep& prep,
+                      const int* lsplit) {
     static bool configured = false;   // one device per process is the supported configuration
     if (!configured) {
         cudaFuncAttributes fa;
@@ -1557,65 +1449,86 @@ cudaError_t launch_lt(fgr_grid* g, cudaStream_t st, const NetsView& nv, const in
     }
     const GridView& v = g->view;
     const HybView hyv = g->hy.view();
-    // The four size classes of one batch are independent: each non-empty class gets its
-    // own stream (forked from and joined back into the caller's stream).
-    const int cls_n[4] = {nlarge, nmidL, nmidS, ntwo};
-    int used = 0;
-    for (int k = 0; k < 4; k++) used += cls_n[k] > 0;
-    const bool fork = used > 1;
+    // Launch units: large-net size buckets 0..4 (the list is in descending size: > 512,
+    // 257..512, 129..256, 65..128, 33..64 nodes; one bucket unless lsplit is given), then
+    // the classes 9..32, 3..8 and 2 nodes.  Units are independent nets: each non-empty
+    // unit gets its own stream (forked from and joined back into the caller's stream).
+    static const int kCap[5] = {1 << 30, 512, 256, 128, 64};
+    int cut[6] = {0, nlarge, nlarge, nlarge, nlarge, nlarge};
+    if (lsplit && !use_old_large())
+        for (int s = 1; s <= 4; s++) cut[s] = max(cut[s - 1], min(lsplit[s - 1], nlarge));
+    struct Unit { int kind, off, n, cap; };   // kind: 0 large, 1 midL, 2 midS, 3 two
+    Unit units[8];
+    int nu = 0;
+    for (int s = 0; s < 5; s++)
+        if (cut[s + 1] > cut[s]) units[nu++] = Unit{0, cut[s], cut[s + 1] - cut[s], min(kCap[s], maxm_large)};
+    if (nmidL > 0) units[nu++] = Unit{1, nlarge, nmidL, 0};
+    if (nmidS > 0) units[nu++] = Unit{2, nlarge + nmidL, nmidS, 0};
+    if (ntwo > 0) units[nu++] = Unit{3, nlarge + nmidL + nmidS, ntwo, 0};
+    const bool fork = nu > 1;
     cudaError_t e;
     if (fork) {
-        // recorded before any launch: the side streams wait for the refresh, not for the large class
+        // recorded before any launch: the side streams wait for the refresh, not for each other
         if ((e = cudaEventRecord(g->ev_fork, st)) != cudaSuccess) return e;
-        for (int i = 0; i < 3; i++)
+        for (int i = 0; i + 1 < nu; i++)
             if ((e = cudaStreamWaitEvent(g->side[i], g->ev_fork, 0)) != cudaSuccess) return e;
     }
-    cudaStream_t sk[4] = {st, fork ? g->side[0] : st, fork ? g->side[1] : st, fork ? g->side[2] : st};
-    int base = 0;
-    for (int k = 0; k < 4; k++) {
-        const int n = cls_n[k];
-        if (n > 0) {
-            Out os = o;
-            os.list_base = o.list_base + base;
-            const int32_t* l = list + base;
-            const int ps = fgr_prof_begin(g, k == 0 ? PROF_DP_LARGE : PROF_DP_SMALL, sk[k]);
-            if (k == 0) {
-                // programmatic dependent launch: the prologue overlaps the refresh that precedes it
-                cudaLaunchConfig_t cfg = {};
-                cfg.gridDim = dim3(n);
-                cfg.blockDim = dim3(32 * kLargeWarps);
-                cfg.dynamicSmemBytes = smem_large(LT, g->nH, g->nV, maxm_large);
-                cfg.stream = sk[k];
-                cudaLaunchAttribute at[1];
-                at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-                at[0].val.programmaticStreamSerializationAllowed = 1;
-                cfg.attrs = at;
-                cfg.numAttrs = 1;
-                e = cudaLaunchKernelEx(&cfg, k_dp_large<LT>, v, nv, l, n, os, commit ? 1 : 0, prep, hyv);
+    // Nets of up to kFlowMax nodes take the dataflow kernel (dp_walk.cu); bigger ones the
+    // heavy-path kernel below, whose root-path transfer matrices shorten the long chains
+    // (measured on t9: equal step time, lower latency for 33..128-node nets).  FGR_FLOW_MAX
+    // overrides the cut for A/B runs.
+    static int flow_cap = -1;
+    if (flow_cap < 0) { const char* s = getenv("FGR_FLOW_MAX"); flow_cap = s ? atoi(s) : kFlowMax; }
+    for (int ui = 0; ui < nu; ui++) {
+        const Unit& un = units[ui];
+        cudaStream_t su = ui == 0 ? st : g->side[ui - 1];
+        Out os = o;
+        os.list_base = o.list_base + un.off;
+        const int32_t* l = list + un.off;
+        const int n = un.n;
+        const int ps = fgr_prof_begin(g, un.kind == 0 ? PROF_DP_LARGE : PROF_DP_SMALL, su);
+        if (un.kind == 0 && !use_old_large() && un.cap <= fgr_flow_max_nodes(g) && un.cap <= flow_cap) {
+            e = fgr_launch_flow(g, su, nv, l, n, un.cap, os, commit, prep);
+            if (e != cudaSuccess) return e;
+        } else if (un.kind == 0) {
+            // programmatic dependent launch: the prologue overlaps the refresh that precedes it
+            cudaLaunchConfig_t cfg = {};
+            cfg.gridDim = dim3(n);
+            cfg.blockDim = dim3(32 * kLargeWarps);
+            cfg.dynamicSmemBytes = smem_large(LT, g->nH, g->nV, un.cap);
+            cfg.stream = su;
+            cudaLaunchAttribute at[1];
+            at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+            at[0].val.programmaticStreamSerializationAllowed = 1;
+            cfg.attrs = at;
+            cfg.numAttrs = 1;
+            e = cudaLaunchKernelEx(&cfg, k_dp_large<LT>, v, nv, l, n, os, commit ? 1 : 0, prep, hyv);
+            if (e != cudaSuccess) return e;
+        } else if (un.kind <= 2) {
+            if (use_old_group()) {
+                const int per_cta = kGroupWarps * groups_of(LT);
+                if (un.kind == 1)
+                    k_dp_group<LT, FGR_SMALL_NET><<<(n + per_cta - 1) / per_cta, 32 * kGroupWarps,
+                                                     smem_group(LT, g->nH, g->nV, FGR_SMALL_NET), su>>>(
+                        v, nv, l, n, os, commit ? 1 : 0, hyv);
+                else
+                    k_dp_group<LT, FGR_MID_NET><<<(n + per_cta - 1) / per_cta, 32 * kGroupWarps,
+                                                   smem_group(LT, g->nH, g->nV, FGR_MID_NET), su>>>(
+                        v, nv, l, n, os, commit ? 1 : 0, hyv);
+            } else {
+                e = fgr_launch_walk(g, su, nv, l, n, un.kind == 1 ? FGR_SMALL_NET : FGR_MID_NET, os, commit);
                 if (e != cudaSuccess) return e;
             }
-            else if (k == 1) {
-                const int per_cta = kGroupWarps * groups_of(LT);
-                k_dp_group<LT, FGR_SMALL_NET><<<(n + per_cta - 1) / per_cta, 32 * kGroupWarps,
-                                                 smem_group(LT, g->nH, g->nV, FGR_SMALL_NET), sk[k]>>>(v, nv, l, n, os,
-                                                                                                      commit ? 1 : 0, hyv);
-            } else if (k == 2) {
-                const int per_cta = kGroupWarps * groups_of(LT);
-                k_dp_group<LT, FGR_MID_NET><<<(n + per_cta - 1) / per_cta, 32 * kGroupWarps,
-                                               smem_group(LT, g->nH, g->nV, FGR_MID_NET), sk[k]>>>(v, nv, l, n, os,
-                                                                                                  commit ? 1 : 0, hyv);
-            } else {
-                k_dp_two<LT><<<(n + kTwoThreads - 1) / kTwoThreads, kTwoThreads, 0, sk[k]>>>(v, nv, l, n, os,
-                                                                                              commit ? 1 : 0, hyv);
-            }
-            fgr_prof_end(g, ps, sk[k]);
-            g->stats.kernel_launches++;
-            if ((e = cudaGetLastError()) != cudaSuccess) return e;
+        } else {
+            k_dp_two<LT><<<(n + kTwoThreads - 1) / kTwoThreads, kTwoThreads, 0, su>>>(v, nv, l, n, os, commit ? 1 : 0,
+                                                                                      hyv);
         }
-        base += n;
+        fgr_prof_end(g, ps, su);
+        g->stats.kernel_launches++;
+        if ((e = cudaGetLastError()) != cudaSuccess) return e;
     }
     if (fork) {
-        for (int i = 0; i < 3; i++) {
+        for (int i = 0; i + 1 < nu; i++) {
             if ((e = cudaEventRecord(g->ev_join[i], g->side[i])) != cudaSuccess) return e;
             if ((e = cudaStreamWaitEvent(st, g->ev_join[i], 0)) != cudaSuccess) return e;
         }
@@ -1631,14 +1544,15 @@ size_t fgr_dp_smem_large(const fgr_grid* g, int m) { return smem_large(g->L, g->
 
 cudaError_t fgr_launch_dp(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int nlarge, int nmidL,
                           int nmidS, int ntwo, int maxm_large, uint32_t* seg_out, uint32_t* cost_out, uint32_t* rec_seg,
-                          const int32_t* rec_off, uint32_t* rec_cost, int list_base, bool commit, const Prep* prep) {
+                          const int32_t* rec_off, uint32_t* rec_cost, int list_base, bool commit, const Prep* prep,
+                          const int* lsplit) {
     const Prep pz = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
     const Prep& pp = prep ? *prep : pz;
     Out o;
     o.seg = seg_out; o.cost = cost_out; o.rec_seg = rec_seg; o.rec_off = rec_off; o.rec_cost = rec_cost;
     o.list_base = list_base;
     switch (g->L) {
-#define FGR_LT(n) case n: return launch_lt<n>(g, st, nv, list, nlarge, nmidL, nmidS, ntwo, maxm_large, o, commit, pp);
+#define FGR_LT(n) case n: return launch_lt<n>(g, st, nv, list, nlarge, nmidL, nmidS, ntwo, maxm_large, o, commit, pp, lsplit);
         FGR_LT(2) FGR_LT(3) FGR_LT(4) FGR_LT(5) FGR_LT(6) FGR_LT(7) FGR_LT(8) FGR_LT(9) FGR_LT(10) FGR_LT(11)
         FGR_LT(12) FGR_LT(13) FGR_LT(14) FGR_LT(15) FGR_LT(16)
 #undef FGR_LT

@@ -32,6 +32,7 @@
 #define FGR_MAXL 16
 #define FGR_SMALL_NET 32    // nets with <= this many nodes take the lane-group path
 #define FGR_MID_NET 8       // ... with a node capacity of 8 (3..8 nodes) or 32 (9..32 nodes)
+#define FGR_SIDE_STREAMS 7
 #define FGR_CTA_THREADS 256
 #define FGR_WARPS_PER_CTA (FGR_CTA_THREADS / 32)
 
@@ -129,6 +130,7 @@ struct PlanCache {
     int* h_maxm = nullptr;     // [B] max nodes of a large net in the batch
     int* h_ntwo = nullptr;     // [B] 2-node nets (the tail of each batch in exec order)
     int* h_n9 = nullptr;       // [B] nets with 9..32 nodes
+    int* h_lsplit = nullptr;   // [B][4] large nets with more than 512, 256, 128, 64 nodes
     const int32_t* exec = nullptr;  // exec order actually used (order itself, or a re-sorted copy)
     bool prep_valid = false;        // large-net tree analysis computed for these nets
     Prep prep{};
@@ -182,8 +184,9 @@ struct fgr_grid {
     int max_smem = 0;
     int num_sms = 0;
     Profiler prof;
-    cudaStream_t side[3] = {nullptr, nullptr, nullptr};   // size classes of one batch run side by side
-    cudaEvent_t ev_fork = nullptr, ev_join[3] = {nullptr, nullptr, nullptr};
+    // size classes of one batch run side by side: 3 small-net classes + 4 more large-net size buckets
+    cudaStream_t side[FGR_SIDE_STREAMS] = {};
+    cudaEvent_t ev_fork = nullptr, ev_join[FGR_SIDE_STREAMS] = {};
     // hybrid L+Z pattern routing (fgr_set_pattern): edges with t1 <= HPWL <= t2; t1 > t2 = L only
     int hyb_t1 = 1, hyb_t2 = 0;
     HybState hy;
@@ -215,7 +218,7 @@ cudaError_t fgr_launch_refresh_sized(fgr_grid* g, cudaStream_t st, bool full, lo
 cudaError_t fgr_launch_dp(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int nlarge,
                           int nmidL, int nmidS, int ntwo, int maxm_large, uint32_t* seg_out, uint32_t* cost_out,
                           uint32_t* rec_seg, const int32_t* rec_off, uint32_t* rec_cost, int list_base,
-                          bool commit, const Prep* prep);
+                          bool commit, const Prep* prep, const int* lsplit = nullptr);
 cudaError_t fgr_launch_large_prep(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int count,
                                   int maxm, uint16_t* cs, uint16_t* cl, uint16_t* hv, uint16_t* bot, uint16_t* pq,
                                   uint16_t* rpos, int32_t* np);
@@ -227,6 +230,22 @@ fgr_status fgr_hyb_prepare(fgr_grid* g, cudaStream_t st, const NetsView& nv, int
 cudaError_t fgr_launch_hyb_tm(fgr_grid* g, cudaStream_t st, const NetsView& nv, int slot0, int n);
 cudaError_t fgr_launch_hyb_zmid(fgr_grid* g, cudaStream_t st, const uint32_t* seg, int32_t* zmid);
 size_t fgr_dp_smem_large(const fgr_grid* g, int m);
+struct Out;
+cudaError_t fgr_launch_walk(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int n, int mc,
+                            const Out& o, bool commit);
+cudaError_t fgr_launch_flow(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int n, int maxm,
+                            const Out& o, bool commit, const Prep& prep);
+int fgr_flow_max_nodes(const fgr_grid* g);
+
+// Output of a DP launch: direct (by node / net id) or route records (multi-GPU).
+struct Out {
+    uint32_t* seg;        // [num_nodes] by global node index (direct mode)
+    uint32_t* cost;       // [num_nets] by net id (direct mode)
+    uint32_t* rec_seg;    // record mode: rec_seg[rec_off[list_base + idx] + local]
+    const int32_t* rec_off;
+    uint32_t* rec_cost;   // record mode: rec_cost[list_base + idx]
+    int list_base;
+};
 
 static inline NetsView fgr_nets_view(const fgr_nets* n) {
     NetsView v;

@@ -404,7 +404,7 @@ __global__ void k_finalize(int N, const int* __restrict__ counters, const unsign
                            const unsigned long long* __restrict__ bkeys, const int* __restrict__ msize,
                            const int* __restrict__ segb, int* __restrict__ order, int* __restrict__ batch_of_net,
                            int* __restrict__ nlarge, int* __restrict__ maxm, unsigned long long* __restrict__ segsum,
-                           int* __restrict__ ntwo, int* __restrict__ n9) {
+                           int* __restrict__ ntwo, int* __restrict__ n9, int* __restrict__ lsplit) {
     const int i = blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= N) return;
     const int R = N - counters[0];
@@ -416,7 +416,14 @@ __global__ void k_finalize(int N, const int* __restrict__ counters, const unsign
         order[i] = id;
         batch_of_net[id] = c;
         const int m = msize[id];
-        if (m > FGR_SMALL_NET) { atomicAdd(&nlarge[c], 1); atomicMax(&maxm[c], m); }
+        if (m > FGR_SMALL_NET) {
+            atomicAdd(&nlarge[c], 1);
+            atomicMax(&maxm[c], m);
+            if (m > 64) atomicAdd(&lsplit[4 * c + 3], 1);   // large-net size buckets (> 512, 256, 128, 64)
+            if (m > 128) atomicAdd(&lsplit[4 * c + 2], 1);
+            if (m > 256) atomicAdd(&lsplit[4 * c + 1], 1);
+            if (m > 512) atomicAdd(&lsplit[4 * c + 0], 1);
+        }
         // per-batch sum of dirty-segment bounds (refresh launch sizing); keys are
         // batch-sorted, so a warp almost always shares one batch id
         const unsigned long long v = (unsigned long long)segb[id];
@@ -569,14 +576,15 @@ extern "C" FGR_API fgr_status fgr_plan(fgr_grid* g, const fgr_nets* nets, int32_
         FGR_CHECK_CUDA(g, cudaGetLastError());
     }
     // colouring
-    auto* bc = take<int>(g, 11, 5 * ((size_t)R + 1), &e);   // bcount | nlarge | maxm | ntwo | n9
+    auto* bc = take<int>(g, 11, 9 * ((size_t)R + 1), &e);   // bcount | nlarge | maxm | ntwo | n9 | lsplit[4]
     if (e != cudaSuccess) return fgr_cuda_fail(g, e, "plan batch scratch");
     int* d_bcount = bc;
     int* d_nlarge = bc + (R + 1);
     int* d_maxm = bc + 2 * (R + 1);
     int* d_ntwo = bc + 3 * (R + 1);
     int* d_n9 = bc + 4 * (R + 1);
-    FGR_CHECK_CUDA(g, cudaMemsetAsync(bc, 0, 5 * sizeof(int) * ((size_t)R + 1), st));
+    int* d_ls = bc + 5 * (R + 1);
+    FGR_CHECK_CUDA(g, cudaMemsetAsync(bc, 0, 9 * sizeof(int) * ((size_t)R + 1), st));
     FGR_CHECK_CUDA(g, cudaMemsetAsync(color, 0xFF, sizeof(int) * ((size_t)N + 1), st));
     FGR_CHECK_CUDA(g, cudaMemsetAsync(batch_of_net, 0xFF, sizeof(int) * (size_t)N, st));
     if (R > 0) {
@@ -619,7 +627,7 @@ extern "C" FGR_API fgr_status fgr_plan(fgr_grid* g, const fgr_nets* nets, int32_
     auto* segsum = (unsigned long long*)box_r;   // box_r no longer needed after colouring
     FGR_CHECK_CUDA(g, cudaMemsetAsync(segsum, 0, sizeof(unsigned long long) * ((size_t)R + 1), st));
     k_finalize<<<(N + 255) / 256, 256, 0, st>>>(N, counters, keys_s, bkeys_s, msize, segb, order, batch_of_net,
-                                                d_nlarge, d_maxm, segsum, d_ntwo, d_n9);
+                                                d_nlarge, d_maxm, segsum, d_ntwo, d_n9, d_ls);
     FGR_CHECK_CUDA(g, cudaGetLastError());
     g->stats.kernel_launches += 6;
     int B = 0;
@@ -628,7 +636,9 @@ extern "C" FGR_API fgr_status fgr_plan(fgr_grid* g, const fgr_nets* nets, int32_
     PlanCache& c = g->cache;
     if (c.cap < B + 1) {
         free(c.h_off); free(c.h_nlarge); free(c.h_maxm); free(c.h_segb); free(c.h_ntwo); free(c.h_n9);
+        free(c.h_lsplit);
         c.cap = B + 1;
+        c.h_lsplit = (int*)malloc(sizeof(int) * 4 * c.cap);
         c.h_off = (int*)malloc(sizeof(int) * c.cap);
         c.h_nlarge = (int*)malloc(sizeof(int) * c.cap);
         c.h_maxm = (int*)malloc(sizeof(int) * c.cap);
@@ -642,6 +652,7 @@ extern "C" FGR_API fgr_status fgr_plan(fgr_grid* g, const fgr_nets* nets, int32_
         FGR_CHECK_CUDA(g, cudaMemcpy(c.h_maxm, d_maxm, sizeof(int) * B, cudaMemcpyDeviceToHost));
         FGR_CHECK_CUDA(g, cudaMemcpy(c.h_ntwo, d_ntwo, sizeof(int) * B, cudaMemcpyDeviceToHost));
         FGR_CHECK_CUDA(g, cudaMemcpy(c.h_n9, d_n9, sizeof(int) * B, cudaMemcpyDeviceToHost));
+        FGR_CHECK_CUDA(g, cudaMemcpy(c.h_lsplit, d_ls, sizeof(int) * 4 * B, cudaMemcpyDeviceToHost));
         FGR_CHECK_CUDA(g, cudaMemcpy(c.h_segb, segsum, sizeof(long long) * B, cudaMemcpyDeviceToHost));
     }
     c.valid = true;

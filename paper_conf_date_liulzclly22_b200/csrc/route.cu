@@ -51,16 +51,18 @@ __global__ void k_batch_info(int B, const int32_t* __restrict__ boff, const int3
                              const int32_t* __restrict__ off, const int16_t* __restrict__ x,
                              const int16_t* __restrict__ y, const int32_t* __restrict__ par,
                              int* __restrict__ nlarge, int* __restrict__ maxm, unsigned long long* __restrict__ segb,
-                             int* __restrict__ ntwo, int* __restrict__ n9, unsigned long long* __restrict__ keys) {
+                             int* __restrict__ ntwo, int* __restrict__ n9, unsigned long long* __restrict__ keys,
+                             int* __restrict__ lsplit) {
     // one block per batch
     const int b = blockIdx.x;
     if (b >= B) return;
-    int nl = 0, mm = 0, n2 = 0, nn9 = 0;
+    int nl = 0, mm = 0, n2 = 0, nn9 = 0, ls[4] = {0, 0, 0, 0};
     unsigned long long sb = 0;
     for (int i = boff[b] + threadIdx.x; i < boff[b + 1]; i += blockDim.x) {
         const int id = order[i];
         const int a0 = off[id], m = off[id + 1] - a0;
         if (m > FGR_SMALL_NET) { nl++; mm = max(mm, m); }
+        ls[0] += m > 512; ls[1] += m > 256; ls[2] += m > 128; ls[3] += m > 64;
         if (m <= 2) n2++;   // the 2-node kernel also finishes trivial nets
         if (m > FGR_MID_NET && m <= FGR_SMALL_NET) nn9++;
         for (int j = 1; j < m; j++) {
@@ -76,6 +78,7 @@ __global__ void k_batch_info(int B, const int32_t* __restrict__ boff, const int3
     atomicAdd(&segb[b], sb);
     atomicAdd(&ntwo[b], n2);
     atomicAdd(&n9[b], nn9);
+    for (int k = 0; k < 4; k++) atomicAdd(&lsplit[4 * b + k], ls[k]);
 }
 
 __global__ void k_large_list(int n, const int32_t* __restrict__ exec, const int32_t* __restrict__ off,
@@ -189,17 +192,20 @@ static fgr_status batch_info(fgr_grid* g, const fgr_nets* nets, const int32_t* o
     cudaError_t e;
     const int R = 0;   // net count of the batches is read back below
     (void)R;
-    void* p = fgr_scratch(g->s_rec[1], (size_t)B * 24 + 64, &e);
+    void* p = fgr_scratch(g->s_rec[1], (size_t)B * 40 + 64, &e);
     if (e != cudaSuccess) return fgr_cuda_fail(g, e, "batch info scratch");
     unsigned long long* d_segb = (unsigned long long*)p;
     int* d_nl = (int*)(d_segb + B);
     int* d_mm = d_nl + B;
     int* d_n2 = d_mm + B;
     int* d_n9 = d_n2 + B;
-    FGR_CHECK_CUDA(g, cudaMemsetAsync(p, 0, (size_t)B * 24, st));
+    int* d_ls = d_n9 + B;
+    FGR_CHECK_CUDA(g, cudaMemsetAsync(p, 0, (size_t)B * 40, st));
     if (c.cap < B + 1) {
         free(c.h_off); free(c.h_nlarge); free(c.h_maxm); free(c.h_segb); free(c.h_ntwo); free(c.h_n9);
+        free(c.h_lsplit);
         c.cap = B + 1;
+        c.h_lsplit = (int*)malloc(sizeof(int) * 4 * c.cap);
         c.h_n9 = (int*)malloc(sizeof(int) * c.cap);
         c.h_off = (int*)malloc(sizeof(int) * c.cap);
         c.h_nlarge = (int*)malloc(sizeof(int) * c.cap);
@@ -218,7 +224,7 @@ static fgr_status batch_info(fgr_grid* g, const fgr_nets* nets, const int32_t* o
     if (e != cudaSuccess) return fgr_cuda_fail(g, e, "exec order");
     if (B > 0) {
         k_batch_info<<<B, 256, 0, st>>>(B, batch_offset, order, nets->node_offset, nets->x, nets->y, nets->parent,
-                                        d_nl, d_mm, d_segb, d_n2, d_n9, keys);
+                                        d_nl, d_mm, d_segb, d_n2, d_n9, keys, d_ls);
         FGR_CHECK_CUDA(g, cudaGetLastError());
         int bits = 42;
         while ((1LL << (bits - 42)) <= B) bits++;
@@ -234,6 +240,7 @@ static fgr_status batch_info(fgr_grid* g, const fgr_nets* nets, const int32_t* o
         FGR_CHECK_CUDA(g, cudaMemcpyAsync(c.h_segb, d_segb, sizeof(long long) * B, cudaMemcpyDeviceToHost, st));
         FGR_CHECK_CUDA(g, cudaMemcpyAsync(c.h_ntwo, d_n2, sizeof(int) * B, cudaMemcpyDeviceToHost, st));
         FGR_CHECK_CUDA(g, cudaMemcpyAsync(c.h_n9, d_n9, sizeof(int) * B, cudaMemcpyDeviceToHost, st));
+        FGR_CHECK_CUDA(g, cudaMemcpyAsync(c.h_lsplit, d_ls, sizeof(int) * 4 * B, cudaMemcpyDeviceToHost, st));
     }
     FGR_CHECK_CUDA(g, cudaStreamSynchronize(st));
     c.valid = true;
@@ -333,7 +340,8 @@ extern "C" FGR_API fgr_status fgr_route_all_ex(fgr_grid* g, const fgr_nets* nets
             if (hy.active) FGR_CHECK_CUDA(g, fgr_launch_hyb_tm(g, st, nv, hy.boff[b], hy.boff[b + 1] - hy.boff[b]));
             const int o0 = c.h_off[b], cnt = c.h_off[b + 1] - o0, nl = c.h_nlarge[b], n2 = c.h_ntwo[b], n9 = c.h_n9[b];
             FGR_CHECK_CUDA(g, fgr_launch_dp(g, st, nv, c.exec + o0, nl, n9, cnt - nl - n9 - n2, n2, c.h_maxm[b],
-                                            seg_out, net_cost, nullptr, nullptr, nullptr, 0, true, &c.prep));
+                                            seg_out, net_cost, nullptr, nullptr, nullptr, 0, true, &c.prep,
+                                            c.h_lsplit + 4 * b));
         }
         FGR_CHECK_CUDA(g, fgr_launch_hyb_zmid(g, st, seg_out, zmid_out));
         return FGR_OK;

@@ -28,5 +28,5 @@ for b in range(nb):
 F.fgr_profile_enable(r.h, False)
 tot = np.array([x[4:] for x in rows]).sum(0)
 print("totals us: refresh %.0f small %.0f large %.0f" % tuple(tot))
-for x in rows[:12] + rows[12::8]:
+for x in rows:
     print("b=%3d nets=%7d large=%4d maxm=%5d | refresh %7.1f us  small %7.1f us  large %7.1f us" % x)
