@@ -446,19 +446,116 @@ __global__ void __launch_bounds__(32 * WARPS, MC <= 8 ? 8 : 4) k_dp_walk(GridVie
 // exact whatever the order (saturating integer sums and minima commute), so the result is
 // the oracle's.  Backtrack: one thread per node in ascending index, waiting on its
 // parent's span flag (parents first, R22).
+constexpr int kRing = 24;        // root-path transfer matrices in flight (ring slots)
+constexpr int kWalkerMin = 64;   // root paths at least this long get the walker warp
+
 __host__ __device__ inline size_t flow_bytes(int m, int L, int warps) {
     const size_t ES = (size_t)((L + 3) & ~3);
     const size_t scratch = a16(L * ES * 4) + a16(L * ES) + a16(2 * ES * 4);
-    return wtabs_bytes(m, L) + a16((size_t)(m + 1) * 2) + 3 * a16((size_t)m * 2) + a16((size_t)m) +
-           (size_t)warps * groups_of(L) * scratch;
+    return wtabs_bytes(m, L) + a16((size_t)(m + 1) * 2) + 6 * a16((size_t)m * 2) + a16((size_t)m) +
+           (size_t)kRing * L * ES * 4 + (size_t)warps * groups_of(L) * scratch;
 }
+
+
+// Value-only transfer matrix of a root-path node v with heavy child h (the product form of
+// the node and edge steps; exact because saturating min-plus is associative and distributes):
+//   E_v(lt) = min_l [E_h(l) + M_v(l, lt)],  M_v(l, lt) = min_ls [G_v(hull(l, ls, pins)) + W_v(ls, lt)],
+// G_v(a, b) = min over spans [lo, hi] with lo <= a, hi >= b of V(lo, hi) + sum_{light c} min_{[lo,hi]} E_c,
+// W_v = the edge step (legs + bend via, or the hybrid matrix).  Lane lt writes mrow[lt * ES + l].
+template <int LT>
+__device__ __forceinline__ void build_tm(const WLane<LT>& c, const WTabs& t, int v, int heavy, bool act, int gl,
+                                         const uint32_t* hm, const uint16_t* cs, const uint16_t* cl, uint32_t* mrow) {
+    constexpr int ES = WK<LT>::ES;
+    uint32_t acc[LT];
+#pragma unroll
+    for (int hi = 0; hi < LT; hi++) acc[hi] = c.vrow[hi];
+    int ck = act ? cs[v] : 0;
+    const int ce = act ? cs[v + 1] : 0;
+    for (; ck < ce; ck++) {
+        const int ch = cl[ck];
+        if (ch == heavy) continue;
+        const uint4* ep = reinterpret_cast<const uint4*>(t.E + ch * ES);
+        uint32_t e[ES];
+#pragma unroll
+        for (int q = 0; q < ES / 4; q++) {
+            const uint4 w = ep[q];
+            e[4 * q] = w.x; e[4 * q + 1] = w.y; e[4 * q + 2] = w.z; e[4 * q + 3] = w.w;
+        }
+        uint32_t run = FGR_INF;
+#pragma unroll
+        for (int hi = 0; hi < LT; hi++) {
+            run = min(run, hi >= gl ? e[hi] : FGR_INF);
+            acc[hi] = sat_add(acc[hi], run);
+        }
+    }
+    if (act) {   // suffix minima over hi (values only)
+        uint32_t srow[ES];
+#pragma unroll
+        for (int hi = LT; hi < ES; hi++) srow[hi] = FGR_INF;
+        uint32_t sm = FGR_INF;
+#pragma unroll
+        for (int hi = LT - 1; hi >= 0; hi--) { sm = min(sm, acc[hi]); srow[hi] = sm; }
+        uint4* sp = reinterpret_cast<uint4*>(t.S + gl * ES);
+#pragma unroll
+        for (int q = 0; q < ES / 4; q++) sp[q] = make_uint4(srow[4 * q], srow[4 * q + 1], srow[4 * q + 2], srow[4 * q + 3]);
+    }
+    __syncwarp();
+    if (act) {   // G(a, b) = min_{lo <= a} S(lo, b): lane b owns column b
+        uint32_t run = FGR_INF;
+#pragma unroll
+        for (int a = 0; a < LT; a++) { run = min(run, t.S[a * ES + gl]); t.S[a * ES + gl] = run; }
+    }
+    __syncwarp();
+    if (act) {
+        const int u = t.par[v];
+        const bool sh = t.y[v] == t.y[u];
+        const bool straight = sh || t.x[v] == t.x[u];
+        const int edir = sh ? 0 : 1;
+        const uint32_t legB = t.LB[v * ES + gl];
+        uint32_t w[LT];
+#pragma unroll
+        for (int ls = 0; ls < LT; ls++) {
+            if (hm) w[ls] = hm[ls];
+            else if (straight) w[ls] = (ls == gl && c.my_dir == edir) ? t.LA[v * ES + gl] : FGR_INF;
+            else w[ls] = sat_add(sat_add(t.LA[v * ES + ls], c.vmeo[ls]), legB);
+        }
+        const int plo = t.plo[v], phi = t.phi[v];
+        uint32_t col[ES];
+#pragma unroll
+        for (int l = LT; l < ES; l++) col[l] = FGR_INF;
+#pragma unroll
+        for (int l = 0; l < LT; l++) {
+            uint32_t best = FGR_INF;
+#pragma unroll
+            for (int ls = 0; ls < LT; ls++) {
+                int lo = min(l, ls), hi = max(l, ls);
+                if (plo >= 0) { lo = min(lo, plo); hi = max(hi, phi); }
+                best = min(best, sat_add(t.S[lo * ES + hi], w[ls]));
+            }
+            col[l] = best;
+        }
+        uint4* mp = reinterpret_cast<uint4*>(mrow + gl * ES);
+#pragma unroll
+        for (int q = 0; q < ES / 4; q++) mp[q] = make_uint4(col[4 * q], col[4 * q + 1], col[4 * q + 2], col[4 * q + 3]);
+    }
+    __syncwarp();
+}
+
+// Root-path state packed above the pending-children count of a node: atomicSub on the
+// count leaves it alone.  0 pending, 1 building, 2 matrix ready, 3 walker inline, 4 kicked.
+#define FST(w) ((w) >> 16)
+#define FCNT(w) ((w) & 0xFFFFu)
 
 template <int LT, int WARPS>
 __global__ void __launch_bounds__(32 * WARPS) k_dp_flow(GridView g, NetsView nv, const int32_t* __restrict__ list,
                                                          int count, Out o, int commit, Prep prep, HybView hy) {
     constexpr int G = WK<LT>::G, ES = WK<LT>::ES;
     extern __shared__ __align__(16) unsigned char smem[];
-    __shared__ int s_ticket, s_nleaf, s_ticket2, s_ntops;
+    __shared__ int s_ticket, s_nleaf, s_ticket2, s_ntops, s_K, s_wpos, s_wdone, s_kqh, s_kqt;
+#ifdef FGR_TIMING
+    __shared__ long long s_wst[4];   // walker: fast steps, inline steps, cycles waiting for a state, cycles waiting for light children
+    if (threadIdx.x < 4) s_wst[threadIdx.x] = 0;
+#endif
     __shared__ uint32_t s_cost;
     WHdr* wh = reinterpret_cast<WHdr*>(smem);
     init_hdr(&wh->h, g);
@@ -471,7 +568,7 @@ __global__ void __launch_bounds__(32 * WARPS) k_dp_flow(GridView g, NetsView nv,
 #else
 #define FMARK(i) do { } while (0)
 #endif
-    if (tid == 0) { s_ticket = 0; s_nleaf = 0; s_cost = 0; s_ticket2 = 0; s_ntops = 0; }
+    if (tid == 0) { s_ticket = 0; s_nleaf = 0; s_cost = 0; s_ticket2 = 0; s_ntops = 0; s_wpos = 0; s_wdone = 0; s_kqh = 0; s_kqt = 0; }
     const int net = list[blockIdx.x];
     const int a0 = nv.off[net], m = nv.off[net + 1] - a0;
     const int hnet = hy.net ? hy.net[net] : -1;
@@ -482,6 +579,10 @@ __global__ void __launch_bounds__(32 * WARPS) k_dp_flow(GridView g, NetsView nv,
     uint16_t* cl = (uint16_t*)p; p += a16((size_t)m * 2);
     uint16_t* leafq = (uint16_t*)p; p += a16((size_t)m * 2);
     uint16_t* hv = (uint16_t*)p; p += a16((size_t)m * 2);     // heavy child (backtrack paths), 0xFFFF at a leaf
+    uint16_t* rpos = (uint16_t*)p; p += a16((size_t)m * 2);   // index along the root path from its bottom, 0xFFFF off
+    uint16_t* rp = (uint16_t*)p; p += a16((size_t)m * 2);     // root path, bottom first
+    uint16_t* kq = (uint16_t*)p; p += a16((size_t)m * 2);     // kicked matrix builds (walker -> workers)
+    uint32_t* mslots = (uint32_t*)p; p += (size_t)kRing * LT * ES * 4;
     uint8_t* sready = p; p += a16((size_t)m);
     unsigned char* scr = p;
     __syncthreads();
@@ -522,8 +623,38 @@ __global__ void __launch_bounds__(32 * WARPS) k_dp_flow(GridView g, NetsView nv,
     for (int i = tid; i < m; i += T) {
         const uint32_t nc = (uint32_t)(cs[i + 1] - cs[i]);
         hv[i] = prep.hv ? prep.hv[a0 + i] : (nc ? cl[cs[i]] : (uint16_t)0xFFFF);
-        t.cm[i] = nc;   // pending children
-        if (nc == 0) leafq[atomicAdd(&s_nleaf, 1)] = (uint16_t)i;
+        rpos[i] = prep.rpos ? prep.rpos[a0 + i] : (uint16_t)0xFFFF;
+    }
+    __syncthreads();
+    if (!prep.rpos && tid == 0) {   // root path = the heavy chain from the root
+        int k = 0;
+        for (int w = 0; w != 0xFFFF; w = hv[w]) k++;
+        int j = k - 1;
+        for (int w = 0; w != 0xFFFF; w = hv[w]) rpos[w] = (uint16_t)(j--);
+    }
+    __syncthreads();
+    for (int i = tid; i < m; i += T) if (rpos[i] != 0xFFFF) rp[rpos[i]] = (uint16_t)i;
+    if (tid == 0) s_K = rpos[0] + 1;
+    __syncthreads();
+    const int K = s_K;
+    const bool usew = K >= kWalkerMin;   // a root-path walker pays off only on long chains
+    // pending children: all of them off the root path, the light ones on it (the walker owns
+    // the heavy chain).  Work queue: matrix builds of the first root-path nodes without light
+    // children, then the leaves off the root path.
+    if (tid == 0) {
+        int n = 0;
+        for (int k = 1; usew && k < K - 1 && k < kRing; k++) {
+            const int v = rp[k];
+            if (cs[v + 1] - cs[v] == 1) leafq[n++] = (uint16_t)(v | 0x8000);
+        }
+        s_nleaf = n;
+    }
+    __syncthreads();
+    for (int i = tid; i < m; i += T) {
+        const uint32_t nc = (uint32_t)(cs[i + 1] - cs[i]);
+        const bool onrp = usew && rpos[i] != 0xFFFF;
+        t.cm[i] = onrp ? (nc ? nc - 1 : 0) : nc;
+        if (nc == 0 && !onrp) leafq[atomicAdd(&s_nleaf, 1)] = (uint16_t)i;
     }
     FMARK(1);
     pdl_wait();   // the refresh that precedes this launch must be done before the gathers
@@ -565,7 +696,10 @@ __global__ void __launch_bounds__(32 * WARPS) k_dp_flow(GridView g, NetsView nv,
     __syncthreads();
     FMARK(2);
     const int nleaf = s_nleaf;
-    // ---- bottom-up dataflow walks
+    // ---- bottom-up: warp 0 walks the root path with one vector x matrix step per node
+    // (M_v built ahead by the workers, else an inline node step); warps 1.. run the
+    // dataflow over the rest of the tree and build the root-path matrices as soon as a
+    // node's light children are final.
     {
         const int gi = lane / LT < G ? lane / LT : G;
         const int gl = lane - gi * LT;
@@ -582,36 +716,211 @@ __global__ void __launch_bounds__(32 * WARPS) k_dp_flow(GridView g, NetsView nv,
         }
         WLane<LT> c;
         c.load(&wh->h, gl);
-        int cur = -1;
-        bool more = true;
-        for (;;) {
-            if (glane && cur < 0 && more) {
-                int tk = 0;
-                if (gl == 0) tk = atomicAdd(&s_ticket, 1);
-                tk = __shfl_sync(gmask, tk, gbase);
-                if (tk < nleaf) cur = leafq[tk];
-                else more = false;
+        auto hmat = [&](int v) -> const uint32_t* {
+            if (hnet < 0 || v <= 0) return nullptr;
+            const int hs = hy.slot[a0 + v];
+            return hs >= 0 ? hy.M + ((size_t)hs * LT + gl) * LT : nullptr;
+        };
+        // matrix build of root-path node v (index k) by a lane group that claimed it
+        auto build = [&](int v, int k, bool act) {
+            build_tm<LT>(c, tg, v, hv[v], act, gl, act ? hmat(v) : nullptr, cs, cl, mslots + (size_t)(k % kRing) * LT * ES);
+            if (act) __threadfence_block();
+            __syncwarp();
+            if (act && gl == 0) atomicAdd(&t.cm[v], (2u - 1u) << 16);   // state 1 -> 2
+        };
+        // claim the build of root-path node v (k = rpos): state 0 -> 1 if its ring slot is free
+        auto claim = [&](int v, int k, uint32_t from) -> bool {
+            if (k >= *(volatile int*)&s_wpos + kRing) return false;
+            const uint32_t w = *(volatile uint32_t*)&t.cm[v];
+            if (FST(w) != from || FCNT(w) != 0) return false;
+            return atomicCAS(&t.cm[v], w, (1u << 16)) == w;
+        };
+        if (usew && warp == 0) {
+            const bool act = gi == 0;   // one lane group walks; the warp's other lanes idle
+            uint32_t Eprev = 0;
+            (void)Eprev;
+            for (int k = 0; k < K; k++) {
+                const int v = rp[k];
+                if (k == 0) {            // bottom leaf
+                    wstep<LT, true>(c, tg, v, act, false, gl, act ? hmat(v) : nullptr, &s_cost, cs, cl);
+                } else if (k == K - 1) { // the root: wait for its light children, generalised Eq. (4)
+                    while (FCNT(*(volatile uint32_t*)&t.cm[0]) != 0) __nanosleep(20);
+                    __threadfence_block();
+                    wstep<LT, true>(c, tg, 0, act, true, gl, nullptr, &s_cost, cs, cl);
+                } else {
+                    bool fast = false;
+#ifdef FGR_TIMING
+                    const long long tw0 = clock64();
+#endif
+                    for (;;) {
+                        uint32_t w = *(volatile uint32_t*)&t.cm[v];
+                        const uint32_t st = FST(w);
+                        if (st == 2) { fast = true; break; }
+                        if (st == 0 || st == 4) {
+                            uint32_t old = 0;
+                            if (lane == 0) old = atomicCAS(&t.cm[v], w, (w & 0xFFFFu) | (3u << 16));
+                            old = __shfl_sync(0xffffffffu, old, 0);
+                            if (old == w) break;   // inline
+                        }
+                        // st == 1: a worker is building it
+                    }
+                    __threadfence_block();
+#ifdef FGR_TIMING
+                    if (lane == 0) { s_wst[fast ? 0 : 1]++; s_wst[2] += clock64() - tw0; }
+#endif
+                    if (fast) {
+                        if (act) {
+                            const uint4* ep = reinterpret_cast<const uint4*>(t.E + rp[k - 1] * ES);
+                            const uint4* mp = reinterpret_cast<const uint4*>(mslots + (size_t)(k % kRing) * LT * ES + gl * ES);
+                            uint32_t e[ES], mc[ES];
+#pragma unroll
+                            for (int q = 0; q < ES / 4; q++) {
+                                const uint4 a = ep[q], b = mp[q];
+                                e[4 * q] = a.x; e[4 * q + 1] = a.y; e[4 * q + 2] = a.z; e[4 * q + 3] = a.w;
+                                mc[4 * q] = b.x; mc[4 * q + 1] = b.y; mc[4 * q + 2] = b.z; mc[4 * q + 3] = b.w;
+                            }
+                            uint32_t best = FGR_INF;
+#pragma unroll
+                            for (int l = 0; l < LT; l++) best = __viaddmin_u32(e[l], mc[l], best);   // e + m <= 2^32 - 2
+                            t.E[v * ES + gl] = best;
+                        }
+                        __syncwarp();
+                    } else {
+#ifdef FGR_TIMING
+                        const long long tw1 = clock64();
+#endif
+                        while (FCNT(*(volatile uint32_t*)&t.cm[v]) != 0) __nanosleep(20);
+                        __threadfence_block();
+#ifdef FGR_TIMING
+                        if (lane == 0) s_wst[3] += clock64() - tw1;
+#endif
+                        wstep<LT, true>(c, tg, v, act, false, gl, act ? hmat(v) : nullptr, &s_cost, cs, cl);
+                    }
+                }
+                __threadfence_block();
+                __syncwarp();
+                if (lane == 0) {
+                    *(volatile int*)&s_wpos = k + 1;
+                    // the ring slot of k + kRing is free now: kick its build if it was skipped
+                    const int kk = k + kRing;
+                    if (kk < K - 1) {
+                        const int vk = rp[kk];
+                        const uint32_t w = *(volatile uint32_t*)&t.cm[vk];
+                        if (FST(w) == 0 && FCNT(w) == 0 && atomicCAS(&t.cm[vk], w, 4u << 16) == w) {
+                            const int tpos = s_kqt;
+                            kq[tpos] = (uint16_t)vk;
+                            __threadfence_block();
+                            *(volatile int*)&s_kqt = tpos + 1;
+                        }
+                    }
+                }
             }
-            const bool busy = glane && cur >= 0;
-            if (!__any_sync(0xffffffffu, busy)) break;
+            if (lane == 0) { __threadfence_block(); *(volatile int*)&s_wdone = 1; }
+        } else {
+            int cur = -1;          // node to step (walk), or 0x8000 | v for a matrix build
+            bool more = true;      // queue not exhausted (leader's view)
+            bool fin = false;      // no work will come to this group any more
+            for (;;) {
+                if (glane && cur < 0 && !fin) {
+                    // never wait here: a group of this warp may hold a node the walker needs
+                    int tk = -1, f = 0;
+                    if (gl == 0) {
+                        const int h = *(volatile int*)&s_kqh;
+                        if (h < *(volatile int*)&s_kqt) {   // kicked builds first
+                            if (atomicCAS(&s_kqh, h, h + 1) == h) { __threadfence_block(); tk = 0x10000 | kq[h]; }
+                        } else if (more) {
+                            const int q = atomicAdd(&s_ticket, 1);
+                            if (q < nleaf) tk = leafq[q];
+                            else more = false;
+                        } else if ((!usew || *(volatile int*)&s_wdone) && h >= *(volatile int*)&s_kqt) {
+                            f = 1;
+                        }
+                    }
+                    tk = __shfl_sync(gmask, tk, gbase);
+                    fin = __shfl_sync(gmask, f, gbase) != 0;
+                    if (tk >= 0x10000) {   // kicked: state 4 -> 1
+                        const int v = tk & 0xFFFF;
+                        uint32_t ok = 0;
+                        if (gl == 0) ok = atomicCAS(&t.cm[v], 4u << 16, 1u << 16) == (4u << 16);
+                        ok = __shfl_sync(gmask, ok, gbase);
+                        cur = ok ? (0x8000 | v) : -1;
+                    } else if (tk >= 0 && (tk & 0x8000)) {   // queued build: state 0 -> 1
+                        const int v = tk & 0x7FFF;
+                        uint32_t ok = 0;
+                        if (gl == 0) ok = claim(v, rpos[v], 0) ? 1u : 0u;
+                        ok = __shfl_sync(gmask, ok, gbase);
+                        cur = ok ? tk : -1;
+                    } else {
+                        cur = tk;
+                    }
+                }
+                const bool busy = glane && cur >= 0;
+                if (!__any_sync(0xffffffffu, glane && !fin)) break;
+                if (!__any_sync(0xffffffffu, busy)) { __nanosleep(100); continue; }
+                const bool bld = busy && (cur & 0x8000);
+                const int v = busy ? (cur & 0x7FFF) : 0;
+                // the warp's groups may mix builds and node steps: both calls run warp-wide
+                build(v, bld ? rpos[v] : 0, bld);
+                const bool stp = busy && !bld;
+                wstep<LT, true>(c, tg, stp ? v : 0, stp, stp && v == 0, gl, stp ? hmat(v) : nullptr, &s_cost, cs, cl);
+                if (busy) __threadfence_block();
+                __syncwarp();
+                if (busy) {
+                    int nxt = -1;
+                    if (gl == 0 && stp && v != 0) {
+                        const int pu = t.par[v];
+                        if (FCNT(atomicSub(&t.cm[pu], 1u)) == 1u) {   // last child
+                            if (!usew || rpos[pu] == 0xFFFF) nxt = pu;  // continue up
+                            else if (pu != 0 && claim(pu, rpos[pu], 0)) nxt = 0x8000 | pu;   // build its matrix
+                        }
+                    }
+                    nxt = __shfl_sync(gmask, nxt, gbase);
+                    __threadfence_block();
+                    cur = nxt;
+                }
+            }
+        }
+    }
+    __syncthreads();
+    // recE / recB of the root-path nodes the walker passed with a matrix step: independent
+    // node steps now that every E is final (same E values, R11 argmins)
+    {
+        const int gi = lane / LT < G ? lane / LT : G;
+        const int gl = lane - gi * LT;
+        const bool glane = gi < G;
+        const int gbase = (glane ? gi : 0) * LT;
+        const unsigned gmask = glane ? (((1u << LT) - 1u) << gbase) : 0u;
+        WTabs tg = t;
+        {
+            const size_t sz = a16(LT * ES * 4) + a16(LT * ES) + a16(2 * ES * 4);
+            unsigned char* q = scr + (size_t)(warp * G + (glane ? gi : 0)) * sz;
+            tg.S = (uint32_t*)q; q += a16(LT * ES * 4);
+            tg.HA = q; q += a16(LT * ES);
+            tg.BW = (uint32_t*)q;
+        }
+        WLane<LT> c;
+        c.load(&wh->h, gl);
+        if (tid == 0) s_ticket = 0;
+        __syncthreads();
+        for (; usew;) {
+            int k = -1;
+            if (glane && gl == 0) {
+                for (;;) {
+                    const int q = atomicAdd(&s_ticket, 1);
+                    if (q >= K - 2) break;
+                    if (FST(t.cm[rp[q + 1]]) == 2) { k = q + 1; break; }
+                }
+            }
+            if (glane) k = __shfl_sync(gmask, k, gbase);
+            const bool act = glane && k > 0;
+            if (!__any_sync(0xffffffffu, act)) break;
+            const int v = act ? rp[k] : 0;
             const uint32_t* hm = nullptr;
-            if (busy && hnet >= 0 && cur > 0) {
-                const int hs = hy.slot[a0 + cur];
+            if (act && hnet >= 0) {
+                const int hs = hy.slot[a0 + v];
                 if (hs >= 0) hm = hy.M + ((size_t)hs * LT + gl) * LT;
             }
-            wstep<LT, true>(c, tg, busy ? cur : 0, busy, cur == 0, gl, hm, &s_cost, cs, cl);
-            if (busy) __threadfence_block();
-            __syncwarp();
-            if (busy) {
-                int nxt = -1;
-                if (gl == 0 && cur != 0) {
-                    const int pu = t.par[cur];
-                    if (atomicSub(&t.cm[pu], 1u) == 1u) nxt = pu;   // last child: continue with the parent
-                }
-                nxt = __shfl_sync(gmask, nxt, gbase);
-                __threadfence_block();
-                cur = nxt;
-            }
+            wstep<LT, true>(c, tg, v, act, false, gl, hm, &s_cost, cs, cl);
         }
     }
     __syncthreads();
@@ -719,8 +1028,8 @@ __global__ void __launch_bounds__(32 * WARPS) k_dp_flow(GridView g, NetsView nv,
 #ifdef FGR_TIMING
     FMARK(5);
     if (tid == 0 && m > 600)
-        printf("FLOW m=%d leaves=%d tops=%d prologue=%lld gather=%lld forward=%lld backtrack=%lld commit=%lld\n", m, nleaf,
-               ntops, tm[1] - tm[0], tm[2] - tm[1], tm[3] - tm[2], tm[4] - tm[3], tm[5] - tm[4]);
+        printf("FLOW m=%d K=%d fast=%lld inline=%lld wstate=%lld wlight=%lld prologue=%lld gather=%lld forward=%lld backtrack=%lld commit=%lld\n", m, K,
+               s_wst[0], s_wst[1], s_wst[2], s_wst[3], tm[1] - tm[0], tm[2] - tm[1], tm[3] - tm[2], tm[4] - tm[3], tm[5] - tm[4]);
 #endif
 #undef FMARK
 }
