@@ -311,7 +311,21 @@ def main():
         roof = {"bound": "hbm", "kernel": dom, "achieved": ach, "peak": peak, "unit": "GB/s", "frac": ach / peak,
                 "traffic": traffic, "traffic_source": tsrc, "bytes_per_launch": per_launch, "avg_launch_us": avg_s * 1e6,
                 "launches_per_step": dom_n / steps, "share_of_step": dom_ms / steps / ms_per_step,
+                "share_note": "sum of the class's launch durations on their streams / step time; the size classes of a "
+                              "batch run concurrently on side streams, so class shares overlap and can exceed 1",
                 "peak_source": peak_src, "byte_model": unit_note}
+
+    # the streaming kernel beside it: the cost refresh (one launch per batch, alone on the stream)
+    roof_refresh = None
+    if "refresh" in prof and prof["refresh"][1] > 0 and stats.get("refresh_bytes"):
+        r_ms, r_n = prof["refresh"]
+        per_launch = stats["refresh_bytes"] * steps / r_n
+        ach = per_launch / (r_ms / r_n / 1000.0) / 1e9
+        traffic, tsrc = committed_traffic("refresh")
+        roof_refresh = {"bound": "hbm", "kernel": "refresh", "achieved": ach, "peak": peak, "unit": "GB/s",
+                        "frac": ach / peak, "traffic": traffic, "traffic_source": tsrc, "bytes_per_launch": per_launch,
+                        "avg_launch_us": r_ms / r_n * 1e3, "share_of_step": r_ms / steps / ms_per_step,
+                        "byte_model": "per refreshed 32-position segment: 32 x 9 x W bytes (int32 demand + uint8 cap + uint32 prefix)"}
 
     # e2e through the public C ABI with host buffers (pinned), copies inside the timed region
     e2e = None
@@ -394,7 +408,7 @@ def main():
             "plan_ms": statistics.mean(plan_ms), "route_ms": statistics.mean(route_ms),
             "clocks": clk, "e2e": e2e, "gpu_launches": int(launches_total // max(1, steps)),
             "gpu_launches_note": "library kernels per step (CUB sort kernels counted as one launch each call)",
-            "roofline": roof, "cpu_baseline": cpu,
+            "roofline": roof, "roofline_refresh": roof_refresh, "cpu_baseline": cpu,
             "kernels_ms_per_step": {c: v[0] / steps for c, v in prof.items() if v[1]},
             "kernels_launches_per_step": {c: v[1] / steps for c, v in prof.items() if v[1]},
             "refresh_segments_per_step": stats["refresh_segments"],
