@@ -29,8 +29,8 @@
 namespace {
 
 constexpr int kGroupWarps = 4;              // warps per CTA in k_dp_group
-constexpr int kLargeWarps = 16;
-constexpr int kFlowMax = 128;               // largest net of the dataflow kernel by default             // warps per CTA in k_dp_large (one path-walking group each)
+constexpr int kLargeWarps = 16;             // warps per CTA in k_dp_large (one path-walking group each)
+constexpr int kFlowMax = 128;               // largest net of the dataflow kernel by default
 
 
 
