@@ -67,58 +67,51 @@ __device__ __forceinline__ void warp_incl_scan(uint32_t (&x)[W]) {
     }
 }
 
-// Segment data of one lane: demand and capacity of position 32*s + lane, all W slots.
+// One segment, transposed: lane = (slot sl = lane % W, run q = lane / W) owns positions
+// 32*s + q*W .. + W-1 of one slot.  ec = len + T[clamp(cap - dem)] per position, a serial
+// prefix over the run in registers, then an exclusive scan of the run totals across the
+// 32/W runs of the slot (log2(32/W) shuffles); P and ST stored.  Same sums as a per-position
+// warp scan, a third of the instructions.
 template <int W>
-struct SegIn {
-    int4 dem[W / 4];        // demand of the W slots
-    uint32_t cap[W / 4];    // capacities, 4 bytes per word
-};
-
-template <int W>
-__device__ __forceinline__ void load_segment(const DirView& d, int line, int s, SegIn<W>& in) {
-    const int pos = s * FGR_SEG + lane_id();
-    if (pos < d.len) {
-        const size_t base = ((size_t)line * d.len + pos) * W;
-#pragma unroll
-        for (int q = 0; q < W / 4; q++) {
-            in.dem[q] = reinterpret_cast<const int4*>(d.D + base)[q];
-            in.cap[q] = reinterpret_cast<const uint32_t*>(d.C + base)[q];
-        }
-    }
-}
-
-// One segment: ec = len + T[clamp(cap - dem)] per slot, warp scan, write P and ST.
-template <int W>
-__device__ __forceinline__ void scan_segment(const GridView& g, const DirView& d, int dsel, int line, int s,
-                                             const SegIn<W>& in) {
+__device__ __forceinline__ void refresh_segment(const GridView& g, const DirView& d, int dsel, int line, int s) {
     const int lane = lane_id();
-    const int pos = s * FGR_SEG + lane;
-    const bool inb = pos < d.len;
-    const bool edge = pos < d.len - 1;
-    const size_t base = ((size_t)line * d.len + pos) * W;
-    uint32_t ec[W], incl[W];
+    const int sl = lane & (W - 1), q = lane / W;
+    const int p0 = s * FGR_SEG + q * W;
+    const bool slot_ok = sl < d.cnt;
     const int span = 2 * g.S + 1;
+    const int32_t* tab = g.table + (slot_ok ? g.layer_of_slot[dsel][sl] : 0) * span + g.S;
+    const size_t base = ((size_t)line * d.len + p0) * W + sl;
+    int32_t dem[W];
+    uint8_t cap[W];
 #pragma unroll
-    for (int k = 0; k < W; k++) {
+    for (int j = 0; j < W; j++) {
+        const bool ok = slot_ok && p0 + j < d.len - 1;
+        dem[j] = ok ? d.D[base + (size_t)j * W] : 0;
+        cap[j] = ok ? d.C[base + (size_t)j * W] : 0;
+    }
+    uint32_t ec[W], run = 0;
+#pragma unroll
+    for (int j = 0; j < W; j++) {
         uint32_t c = 0;
-        if (edge && k < d.cnt) {
-            const int4 dq = in.dem[k >> 2];
-            const int dm = (k & 3) == 0 ? dq.x : (k & 3) == 1 ? dq.y : (k & 3) == 2 ? dq.z : dq.w;
-            int sl = (int)((in.cap[k >> 2] >> (8 * (k & 3))) & 0xFFu) - dm;
-            sl = sl < -g.S ? -g.S : (sl > g.S ? g.S : sl);
-            c = (uint32_t)g.len_cost + (uint32_t)__ldg(g.table + g.layer_of_slot[dsel][k] * span + sl + g.S);
+        if (slot_ok && p0 + j < d.len - 1) {
+            int sk = (int)cap[j] - dem[j];
+            sk = sk < -g.S ? -g.S : (sk > g.S ? g.S : sk);
+            c = (uint32_t)g.len_cost + (uint32_t)__ldg(tab + sk);
         }
-        ec[k] = c;
-        incl[k] = c;
+        ec[j] = run;   // exclusive prefix inside the run
+        run += c;
     }
-    warp_incl_scan<W>(incl);
-    if (inb) {
-        uint32_t p[W];
+    uint32_t x = run;  // inclusive scan of the run totals over the runs of this slot
 #pragma unroll
-        for (int k = 0; k < W; k++) p[k] = incl[k] - ec[k];
-        Vec<W>::store_u32(d.P + base, p);
+    for (int off = W; off < 32; off <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, x, off);
+        if (lane >= off) x += y;
     }
-    if (lane == 31) Vec<W>::store_u32(d.ST + ((size_t)line * d.nseg + s) * W, incl);
+    const uint32_t before = x - run;
+#pragma unroll
+    for (int j = 0; j < W; j++)
+        if (p0 + j < d.len) d.P[base + (size_t)j * W] = before + ec[j];
+    if (q == 32 / W - 1) d.ST[((size_t)line * d.nseg + s) * W + sl] = x;
 }
 
 // Segment bases of one line: exclusive scan of all its segment totals.
@@ -177,24 +170,12 @@ __device__ __forceinline__ int refresh_chunk(const GridView& g, const DirView& d
         if (chunk >= c0 && chunk < c0 + 32) own = o;
     }
     if (own == 0) return 0;
-    // the loads of up to kInflight dirty segments are issued before any of them is scanned
-    constexpr int kInflight = W >= 16 ? 1 : (W >= 8 ? 2 : 4);
     int done = 0;
     while (own) {
-        int qs[kInflight];
-        SegIn<W> in[kInflight];
-#pragma unroll
-        for (int j = 0; j < kInflight; j++) {
-            qs[j] = own ? __ffs(own) - 1 : -1;
-            if (own) own &= own - 1;
-            if (qs[j] >= 0) load_segment<W>(d, line, chunk * FGR_CHUNK_SEGS + qs[j], in[j]);
-        }
-#pragma unroll
-        for (int j = 0; j < kInflight; j++)
-            if (qs[j] >= 0) {
-                scan_segment<W>(g, d, dsel, line, chunk * FGR_CHUNK_SEGS + qs[j], in[j]);
-                done++;
-            }
+        const int q = __ffs(own) - 1;
+        own &= own - 1;
+        refresh_segment<W>(g, d, dsel, line, chunk * FGR_CHUNK_SEGS + q);
+        done++;
     }
     int last = 0;
     if (lane == 0) {
@@ -214,7 +195,7 @@ __device__ __forceinline__ int refresh_chunk(const GridView& g, const DirView& d
 }
 
 template <int WH, int WV>
-__global__ void __launch_bounds__(256, 3) k_refresh(GridView g, int full) {
+__global__ void __launch_bounds__(256) k_refresh(GridView g, int full) {
     pdl_trigger();   // the next DP kernel may start its prologue now
     pdl_wait();      // the previous batch's commits must be complete
     const int chH = (g.h.nseg + FGR_CHUNK_SEGS - 1) / FGR_CHUNK_SEGS;
