@@ -1180,19 +1180,42 @@ __global__ void __launch_bounds__(32 * kLargeWarps, 1) k_dp_large(GridView g, Ne
 }
 
 // One CTA per large net: the demand-independent tree analysis, written to global memory once per stage.
+// Only the analysis arrays live in shared memory (~38 B/node, not the DP tables), and 256
+// threads at <= 64 registers, so several nets share an SM.
+constexpr int kPrepThreads = 256;
+
+__host__ __device__ inline size_t prep_bytes(int m) {
+    return 2 * a16((size_t)(m + 1) * 4) + 11 * a16((size_t)m * 2) + 2 * a16((size_t)(m + 1) * 2) + 4 * a16((size_t)m);
+}
+
+__device__ inline Tabs carve_prep(unsigned char* p, int m) {
+    Tabs t;
+    t.E = nullptr; t.aux = nullptr; t.recE = nullptr; t.recB = nullptr; t.span = nullptr; t.rp = nullptr; t.argq = nullptr;
+    auto u16 = [&](size_t n) { uint16_t* q = (uint16_t*)p; p += a16(n * 2); return q; };
+    t.legH = (uint32_t*)p; p += a16((size_t)(m + 1) * 4);   // child counts (scratch)
+    t.legV = (uint32_t*)p; p += a16((size_t)(m + 1) * 4);   // level counts (scratch)
+    t.x = (int16_t*)u16(m); t.y = (int16_t*)u16(m); t.par = (int16_t*)u16(m); t.depth = u16(m);
+    t.anc = u16(m); t.hv = u16(m); t.top = u16(m); t.bot = u16(m); t.pq = u16(m); t.rpos = u16(m); t.clist = u16(m);
+    t.cstart = u16(m + 1); t.lvstart = u16(m + 1);
+    t.done = p; p += a16((size_t)m);
+    t.sready = p; p += a16((size_t)m);
+    t.plo = (int8_t*)p; p += a16((size_t)m);
+    t.phi = (int8_t*)p;
+    return t;
+}
+
 template <int LT>
-__global__ void __launch_bounds__(32 * kLargeWarps, 1) k_large_prep(GridView g, NetsView nv, const int32_t* __restrict__ list,
-                                                                    uint16_t* cs, uint16_t* cl, uint16_t* hv, uint16_t* bot,
-                                                                    uint16_t* pq, uint16_t* rpos, int32_t* npaths) {
+__global__ void __launch_bounds__(kPrepThreads, 4) k_large_prep(GridView g, NetsView nv, const int32_t* __restrict__ list,
+                                                                 uint16_t* cs, uint16_t* cl, uint16_t* hv, uint16_t* bot,
+                                                                 uint16_t* pq, uint16_t* rpos, int32_t* npaths) {
     extern __shared__ __align__(16) unsigned char smem[];
     __shared__ int s_maxd, s_npaths, s_deep;
     if (threadIdx.x == 0) { s_maxd = 0; s_npaths = 0; }
-    const int nH = g.h.cnt, nV = g.v.cnt;
     const int warp = threadIdx.x >> 5, lane = lane_id(), tid = threadIdx.x, T = blockDim.x;
     const int net = list[blockIdx.x];
     const int a0 = nv.off[net];
     const int m = nv.off[net + 1] - a0;
-    const Tabs t = carve_tabs(smem + a16(sizeof(Hdr)) + (size_t)kLargeWarps * wscr_bytes(LT), m, LT, nH, nV, true);
+    const Tabs t = carve_prep(smem, m);
     large_prologue(t, nv, a0, m, tid, T, warp, lane, &s_maxd, &s_npaths, &s_deep);
     __syncthreads();
     for (int i = tid; i < m; i += T) {
@@ -1571,8 +1594,7 @@ cudaError_t launch_prep_lt(fgr_grid* g, cudaStream_t st, const NetsView& nv, con
         e = cudaFuncSetAttribute(k_large_prep<LT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                  g->max_smem - (int)fa.sharedSizeBytes);
     if (e != cudaSuccess) return e;
-    k_large_prep<LT><<<count, 32 * kLargeWarps, smem_large(LT, g->nH, g->nV, maxm), st>>>(g->view, nv, list, cs, cl, hv,
-                                                                                        bot, pq, rpos, np);
+    k_large_prep<LT><<<count, kPrepThreads, prep_bytes(maxm), st>>>(g->view, nv, list, cs, cl, hv, bot, pq, rpos, np);
     g->stats.kernel_launches++;
     return cudaGetLastError();
 }
