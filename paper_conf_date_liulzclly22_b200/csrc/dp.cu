@@ -1106,63 +1106,158 @@ __global__ void __launch_bounds__(32 * kLargeWarps, 1) k_dp_large(GridView g, Ne
     }
     __syncthreads();
     TMARK(3);
-    // ---------------- backtrack: top-down path walks (S5), one lane per path
-    // A walk is a scalar chain (span of u -> lt -> ls -> span of v), so lane 0 of a warp
-    // walks a path with the parent's span in a register (no shuffles, no per-node warp
-    // synchronisation); a path whose top hangs off another path waits for that node's span
-    // (sready).  Warps take paths by ticket, shallowest top first, so every awaited path is
-    // already held by a running warp (no deadlock).
-    for (;;) {
-        int p = 0;
-        if (lane == 0) p = atomicAdd(&s_ticket2, 1);
-        p = __shfl_sync(0xffffffffu, p, 0);
-        if (p >= npaths) break;
-        if (lane != 0) continue;
-        const int tp = t.pq[npaths - 1 - p];
-        int v, sp;
-        if (tp == 0) { v = t.hv[0]; sp = t.span[0]; }
-        else {
-            const int u0 = t.par[tp];
-            while (ld_flag(&t.sready[u0]) == 0) __nanosleep(32);
-            __threadfence_block();
-            v = tp;
-            sp = t.span[u0];
-        }
-        while (v != 0xFFFF) {
-            const int u = t.par[v];
+    // ---------------- backtrack: top-down path walks (S5)
+    // The backtrack step of a node is a fixed map from its parent's span to its own span
+    // (lt = smallest l of the span minimising E_v(l), R11; ls = recE_v(lt); span = recB_v(ls)).
+    // All threads tabulate that map per node (spans as triangular codes, one byte per parent
+    // span) into the dead leg-cost tables; a path walk is then one shared-memory byte load per
+    // node, and the segment records are derived in the parallel output pass below.
+    if constexpr (LT * (LT + 1) / 2 <= 8 * LT) {
+        constexpr int NSP = LT * (LT + 1) / 2;
+        constexpr int MSB = (NSP + 3) & ~3;   // map bytes per node (legH + legV give 8 LT per node)
+        uint8_t* smap = reinterpret_cast<uint8_t*>(t.legH);
+        auto code = [](int sp) -> int {        // (lo << 4 | hi) -> triangular code
             const int lo = sp >> 4, hi = sp & 15;
-            uint32_t ev[LT];
+            return max(0, min(lo * (2 * LT - lo + 1) / 2 + (hi - lo), NSP - 1));
+        };
+        for (int v = 1 + tid; v < m; v += T) {
+            uint32_t ev[LT], cs[LT];
 #pragma unroll
-            for (int l = 0; l < LT; l++) ev[l] = t.E[(size_t)v * LT + l];
+            for (int l = 0; l < LT; l++) {
+                ev[l] = t.E[(size_t)v * LT + l];
+                cs[l] = (uint32_t)code(t.recB[(size_t)v * LT + t.recE[(size_t)v * LT + l]]);
+            }
+            uint32_t* out = reinterpret_cast<uint32_t*>(smap + (size_t)v * MSB);
+            uint32_t word = 0;
+            int idx = 0;
+#pragma unroll
+            for (int lo = 0; lo < LT; lo++) {
+                uint32_t be = ev[lo], cc = cs[lo];
+#pragma unroll
+                for (int hi = lo; hi < LT; hi++) {
+                    if (hi > lo && ev[hi] < be) { be = ev[hi]; cc = cs[hi]; }
+                    word |= cc << (8 * (idx & 3));
+                    if ((idx & 3) == 3) { out[idx >> 2] = word; word = 0; }
+                    idx++;
+                }
+            }
+            if (idx & 3) out[idx >> 2] = word;
+        }
+        if (tid == 0) t.span[0] = (uint8_t)code(t.span[0]);
+        __syncthreads();
+        // one lane per path; warps take paths by ticket, shallowest top first, so every
+        // awaited path top's parent is held by a running warp (no deadlock)
+        for (;;) {
+            int p = 0;
+            if (lane == 0) p = atomicAdd(&s_ticket2, 1);
+            p = __shfl_sync(0xffffffffu, p, 0);
+            if (p >= npaths) break;
+            if (lane != 0) continue;
+            const int tp = t.pq[npaths - 1 - p];
+            int v, sp;
+            if (tp == 0) { v = t.hv[0]; sp = t.span[0]; }
+            else {
+                const int u0 = t.par[tp];
+                while (ld_flag(&t.sready[u0]) == 0) __nanosleep(32);
+                __threadfence_block();
+                v = tp;
+                sp = t.span[u0];
+            }
+            while (v != 0xFFFF) {
+                sp = smap[(size_t)v * MSB + sp];
+                t.span[v] = (uint8_t)sp;
+                if (t.cstart[v + 1] - t.cstart[v] > 1) {   // light children wait for this span
+                    __threadfence_block();
+                    *(volatile uint8_t*)&t.sready[v] = 1;
+                }
+                v = t.hv[v];
+            }
+        }
+        __syncthreads();
+        TMARK(4);
+        TMARK(5);
+        // segment records from the parent's span, outputs, and S6 for the whole net in one pass
+        for (int i = 1 + tid; i < m; i += T) {
+            const int u = t.par[i];
+            const int cp = t.span[u];
+            int lo = 0;
+#pragma unroll
+            for (int l = 1; l < LT; l++) lo += cp >= l * (2 * LT - l + 1) / 2 ? 1 : 0;
+            const int hi = lo + cp - lo * (2 * LT - lo + 1) / 2;
             uint32_t be = 0xFFFFFFFFu;
             int lt = lo;
 #pragma unroll
-            for (int l = 0; l < LT; l++)
-                if (l >= lo && l <= hi && ev[l] < be) { be = ev[l]; lt = l; }   // smallest l attaining the min (R11)
-            const int ls = t.recE[(size_t)v * LT + lt];
-            sp = t.recB[(size_t)v * LT + ls];
-            t.span[v] = (uint8_t)sp;
-            const bool straight = (t.x[v] == t.x[u]) || (t.y[v] == t.y[u]);
-            const uint32_t bend = seg_bend(h->dir[ls], h->dir[lt], straight);
-            t.legH[(size_t)v * 2 * nH] = bend | ((uint32_t)ls << 8) | ((uint32_t)lt << 16) | ((uint32_t)straight << 24);
-            if (t.cstart[v + 1] - t.cstart[v] > 1) {   // light children wait for this span
-                __threadfence_block();
-                *(volatile uint8_t*)&t.sready[v] = 1;
+            for (int l = 0; l < LT; l++) {
+                const uint32_t e = t.E[(size_t)i * LT + l];
+                if (l >= lo && l <= hi && e < be) { be = e; lt = l; }   // smallest l attaining the min (R11)
             }
-            v = t.hv[v];
+            const int ls = t.recE[(size_t)i * LT + lt];
+            const bool straight = (t.x[i] == t.x[u]) || (t.y[i] == t.y[u]);
+            const uint32_t s = seg_bend(h->dir[ls], h->dir[lt], straight) | ((uint32_t)ls << 8) | ((uint32_t)lt << 16) |
+                               ((uint32_t)straight << 24);
+            if (o.rec_seg) o.rec_seg[o.rec_off[o.list_base + idx] + i] = s;
+            else o.seg[a0 + i] = s;
+            if (commit) commit_edge(g, h, t.x[i], t.y[i], t.x[u], t.y[u], s, hyb_z(hy, a0 + i, s, LT));
         }
-    }
-    __syncthreads();
-    TMARK(4);
-    TMARK(5);
-    // outputs and S6 for the whole net in one pass (the atomics' latencies overlap across threads)
-    for (int i = 1 + tid; i < m; i += T) {
-        const uint32_t s = t.legH[(size_t)i * 2 * nH];
-        if (o.rec_seg) o.rec_seg[o.rec_off[o.list_base + idx] + i] = s;
-        else o.seg[a0 + i] = s;
-        if (commit) {
-            const int u = t.par[i];
-            commit_edge(g, h, t.x[i], t.y[i], t.x[u], t.y[u], s, hyb_z(hy, a0 + i, s, LT));
+    } else {
+        // ---------------- backtrack: top-down path walks (S5), one lane per path
+        // A walk is a scalar chain (span of u -> lt -> ls -> span of v), so lane 0 of a warp
+        // walks a path with the parent's span in a register (no shuffles, no per-node warp
+        // synchronisation); a path whose top hangs off another path waits for that node's span
+        // (sready).  Warps take paths by ticket, shallowest top first, so every awaited path is
+        // already held by a running warp (no deadlock).
+        for (;;) {
+            int p = 0;
+            if (lane == 0) p = atomicAdd(&s_ticket2, 1);
+            p = __shfl_sync(0xffffffffu, p, 0);
+            if (p >= npaths) break;
+            if (lane != 0) continue;
+            const int tp = t.pq[npaths - 1 - p];
+            int v, sp;
+            if (tp == 0) { v = t.hv[0]; sp = t.span[0]; }
+            else {
+                const int u0 = t.par[tp];
+                while (ld_flag(&t.sready[u0]) == 0) __nanosleep(32);
+                __threadfence_block();
+                v = tp;
+                sp = t.span[u0];
+            }
+            while (v != 0xFFFF) {
+                const int u = t.par[v];
+                const int lo = sp >> 4, hi = sp & 15;
+                uint32_t ev[LT];
+#pragma unroll
+                for (int l = 0; l < LT; l++) ev[l] = t.E[(size_t)v * LT + l];
+                uint32_t be = 0xFFFFFFFFu;
+                int lt = lo;
+#pragma unroll
+                for (int l = 0; l < LT; l++)
+                    if (l >= lo && l <= hi && ev[l] < be) { be = ev[l]; lt = l; }   // smallest l attaining the min (R11)
+                const int ls = t.recE[(size_t)v * LT + lt];
+                sp = t.recB[(size_t)v * LT + ls];
+                t.span[v] = (uint8_t)sp;
+                const bool straight = (t.x[v] == t.x[u]) || (t.y[v] == t.y[u]);
+                const uint32_t bend = seg_bend(h->dir[ls], h->dir[lt], straight);
+                t.legH[(size_t)v * 2 * nH] = bend | ((uint32_t)ls << 8) | ((uint32_t)lt << 16) | ((uint32_t)straight << 24);
+                if (t.cstart[v + 1] - t.cstart[v] > 1) {   // light children wait for this span
+                    __threadfence_block();
+                    *(volatile uint8_t*)&t.sready[v] = 1;
+                }
+                v = t.hv[v];
+            }
+        }
+        __syncthreads();
+        TMARK(4);
+        TMARK(5);
+        // outputs and S6 for the whole net in one pass (the atomics' latencies overlap across threads)
+        for (int i = 1 + tid; i < m; i += T) {
+            const uint32_t s = t.legH[(size_t)i * 2 * nH];
+            if (o.rec_seg) o.rec_seg[o.rec_off[o.list_base + idx] + i] = s;
+            else o.seg[a0 + i] = s;
+            if (commit) {
+                const int u = t.par[i];
+                commit_edge(g, h, t.x[i], t.y[i], t.x[u], t.y[u], s, hyb_z(hy, a0 + i, s, LT));
+            }
         }
     }
 #ifdef FGR_TIMING
