@@ -950,75 +950,164 @@ __global__ void __launch_bounds__(32 * WARPS) k_dp_flow(GridView g, NetsView nv,
     }
     __syncthreads();
     const int ntops = s_ntops;
-    if (lane == 0) {
-        for (;;) {
-            const int k = atomicAdd(&s_ticket2, 1);
-            if (k >= ntops) break;
-            int v = leafq[k], sp;
-            if (v == 0) {
-                sp = t.span[0];
-                v = hv[0];
-            } else {
-                const int u0 = t.par[v];
-                while (*(volatile uint8_t*)&sready[u0] == 0) __nanosleep(20);
-                __threadfence_block();
-                sp = *(volatile uint8_t*)&t.span[u0];
-            }
-            uint32_t e[ES];
-            {
-                const uint4* ep = reinterpret_cast<const uint4*>(t.E + v * ES);
+    if constexpr (LT * (LT + 1) / 2 <= 8 * LT) {
+        // The backtrack step of a node is a fixed map from its parent's span to its own
+        // (same derivation as k_dp_large): tabulated per node by all threads into the dead
+        // leg tables (LA, LB), so a path walk is one shared-memory byte load per node; the
+        // segment records are derived from the parent's span in the parallel output pass.
+        constexpr int NSP = LT * (LT + 1) / 2;
+        constexpr int MSB = (NSP + 3) & ~3;
+        uint8_t* smap = reinterpret_cast<uint8_t*>(t.LA);
+        auto code = [](int sp) -> int {        // (lo << 4 | hi) -> triangular code
+            const int lo = sp >> 4, hi = sp & 15;
+            return max(0, min(lo * (2 * LT - lo + 1) / 2 + (hi - lo), NSP - 1));
+        };
+        for (int v = 1 + tid; v < m; v += T) {
+            uint32_t ev[LT], cc[LT];
 #pragma unroll
-                for (int q = 0; q < ES / 4; q++) {
-                    const uint4 w = ep[q];
-                    e[4 * q] = w.x; e[4 * q + 1] = w.y; e[4 * q + 2] = w.z; e[4 * q + 3] = w.w;
+            for (int l = 0; l < LT; l++) {
+                ev[l] = t.E[v * ES + l];
+                cc[l] = (uint32_t)code(t.recB[v * ES + t.recE[v * ES + l]]);
+            }
+            uint32_t* out = reinterpret_cast<uint32_t*>(smap + (size_t)v * MSB);
+            uint32_t word = 0;
+            int idx = 0;
+#pragma unroll
+            for (int lo = 0; lo < LT; lo++) {
+                uint32_t be = ev[lo], c0 = cc[lo];
+#pragma unroll
+                for (int hi = lo; hi < LT; hi++) {
+                    if (hi > lo && ev[hi] < be) { be = ev[hi]; c0 = cc[hi]; }
+                    word |= c0 << (8 * (idx & 3));
+                    if ((idx & 3) == 3) { out[idx >> 2] = word; word = 0; }
+                    idx++;
                 }
             }
+            if (idx & 3) out[idx >> 2] = word;
+        }
+        if (tid == 0) t.span[0] = (uint8_t)code(t.span[0]);
+        __syncthreads();
+        if (lane == 0) {
             for (;;) {
-                const int u = t.par[v];
-                const int nx = hv[v];
-                const int nc = cs[v + 1] - cs[v];
-                uint32_t en[ES];   // prefetch the next node's E row while this node's argmins resolve
+                const int k = atomicAdd(&s_ticket2, 1);
+                if (k >= ntops) break;
+                int v = leafq[k], sp;
+                if (v == 0) {
+                    sp = t.span[0];
+                    v = hv[0];
+                } else {
+                    const int u0 = t.par[v];
+                    while (*(volatile uint8_t*)&sready[u0] == 0) __nanosleep(20);
+                    __threadfence_block();
+                    sp = *(volatile uint8_t*)&t.span[u0];
+                }
+                while (v != 0xFFFF) {
+                    sp = smap[(size_t)v * MSB + sp];
+                    t.span[v] = (uint8_t)sp;
+                    if (cs[v + 1] - cs[v] > 1) {   // light children start paths below v
+                        __threadfence_block();
+                        *(volatile uint8_t*)&sready[v] = 1;
+                    }
+                    v = hv[v];
+                }
+            }
+        }
+        __syncthreads();
+        FMARK(4);
+        // ---- segment records, outputs and S6
+        for (int i = 1 + tid; i < m; i += T) {
+            const int u = t.par[i];
+            const int cp = t.span[u];
+            int lo = 0;
+#pragma unroll
+            for (int l = 1; l < LT; l++) lo += cp >= l * (2 * LT - l + 1) / 2 ? 1 : 0;
+            const int hi = lo + cp - lo * (2 * LT - lo + 1) / 2;
+            uint32_t be = 0xFFFFFFFFu;
+            int lt = lo;
+#pragma unroll
+            for (int l = 0; l < LT; l++) {
+                const uint32_t e = t.E[i * ES + l];
+                if (l >= lo && l <= hi && e < be) { be = e; lt = l; }   // smallest l attaining the min (R11)
+            }
+            const int ls = t.recE[i * ES + lt];
+            const bool straight = (t.x[i] == t.x[u]) || (t.y[i] == t.y[u]);
+            const uint32_t s = seg_bend(wh->h.dir[ls], wh->h.dir[lt], straight) | ((uint32_t)ls << 8) |
+                               ((uint32_t)lt << 16) | ((uint32_t)straight << 24);
+            if (o.rec_seg) o.rec_seg[o.rec_off[o.list_base + blockIdx.x] + i] = s;
+            else o.seg[a0 + i] = s;
+            if (commit) commit_edge(g, &wh->h, t.x[i], t.y[i], t.x[u], t.y[u], s, hyb_z(hy, a0 + i, s, LT));
+        }
+    } else {
+        if (lane == 0) {
+            for (;;) {
+                const int k = atomicAdd(&s_ticket2, 1);
+                if (k >= ntops) break;
+                int v = leafq[k], sp;
+                if (v == 0) {
+                    sp = t.span[0];
+                    v = hv[0];
+                } else {
+                    const int u0 = t.par[v];
+                    while (*(volatile uint8_t*)&sready[u0] == 0) __nanosleep(20);
+                    __threadfence_block();
+                    sp = *(volatile uint8_t*)&t.span[u0];
+                }
+                uint32_t e[ES];
                 {
-                    const uint4* ep = reinterpret_cast<const uint4*>(t.E + (nx == 0xFFFF ? v : nx) * ES);
+                    const uint4* ep = reinterpret_cast<const uint4*>(t.E + v * ES);
 #pragma unroll
                     for (int q = 0; q < ES / 4; q++) {
                         const uint4 w = ep[q];
-                        en[4 * q] = w.x; en[4 * q + 1] = w.y; en[4 * q + 2] = w.z; en[4 * q + 3] = w.w;
+                        e[4 * q] = w.x; e[4 * q + 1] = w.y; e[4 * q + 2] = w.z; e[4 * q + 3] = w.w;
                     }
                 }
-                const int lo = sp >> 4, hi = sp & 15;
-                uint32_t be = 0xFFFFFFFFu;
-                int lt = lo;
+                for (;;) {
+                    const int u = t.par[v];
+                    const int nx = hv[v];
+                    const int nc = cs[v + 1] - cs[v];
+                    uint32_t en[ES];   // prefetch the next node's E row while this node's argmins resolve
+                    {
+                        const uint4* ep = reinterpret_cast<const uint4*>(t.E + (nx == 0xFFFF ? v : nx) * ES);
 #pragma unroll
-                for (int l = 0; l < LT; l++)
-                    if (l >= lo && l <= hi && e[l] < be) { be = e[l]; lt = l; }   // smallest l attaining the min (R11)
-                const int ls = t.recE[v * ES + lt];
-                sp = t.recB[v * ES + ls];
-                const bool straight = (t.x[v] == t.x[u]) || (t.y[v] == t.y[u]);
-                const uint32_t bend = seg_bend(wh->h.dir[ls], wh->h.dir[lt], straight);
-                t.seg[v] = bend | ((uint32_t)ls << 8) | ((uint32_t)lt << 16) | ((uint32_t)straight << 24);
-                if (nc > 1) {   // light children start paths below v: publish its span
-                    t.span[v] = (uint8_t)sp;
-                    __threadfence_block();
-                    *(volatile uint8_t*)&sready[v] = 1;
+                        for (int q = 0; q < ES / 4; q++) {
+                            const uint4 w = ep[q];
+                            en[4 * q] = w.x; en[4 * q + 1] = w.y; en[4 * q + 2] = w.z; en[4 * q + 3] = w.w;
+                        }
+                    }
+                    const int lo = sp >> 4, hi = sp & 15;
+                    uint32_t be = 0xFFFFFFFFu;
+                    int lt = lo;
+#pragma unroll
+                    for (int l = 0; l < LT; l++)
+                        if (l >= lo && l <= hi && e[l] < be) { be = e[l]; lt = l; }   // smallest l attaining the min (R11)
+                    const int ls = t.recE[v * ES + lt];
+                    sp = t.recB[v * ES + ls];
+                    const bool straight = (t.x[v] == t.x[u]) || (t.y[v] == t.y[u]);
+                    const uint32_t bend = seg_bend(wh->h.dir[ls], wh->h.dir[lt], straight);
+                    t.seg[v] = bend | ((uint32_t)ls << 8) | ((uint32_t)lt << 16) | ((uint32_t)straight << 24);
+                    if (nc > 1) {   // light children start paths below v: publish its span
+                        t.span[v] = (uint8_t)sp;
+                        __threadfence_block();
+                        *(volatile uint8_t*)&sready[v] = 1;
+                    }
+                    if (nx == 0xFFFF) break;
+                    v = nx;
+#pragma unroll
+                    for (int q = 0; q < ES; q++) e[q] = en[q];
                 }
-                if (nx == 0xFFFF) break;
-                v = nx;
-#pragma unroll
-                for (int q = 0; q < ES; q++) e[q] = en[q];
             }
         }
-    }
-    __syncthreads();
-    FMARK(4);
-    // ---- outputs and S6
-    for (int i = 1 + tid; i < m; i += T) {
-        const uint32_t s = t.seg[i];
-        if (o.rec_seg) o.rec_seg[o.rec_off[o.list_base + blockIdx.x] + i] = s;
-        else o.seg[a0 + i] = s;
-        if (commit) {
-            const int u = t.par[i];
-            commit_edge(g, &wh->h, t.x[i], t.y[i], t.x[u], t.y[u], s, hyb_z(hy, a0 + i, s, LT));
+        __syncthreads();
+        FMARK(4);
+        // ---- outputs and S6
+        for (int i = 1 + tid; i < m; i += T) {
+            const uint32_t s = t.seg[i];
+            if (o.rec_seg) o.rec_seg[o.rec_off[o.list_base + blockIdx.x] + i] = s;
+            else o.seg[a0 + i] = s;
+            if (commit) {
+                const int u = t.par[i];
+                commit_edge(g, &wh->h, t.x[i], t.y[i], t.x[u], t.y[u], s, hyb_z(hy, a0 + i, s, LT));
+            }
         }
     }
     if (tid == 0) {
