@@ -73,7 +73,29 @@ __device__ __forceinline__ void warp_incl_scan(uint32_t (&x)[W]) {
 // 32/W runs of the slot (log2(32/W) shuffles); P and ST stored.  Same sums as a per-position
 // warp scan, a third of the instructions.
 template <int W>
-__device__ __forceinline__ void refresh_segment(const GridView& g, const DirView& d, int dsel, int line, int s) {
+struct SegIn {         // one lane's loaded inputs of a segment: demand and capacity of its W positions
+    int32_t dem[W];
+    uint8_t cap[W];
+};
+
+template <int W>
+__device__ __forceinline__ void load_segment(const GridView& g, const DirView& d, int line, int s, SegIn<W>& in) {
+    const int lane = lane_id();
+    const int sl = lane & (W - 1), q = lane / W;
+    const int p0 = s * FGR_SEG + q * W;
+    const bool slot_ok = sl < d.cnt;
+    const size_t base = ((size_t)line * d.len + p0) * W + sl;
+#pragma unroll
+    for (int j = 0; j < W; j++) {
+        const bool ok = slot_ok && p0 + j < d.len - 1;
+        in.dem[j] = ok ? d.D[base + (size_t)j * W] : 0;
+        in.cap[j] = ok ? d.C[base + (size_t)j * W] : 0;
+    }
+}
+
+template <int W>
+__device__ __forceinline__ void scan_segment(const GridView& g, const DirView& d, int dsel, int line, int s,
+                                             const SegIn<W>& in) {
     const int lane = lane_id();
     const int sl = lane & (W - 1), q = lane / W;
     const int p0 = s * FGR_SEG + q * W;
@@ -81,20 +103,12 @@ __device__ __forceinline__ void refresh_segment(const GridView& g, const DirView
     const int span = 2 * g.S + 1;
     const int32_t* tab = g.table + (slot_ok ? g.layer_of_slot[dsel][sl] : 0) * span + g.S;
     const size_t base = ((size_t)line * d.len + p0) * W + sl;
-    int32_t dem[W];
-    uint8_t cap[W];
-#pragma unroll
-    for (int j = 0; j < W; j++) {
-        const bool ok = slot_ok && p0 + j < d.len - 1;
-        dem[j] = ok ? d.D[base + (size_t)j * W] : 0;
-        cap[j] = ok ? d.C[base + (size_t)j * W] : 0;
-    }
     uint32_t ec[W], run = 0;
 #pragma unroll
     for (int j = 0; j < W; j++) {
         uint32_t c = 0;
         if (slot_ok && p0 + j < d.len - 1) {
-            int sk = (int)cap[j] - dem[j];
+            int sk = (int)in.cap[j] - in.dem[j];
             sk = sk < -g.S ? -g.S : (sk > g.S ? g.S : sk);
             c = (uint32_t)g.len_cost + (uint32_t)__ldg(tab + sk);
         }
@@ -170,12 +184,26 @@ __device__ __forceinline__ int refresh_chunk(const GridView& g, const DirView& d
         if (chunk >= c0 && chunk < c0 + 32) own = o;
     }
     if (own == 0) return 0;
+    // two dirty segments in flight: the next segment's loads are issued before this one's scan
     int done = 0;
-    while (own) {
-        const int q = __ffs(own) - 1;
+    int q = __ffs(own) - 1;
+    own &= own - 1;
+    SegIn<W> cur;
+    load_segment<W>(g, d, line, chunk * FGR_CHUNK_SEGS + q, cur);
+    for (;;) {
+        if (own == 0) {
+            scan_segment<W>(g, d, dsel, line, chunk * FGR_CHUNK_SEGS + q, cur);
+            done++;
+            break;
+        }
+        const int q2 = __ffs(own) - 1;
         own &= own - 1;
-        refresh_segment<W>(g, d, dsel, line, chunk * FGR_CHUNK_SEGS + q);
+        SegIn<W> nxt;
+        load_segment<W>(g, d, line, chunk * FGR_CHUNK_SEGS + q2, nxt);
+        scan_segment<W>(g, d, dsel, line, chunk * FGR_CHUNK_SEGS + q, cur);
         done++;
+        cur = nxt;
+        q = q2;
     }
     int last = 0;
     if (lane == 0) {

@@ -96,6 +96,18 @@ def test_big_nets_cta_path():
     check_against_oracle(d)
 
 
+@pytest.mark.parametrize("L", [3, 5, 12, 16])
+def test_big_nets_layer_counts(L):
+    """The flow (33..128 nodes) and heavy-path (> 128 nodes) kernels at other layer counts:
+    L <= 15 backtracks through tabulated span maps, L = 16 through the scalar span walk."""
+    caps = [2] + [6] * (L - 1)
+    d = gen.generate(nx=90, ny=80, nlayers=L, num_nets=150, seed=300 + L, caps=caps, pin_dist=1, kmin=20,
+                     kmax=300, hpwl_base=18.0, hpwl_sigma=0.5, literal_frac=0.2, name=f"big{L}")
+    sizes = d.net_sizes()
+    assert ((sizes > 32) & (sizes <= 128)).sum() > 10 and (sizes > 128).sum() > 5
+    check_against_oracle(d)
+
+
 def test_route_batch_matches_oracle_batches():
     import torch
     d = gen.make_config("t1")
