@@ -200,6 +200,12 @@ def test_t9_full_size_bit_exact():
     check_against_oracle(gen.make_config("t9"))
 
 
+def test_scale_full_size_bit_exact():
+    """BASELINE.json configs[4] (2M nets, 2000 x 2000, 9 layers) at full size: the
+    largest design the library routes, every net, batch and demand cell compared."""
+    check_against_oracle(gen.make_config("scale"))
+
+
 @pytest.mark.parametrize("cfg", ["tiny", "t5"])
 def test_exchange_path_world1_bit_exact(cfg):
     """The multi-GPU path (split -> route records -> NCCL all-reduce -> commit from
