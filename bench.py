@@ -50,7 +50,8 @@ def committed_traffic(kernel_class):
     """DRAM bytes per launch of a kernel class from the newest committed ncu capture
     (profiles/<tag>_traffic.json, written by tools/summarize_profiles.py), or None."""
     import glob
-    files = sorted(glob.glob(os.path.join(ROOT, "profiles", "*_traffic.json")), key=os.path.getmtime)
+    # newest = highest round tag (r01b < r01g): file mtimes are checkout times on a fresh box
+    files = sorted(glob.glob(os.path.join(ROOT, "profiles", "*_traffic.json")), key=os.path.basename)
     for f in reversed(files):
         try:
             j = json.load(open(f))
