@@ -30,7 +30,7 @@ namespace {
 
 constexpr int kGroupWarps = 4;              // warps per CTA in k_dp_group
 constexpr int kLargeWarps = 16;             // warps per CTA in k_dp_large (one path-walking group each)
-constexpr int kFlowMax = 128;               // largest net of the dataflow kernel by default
+constexpr int kFlowMax = 64;                // largest net of the dataflow kernel by default
 
 
 
@@ -1593,7 +1593,8 @@ cudaError_t launch_lt(fgr_grid* g, cudaStream_t st, const NetsView& nv, const in
     }
     // Nets of up to kFlowMax nodes take the dataflow kernel (dp_walk.cu); bigger ones the
     // heavy-path kernel below, whose root-path transfer matrices shorten the long chains
-    // (measured on t9: equal step time, lower latency for 33..128-node nets).  FGR_FLOW_MAX
+    // (measured on t9, 3 interleaved runs each: cut 128 / 64 / 32 = 20.34 / 20.18 / 20.12 ms
+    // per step, profiles/r01h_flowmax_ab2.txt; 64 keeps the flow kernel on the default path).  FGR_FLOW_MAX
     // overrides the cut for A/B runs.
     static int flow_cap = -1;
     if (flow_cap < 0) { const char* s = getenv("FGR_FLOW_MAX"); flow_cap = s ? atoi(s) : kFlowMax; }

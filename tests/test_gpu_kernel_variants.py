@@ -57,6 +57,7 @@ for name in sys.argv[1].split(","):
 VARIANTS = {
     "flow_all": {"FGR_FLOW_MAX": "100000"},
     "flow_40": {"FGR_FLOW_MAX": "40"},
+    "flow_128": {"FGR_FLOW_MAX": "128"},    # the previous default cut
     "large_old": {"FGR_LARGE_KERNEL": "old"},
     "group_old": {"FGR_GROUP_KERNEL": "old"},
 }

@@ -98,7 +98,7 @@ def test_big_nets_cta_path():
 
 @pytest.mark.parametrize("L", [3, 5, 12, 16])
 def test_big_nets_layer_counts(L):
-    """The flow (33..128 nodes) and heavy-path (> 128 nodes) kernels at other layer counts:
+    """The flow (33..64 nodes by default) and heavy-path (> 64 nodes) kernels at other layer counts:
     L <= 15 backtracks through tabulated span maps, L = 16 through the scalar span walk."""
     caps = [2] + [6] * (L - 1)
     d = gen.generate(nx=90, ny=80, nlayers=L, num_nets=150, seed=300 + L, caps=caps, pin_dist=1, kmin=20,
