@@ -15,6 +15,8 @@
 // moved per batch follow the demand that changed, not the grid size.
 #include "fgr_internal.cuh"
 
+#include <cstdlib>
+
 template <int W>
 struct Vec {
     static __device__ __forceinline__ void load_i32(const int32_t* p, int32_t (&o)[W]) {
@@ -264,7 +266,10 @@ cudaError_t fgr_launch_refresh_sized(fgr_grid* g, cudaStream_t st, bool full, lo
     const long long tasks = (long long)v.h.lines * ((v.h.nseg + FGR_CHUNK_SEGS - 1) / FGR_CHUNK_SEGS) +
                             (long long)v.v.lines * ((v.v.nseg + FGR_CHUNK_SEGS - 1) / FGR_CHUNK_SEGS);
     int blocks = (int)((tasks + 7) / 8);
-    const int cap_blocks = g->num_sms * 8;
+    // FGR_REFRESH_CTAS_PER_SM overrides the cap for A/B runs (grid-stride keeps any grid exact)
+    static int per_sm = -1;
+    if (per_sm < 0) { const char* s = getenv("FGR_REFRESH_CTAS_PER_SM"); per_sm = s ? max(1, atoi(s)) : 8; }
+    const int cap_blocks = g->num_sms * per_sm;
     if (blocks > cap_blocks) blocks = cap_blocks;
     if (blocks < 1) blocks = 1;
     g->stats.kernel_launches++;
