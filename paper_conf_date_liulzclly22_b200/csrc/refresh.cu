@@ -225,7 +225,7 @@ __device__ __forceinline__ int refresh_chunk(const GridView& g, const DirView& d
 }
 
 template <int WH, int WV>
-__global__ void __launch_bounds__(256) k_refresh(GridView g, int full) {
+__device__ __forceinline__ void refresh_body(const GridView& g, int full) {
     pdl_trigger();   // the next DP kernel may start its prologue now
     pdl_wait();      // the previous batch's commits must be complete
     const int chH = (g.h.nseg + FGR_CHUNK_SEGS - 1) / FGR_CHUNK_SEGS;
@@ -252,9 +252,22 @@ __global__ void __launch_bounds__(256) k_refresh(GridView g, int full) {
 }
 
 template <int WH, int WV>
+__global__ void __launch_bounds__(256) k_refresh(GridView g, int full) { refresh_body<WH, WV>(g, full); }
+
+// register-budget variants for A/B runs (FGR_REFRESH_MINB)
+template <int WH, int WV, int MB>
+__global__ void __launch_bounds__(256, MB) k_refresh_mb(GridView g, int full) { refresh_body<WH, WV>(g, full); }
+
+template <int WH, int WV>
 static cudaError_t launch_t(fgr_grid* g, cudaStream_t st, bool full, int blocks) {
+    // FGR_REFRESH_MINB (A/B runs): register budget via min resident CTAs per SM; 0 = compiler's choice
+    static int minb = -1;
+    if (minb < 0) { const char* s = getenv("FGR_REFRESH_MINB"); minb = s ? atoi(s) : 0; }
     const int ps = fgr_prof_begin(g, PROF_REFRESH, st);
-    k_refresh<WH, WV><<<blocks, 256, 0, st>>>(g->view, full ? 1 : 0);
+    if (minb == 6) k_refresh_mb<WH, WV, 6><<<blocks, 256, 0, st>>>(g->view, full ? 1 : 0);
+    else if (minb == 5) k_refresh_mb<WH, WV, 5><<<blocks, 256, 0, st>>>(g->view, full ? 1 : 0);
+    else if (minb == 4) k_refresh_mb<WH, WV, 4><<<blocks, 256, 0, st>>>(g->view, full ? 1 : 0);
+    else k_refresh<WH, WV><<<blocks, 256, 0, st>>>(g->view, full ? 1 : 0);
     fgr_prof_end(g, ps, st);
     return cudaGetLastError();
 }
