@@ -162,14 +162,14 @@ __device__ __forceinline__ void rebase_line(const DirView& d, int line) {
 // One task = (line, chunk of 8 segments).  The dirty segments of the chunk are
 // rescanned; the warp finishing the last dirty chunk of the line rebuilds the
 // segment bases and clears the line's flags.  Returns the segments rescanned.
-template <int W>
+template <int W, int CS>
 __device__ __forceinline__ int refresh_chunk(const GridView& g, const DirView& d, int dsel, int line, int chunk,
                                              bool full) {
     const int lane = lane_id();
     const int lidx = d.line_base + line;
     if (!full && g.dline[lidx] == 0) return 0;
     const uint8_t* f = g.dseg + d.seg_base + (size_t)line * d.nseg;
-    const int nchunks = (d.nseg + FGR_CHUNK_SEGS - 1) / FGR_CHUNK_SEGS;
+    const int nchunks = (d.nseg + CS - 1) / CS;
     // dirty chunks of the line (every task of the line computes the same count)
     int nd = 0;
     uint32_t own = 0;
@@ -177,8 +177,8 @@ __device__ __forceinline__ int refresh_chunk(const GridView& g, const DirView& d
         const int c = c0 + lane;
         uint32_t m = 0;
         if (c < nchunks)
-            for (int q = 0; q < FGR_CHUNK_SEGS; q++) {
-                const int sg = c * FGR_CHUNK_SEGS + q;
+            for (int q = 0; q < CS; q++) {
+                const int sg = c * CS + q;
                 if (sg < d.nseg && (full || f[sg])) m |= 1u << q;
             }
         nd += __popc(__ballot_sync(0xffffffffu, m != 0));
@@ -191,18 +191,18 @@ __device__ __forceinline__ int refresh_chunk(const GridView& g, const DirView& d
     int q = __ffs(own) - 1;
     own &= own - 1;
     SegIn<W> cur;
-    load_segment<W>(g, d, line, chunk * FGR_CHUNK_SEGS + q, cur);
+    load_segment<W>(g, d, line, chunk * CS + q, cur);
     for (;;) {
         if (own == 0) {
-            scan_segment<W>(g, d, dsel, line, chunk * FGR_CHUNK_SEGS + q, cur);
+            scan_segment<W>(g, d, dsel, line, chunk * CS + q, cur);
             done++;
             break;
         }
         const int q2 = __ffs(own) - 1;
         own &= own - 1;
         SegIn<W> nxt;
-        load_segment<W>(g, d, line, chunk * FGR_CHUNK_SEGS + q2, nxt);
-        scan_segment<W>(g, d, dsel, line, chunk * FGR_CHUNK_SEGS + q, cur);
+        load_segment<W>(g, d, line, chunk * CS + q2, nxt);
+        scan_segment<W>(g, d, dsel, line, chunk * CS + q, cur);
         done++;
         cur = nxt;
         q = q2;
@@ -224,12 +224,12 @@ __device__ __forceinline__ int refresh_chunk(const GridView& g, const DirView& d
     return done;
 }
 
-template <int WH, int WV>
+template <int WH, int WV, int CS>
 __device__ __forceinline__ void refresh_body(const GridView& g, int full) {
     pdl_trigger();   // the next DP kernel may start its prologue now
     pdl_wait();      // the previous batch's commits must be complete
-    const int chH = (g.h.nseg + FGR_CHUNK_SEGS - 1) / FGR_CHUNK_SEGS;
-    const int chV = (g.v.nseg + FGR_CHUNK_SEGS - 1) / FGR_CHUNK_SEGS;
+    const int chH = (g.h.nseg + CS - 1) / CS;
+    const int chV = (g.v.nseg + CS - 1) / CS;
     const int tH = g.h.lines * chH;
     const int ntasks = tH + g.v.lines * chV;
     const int warp = (int)((blockIdx.x * (size_t)blockDim.x + threadIdx.x) >> 5);
@@ -238,11 +238,11 @@ __device__ __forceinline__ void refresh_body(const GridView& g, int full) {
     for (int t = warp; t < ntasks; t += nwarps) {
         if (t < tH) {
             const int line = t / chH;
-            nh += refresh_chunk<WH>(g, g.h, 0, line, t - line * chH, full);
+            nh += refresh_chunk<WH, CS>(g, g.h, 0, line, t - line * chH, full);
         } else {
             const int r = t - tH;
             const int line = r / chV;
-            nv += refresh_chunk<WV>(g, g.v, 1, line, r - line * chV, full);
+            nv += refresh_chunk<WV, CS>(g, g.v, 1, line, r - line * chV, full);
         }
     }
     if (lane_id() == 0 && (nh | nv)) {
@@ -252,11 +252,27 @@ __device__ __forceinline__ void refresh_body(const GridView& g, int full) {
 }
 
 template <int WH, int WV>
-__global__ void __launch_bounds__(256) k_refresh(GridView g, int full) { refresh_body<WH, WV>(g, full); }
+__global__ void __launch_bounds__(256) k_refresh(GridView g, int full) { refresh_body<WH, WV, FGR_CHUNK_SEGS>(g, full); }
+
+// task-size variants for A/B runs (FGR_REFRESH_CHUNK: segments per warp task)
+template <int WH, int WV, int CS>
+__global__ void __launch_bounds__(256) k_refresh_cs(GridView g, int full) { refresh_body<WH, WV, CS>(g, full); }
 
 // register-budget variants for A/B runs (FGR_REFRESH_MINB)
 template <int WH, int WV, int MB>
-__global__ void __launch_bounds__(256, MB) k_refresh_mb(GridView g, int full) { refresh_body<WH, WV>(g, full); }
+__global__ void __launch_bounds__(256, MB) k_refresh_mb(GridView g, int full) {
+    refresh_body<WH, WV, FGR_CHUNK_SEGS>(g, full);
+}
+
+static int refresh_chunk_segs() {
+    static int cs = -1;
+    if (cs < 0) {
+        const char* e = getenv("FGR_REFRESH_CHUNK");
+        cs = e ? atoi(e) : FGR_CHUNK_SEGS;
+        if (cs != 4 && cs != 16) cs = FGR_CHUNK_SEGS;
+    }
+    return cs;
+}
 
 template <int WH, int WV>
 static cudaError_t launch_t(fgr_grid* g, cudaStream_t st, bool full, int blocks) {
@@ -267,6 +283,8 @@ static cudaError_t launch_t(fgr_grid* g, cudaStream_t st, bool full, int blocks)
     if (minb == 6) k_refresh_mb<WH, WV, 6><<<blocks, 256, 0, st>>>(g->view, full ? 1 : 0);
     else if (minb == 5) k_refresh_mb<WH, WV, 5><<<blocks, 256, 0, st>>>(g->view, full ? 1 : 0);
     else if (minb == 4) k_refresh_mb<WH, WV, 4><<<blocks, 256, 0, st>>>(g->view, full ? 1 : 0);
+    else if (refresh_chunk_segs() == 4) k_refresh_cs<WH, WV, 4><<<blocks, 256, 0, st>>>(g->view, full ? 1 : 0);
+    else if (refresh_chunk_segs() == 16) k_refresh_cs<WH, WV, 16><<<blocks, 256, 0, st>>>(g->view, full ? 1 : 0);
     else k_refresh<WH, WV><<<blocks, 256, 0, st>>>(g->view, full ? 1 : 0);
     fgr_prof_end(g, ps, st);
     return cudaGetLastError();
@@ -276,8 +294,9 @@ static cudaError_t launch_t(fgr_grid* g, cudaStream_t st, bool full, int blocks)
 cudaError_t fgr_launch_refresh_sized(fgr_grid* g, cudaStream_t st, bool full, long long max_tasks) {
     (void)max_tasks;
     const GridView& v = g->view;
-    const long long tasks = (long long)v.h.lines * ((v.h.nseg + FGR_CHUNK_SEGS - 1) / FGR_CHUNK_SEGS) +
-                            (long long)v.v.lines * ((v.v.nseg + FGR_CHUNK_SEGS - 1) / FGR_CHUNK_SEGS);
+    const int cs = refresh_chunk_segs();
+    const long long tasks = (long long)v.h.lines * ((v.h.nseg + cs - 1) / cs) +
+                            (long long)v.v.lines * ((v.v.nseg + cs - 1) / cs);
     int blocks = (int)((tasks + 7) / 8);
     // FGR_REFRESH_CTAS_PER_SM overrides the cap for A/B runs (grid-stride keeps any grid exact)
     static int per_sm = -1;
