@@ -209,6 +209,9 @@ def main():
     ap.add_argument("--ref-fraction", type=float, default=0.25)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--dp-policy", default="auto", choices=["auto", "heavy", "hld"],
+                    help="large-net DP kernel selection (fgr_set_dp_policy); all give identical routes")
+    ap.add_argument("--flow-max", type=int, default=64)
     ap.add_argument("--hybrid", default=None,
                     help="T1,T2: hybrid L+Z patterns on tree edges with T1 <= HPWL <= T2 (FastGRH; default L only)")
     args = ap.parse_args()
@@ -231,7 +234,8 @@ def main():
     d = gen.make_config(args.config)
     ds = design_stats(d)
     hybrid = tuple(int(v) for v in args.hybrid.split(",")) if args.hybrid else None
-    r = Router(d, device=local, hybrid=hybrid)
+    policy = {"auto": F.FGR_DP_AUTO, "heavy": F.FGR_DP_HEAVY, "hld": F.FGR_DP_HLD}[args.dp_policy]
+    r = Router(d, device=local, hybrid=hybrid, dp_policy=(policy, args.flow_max))
     if world > 1:
         uid = [F.fgr_comm_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(uid, src=0)

@@ -167,6 +167,25 @@ FGR_API fgr_status fgr_route_batch(fgr_grid* grid, const fgr_nets* nets, const i
  */
 FGR_API fgr_status fgr_set_pattern(fgr_grid* grid, int32_t hybrid_t1, int32_t hybrid_t2);
 
+/*
+ * fgr_set_dp_policy — which tree-DP kernel routes nets of more than 32 nodes
+ * (all kernels compute the same DP, §III-D Eqs. (1)-(7), and give
+ * bit-identical routes; the choice only changes speed):
+ *   FGR_DP_AUTO  (default) nets of up to flow_max nodes: the tree-dataflow
+ *                kernel; bigger nets: the heavy-path kernel while the net fits
+ *                its shared-memory tables (~1.3k nodes at L = 9), above that the
+ *                heavy-path contraction kernel (global workspace, any size up to
+ *                65535 nodes);
+ *   FGR_DP_HEAVY as AUTO without the tree-dataflow kernel;
+ *   FGR_DP_HLD   the heavy-path contraction kernel for every net of > 32 nodes.
+ * flow_max in [33, 65535] (default 64; ignored unless AUTO).  Errors: INVALID.
+ * Host-only; takes effect at the next route call.
+ */
+#define FGR_DP_AUTO 0
+#define FGR_DP_HEAVY 1
+#define FGR_DP_HLD 2
+FGR_API fgr_status fgr_set_dp_policy(fgr_grid* grid, int32_t policy, int32_t flow_max);
+
 /* fgr_route_batch with the Z middles: zmid_out [num_nodes] DEVICE out (may be NULL):
  * for the listed nets' nodes, mid | lb << 16 of an edge routed as a Z shape
  * (seg bend 2 or 3), -1 otherwise.  Same synchronisation and errors. */

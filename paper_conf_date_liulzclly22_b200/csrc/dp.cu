@@ -17,8 +17,6 @@
 // loop is unrolled exactly).  A "group" of LT lanes evaluates one node: lane l
 // owns layer l of the node's vectors (F rows, B, E — the L parallel computation
 // flows of P:L754-756).  A warp holds G = min(4, 32/LT) groups:
-//   * k_dp_group: nets with <= 32 nodes, G nets per warp, each group walking
-//     its net's nodes children-first (parent[i] < i, so descending index order);
 //   * k_dp_large: nets with > 32 nodes, one 256-thread CTA per net, level by
 //     level, 8*G nodes of a level in flight.
 // All prefix gathers of a net are issued up front (costs are fixed during the
@@ -28,7 +26,6 @@
 
 namespace {
 
-constexpr int kGroupWarps = 4;              // warps per CTA in k_dp_group
 constexpr int kLargeWarps = 16;             // warps per CTA in k_dp_large (one path-walking group each)
 constexpr int kFlowMax = 64;                // largest net of the dataflow kernel by default
 
@@ -174,26 +171,6 @@ __device__ __forceinline__ void gather_task(const GridView& g, const Tabs& t, in
 
 // ------------------------------------------------------------- DP steps (one group of LT lanes)
 
-// S5: child layer = smallest l in the parent's span minimising E_v(l) (R11).
-template <int LT>
-__device__ __forceinline__ uint32_t backtrack_node(const Hdr* h, const Tabs& t, int v) {
-    const int u = t.par[v];
-    const int sp = t.span[u];
-    const int lo = sp >> 4, hi = sp & 15;
-    int lt = lo;
-    uint32_t be = t.E[(size_t)v * LT + lo];
-    for (int l = lo + 1; l <= hi; l++) {
-        const uint32_t e = t.E[(size_t)v * LT + l];
-        if (e < be) { be = e; lt = l; }
-    }
-    const int ls = t.recE[(size_t)v * LT + lt];
-    t.span[v] = t.recB[(size_t)v * LT + ls];
-    const bool straight = (t.x[v] == t.x[u]) || (t.y[v] == t.y[u]);
-    const uint32_t bend = seg_bend(h->dir[ls], h->dir[lt], straight);
-    return bend | ((uint32_t)ls << 8) | ((uint32_t)lt << 16) | ((uint32_t)straight << 24);
-}
-
-
 // Packed G entry of a node without light children (K = V): value V(a,b), span (zlo[a], b).
 __device__ __forceinline__ unsigned long long gclosed(const Hdr* h, int a, int b) {
     return ((unsigned long long)(h->viapre[b] - h->viapre[a]) << 8) | (unsigned)(h->zlo[a] << 4) | (unsigned)b;
@@ -207,301 +184,6 @@ __device__ __forceinline__ unsigned long long tree_min(unsigned long long (&k)[N
 #pragma unroll
         for (int i = 0; i + s < N; i += 2 * s) k[i] = k[i + s] < k[i] ? k[i + s] : k[i];
     return k[0];
-}
-
-// Product-form node step (the identity of the k_dp_large header comment) for one lane
-// group of a warp whose groups run in lockstep: every lane of the warp calls it (the
-// shuffles are full-warp).  All children of v are final; the highest-index child plays
-// the "heavy" child, the others fold into G.  Writes E_v / recE_v / recB_v, or returns
-// the root's packed (total, lo, hi) key when is_root.
-template <int LT>
-__device__ __forceinline__ unsigned long long node_step_group(const Hdr* h, const LaneConst<LT>& c, const Tabs& t,
-                                                              const WScr& w, int v, bool act, bool is_root, int gl,
-                                                              int gbase, int nH, int nV, uint32_t opp,
-                                                              const uint32_t* hm) {
-    const uint32_t cm = act ? t.aux[v] : 0u;
-    const int hc = cm ? 31 - __clz(cm) : -1;
-    const uint32_t lm = hc >= 0 ? (cm & ~(1u << hc)) : 0u;
-    const bool light = lm != 0;
-    if (light) {   // K rows from the light children, suffix minima over hi (lane = lo)
-        const int lo = gl;
-        uint32_t acc[LT];
-#pragma unroll
-        for (int hi = 0; hi < LT; hi++) acc[hi] = hi >= lo ? c.vme[hi] : FGR_INF;
-        uint32_t lmm = lm;
-        while (lmm) {
-            const int ch = __ffs(lmm) - 1;
-            lmm &= lmm - 1;
-            const uint32_t* Ec = t.E + (size_t)ch * LT;
-            uint32_t run = FGR_INF;
-#pragma unroll
-            for (int hi = 0; hi < LT; hi++) {
-                const uint32_t e = Ec[hi];
-                if (hi >= lo) { run = min(run, e); acc[hi] = sat_add(acc[hi], run); }
-            }
-        }
-        unsigned long long run = ~0ull;
-#pragma unroll
-        for (int hi = LT - 1; hi >= 0; hi--)
-            if (hi >= lo) {
-                const unsigned long long key = ((unsigned long long)acc[hi] << 8) | (unsigned)(lo << 4) | (unsigned)hi;
-                run = key < run ? key : run;
-                w.R[lo * LT + hi] = run;
-            }
-    }
-    __syncwarp();
-    if (light) {   // column prefix over lo: G(a, b) = min_{lo <= a} R(lo, b) (lane = b)
-        unsigned long long pr = ~0ull;
-#pragma unroll
-        for (int a = 0; a < LT; a++)
-            if (a <= gl) {
-                const unsigned long long x = w.R[a * LT + gl];
-                pr = x < pr ? x : pr;
-                w.R[a * LT + gl] = pr;
-            }
-    }
-    __syncwarp();
-    const uint32_t eh = (act && hc >= 0) ? t.E[(size_t)hc * LT + gl] : FGR_INF;
-    int plo = -1, phi = -1;
-    if (act) { plo = t.plo[v]; phi = t.phi[v]; }
-    int a0, b0;
-    if (is_root) { a0 = plo >= 0 ? plo : LT - 1; b0 = plo >= 0 ? phi : 0; }
-    else { a0 = gl; b0 = gl; if (plo >= 0) { a0 = min(a0, plo); b0 = max(b0, phi); } }
-    unsigned long long kk[LT];
-    uint32_t va0 = 0, vb0 = 0, za0 = 0;
-#pragma unroll
-    for (int l = 0; l < LT; l++) {
-        va0 = (l == a0) ? c.vp[l] : va0;
-        vb0 = (l == b0) ? c.vp[l] : vb0;
-        za0 = (l == a0) ? c.zl[l] : za0;
-    }
-#pragma unroll
-    for (int l = 0; l < LT; l++) {
-        const uint32_t e = __shfl_sync(0xffffffffu, eh, (gbase + l) & 31);
-        if (light) {
-            const unsigned long long gk = w.R[min(a0, l) * LT + max(b0, l)];
-            kk[l] = ((unsigned long long)sat_add(e, (uint32_t)(gk >> 8)) << 8) | (gk & 0xFFull);
-        } else {
-            const bool la = l < a0, lb = l > b0;
-            const uint32_t va = la ? c.vp[l] : va0, vb = lb ? c.vp[l] : vb0;
-            const uint32_t za = la ? c.zl[l] : za0;
-            const uint32_t bb = lb ? (uint32_t)l : (uint32_t)b0;
-            kk[l] = ((unsigned long long)sat_add(e, vb - va) << 8) | (za << 4) | bb;
-        }
-    }
-    unsigned long long bk = tree_min<LT>(kk);
-    if (hc < 0) bk = ((unsigned long long)(vb0 - va0) << 8) | (za0 << 4) | (unsigned)b0;   // leaf: no child term
-    if (is_root) return bk;
-    const uint32_t Bv = (uint32_t)(bk >> 8);
-    uint32_t Bl[LT];
-#pragma unroll
-    for (int l = 0; l < LT; l++) Bl[l] = __shfl_sync(0xffffffffu, Bv, (gbase + l) & 31);
-    if (!act) return 0;
-    t.recB[(size_t)v * LT + gl] = (uint8_t)(bk & 0xFF);
-    const int u = t.par[v];
-    const int xv = t.x[v], yv = t.y[v], xu = t.x[u], yu = t.y[u];
-    uint32_t best = FGR_INF;
-    int bls = gl;
-    if (hm) {                                     // hybrid edge: E_v(lt) = min_ls [B_v(ls) + M_e(ls, lt)]
-#pragma unroll
-        for (int l = 0; l < LT; l++) {
-            const uint32_t cst = sat_add(Bl[l], hm[l]);
-            if (cst < best) { best = cst; bls = l; }
-        }
-    } else if (yv == yu || xv == xu) {            // straight: one leg on ls = lt (R7)
-        const int de = (yv == yu) ? 0 : 1;
-        if (c.my_dir == de) {
-            const uint32_t leg = de == 0 ? t.legH[(size_t)v * 2 * nH + c.my_slot] : t.legV[(size_t)v * 2 * nV + c.my_slot];
-            best = sat_add(Bv, leg);
-        }
-    } else {
-        const bool b0v = c.my_dir == 1;
-        const uint32_t leg2 = b0v ? t.legV[((size_t)v * 2 + 1) * nV + c.my_slot] : t.legH[((size_t)v * 2 + 1) * nH + c.my_slot];
-        const uint32_t* l1 = b0v ? t.legH + (size_t)v * 2 * nH : t.legV + (size_t)v * 2 * nV;
-        int sidx = 0;
-#pragma unroll
-        for (int l = 0; l < LT; l++)
-            if ((opp >> l) & 1u) {
-                const uint32_t cst = sat_add(sat_add(sat_add(Bl[l], l1[sidx]), c.vme[l]), leg2);
-                if (cst < best) { best = cst; bls = l; }
-                sidx++;
-            }
-    }
-    t.E[(size_t)v * LT + gl] = best;
-    t.recE[(size_t)v * LT + gl] = (uint8_t)bls;
-    return 0;
-}
-
-// ------------------------------------------------------------- group kernel (nets <= 32 nodes)
-
-template <int LT, int kMC>
-__global__ void __launch_bounds__(32 * kGroupWarps) k_dp_group(GridView g, NetsView nv, const int32_t* __restrict__ list,
-                                                               int count, Out o, int commit, HybView hy) {
-    constexpr int G = groups_of(LT);
-    extern __shared__ __align__(16) unsigned char smem[];
-    Hdr* h = reinterpret_cast<Hdr*>(smem);
-    init_hdr(h, g);
-    __syncthreads();
-    const int nH = g.h.cnt, nV = g.v.cnt;
-    const int warp = threadIdx.x >> 5, lane = lane_id();
-    const int idx0 = (blockIdx.x * kGroupWarps + warp) * G;
-    if (idx0 >= count) return;
-    const int gi = lane / LT < G ? lane / LT : G;      // my group (G = idle lane)
-    const int gl = lane - gi * LT;                     // my layer inside the group
-    const size_t tb = tabs_bytes(kMC, LT, nH, nV, false), wb = wscr_bytes(LT);
-    unsigned char* wbase = smem + a16(sizeof(Hdr)) + (size_t)warp * G * (tb + wb);
-    auto tabs_of = [&](int q) { return carve_tabs(wbase + (size_t)q * (tb + wb), kMC, LT, nH, nV, false); };
-    auto wscr_of = [&](int q) { return carve_wscr(wbase + (size_t)q * (tb + wb) + tb, LT); };
-    LaneConst<LT> c;
-    c.load(h, gl);
-    // nets of the G groups
-    int net_l = -1, a0_l = 0, m_l = 0, hn_l = -1;
-    if (lane < G && idx0 + lane < count) {
-        net_l = list[idx0 + lane];
-        a0_l = nv.off[net_l];
-        m_l = nv.off[net_l + 1] - a0_l;
-        if (hy.net) hn_l = hy.net[net_l];
-    }
-    int mq[G], aq[G];
-#pragma unroll
-    for (int q = 0; q < G; q++) { mq[q] = __shfl_sync(0xffffffffu, m_l, q); aq[q] = __shfl_sync(0xffffffffu, a0_l, q); }
-    int my_m = 0, my_a = 0, my_hn = -1;
-#pragma unroll
-    for (int q = 0; q < G; q++) {
-        const int hq = __shfl_sync(0xffffffffu, hn_l, q);
-        my_m = (gi == q) ? mq[q] : my_m;
-        my_a = (gi == q) ? aq[q] : my_a;
-        my_hn = (gi == q) ? hq : my_hn;
-    }
-    Flat<G> nodes;
-    nodes.build(mq);
-    // node data, zeroed child masks
-    for (int it = lane; it < nodes.total(); it += 32) {
-        const int q = nodes.group(it), i = it - nodes.base(q);
-        int a = 0;
-#pragma unroll
-        for (int k = 0; k < G; k++) a = (k == q) ? aq[k] : a;
-        const Tabs t = tabs_of(q);
-        t.x[i] = nv.x[a + i]; t.y[i] = nv.y[a + i]; t.par[i] = (int16_t)nv.par[a + i];
-        t.plo[i] = nv.plo[a + i]; t.phi[i] = nv.phi[a + i];
-        t.aux[i] = 0;
-    }
-    __syncwarp();
-    for (int it = lane; it < nodes.total(); it += 32) {
-        const int q = nodes.group(it), i = it - nodes.base(q);
-        if (i > 0) { const Tabs t = tabs_of(q); atomicOr(&t.aux[t.par[i]], 1u << i); }
-    }
-    // all prefix gathers of the G nets up front
-    int tq[G];
-#pragma unroll
-    for (int q = 0; q < G; q++) tq[q] = mq[q] > 1 ? 4 * (mq[q] - 1) : 0;
-    Flat<G> tasks;
-    tasks.build(tq);
-    for (int it = lane; it < tasks.total(); it += 32) {
-        const int q = tasks.group(it);
-        gather_task(g, tabs_of(q), it - tasks.base(q));
-    }
-    __syncwarp();
-    // bottom-up DP: descending node index is children-first (parent[i] < i)
-    int maxm = 0;
-#pragma unroll
-    for (int q = 0; q < G; q++) maxm = max(maxm, mq[q]);
-    const Tabs t = tabs_of(gi < G ? gi : 0);
-    const WScr w = wscr_of(gi < G ? gi : 0);
-    const bool glane = gi < G && gl < LT;
-    unsigned long long rootkey = ~0ull;
-    const uint32_t opp = c.my_dir == 1 ? c.hmask : (~c.hmask & ((1u << LT) - 1u));   // bend partner layers
-    const int gbase = (gi < G ? gi : 0) * LT;
-    for (int k = 0; k + 1 < maxm; k++) {
-        const int v = my_m - 1 - k;
-        const uint32_t* hm = nullptr;   // hybrid edge: its transfer matrix column for lt = gl
-        if (my_hn >= 0 && glane && v >= 1) {
-            const int hs = hy.slot[my_a + v];
-            if (hs >= 0) hm = hy.M + ((size_t)hs * LT + gl) * LT;
-        }
-        node_step_group<LT>(h, c, t, w, v, glane && v >= 1, false, gl, gbase, nH, nV, opp, hm);
-        __syncwarp();
-    }
-    // root (generalised Eq. (4))
-    {
-        const bool act = glane && my_m >= 2;
-        const unsigned long long rk = node_step_group<LT>(h, c, t, w, 0, act, true, gl, gbase, nH, nV, opp, nullptr);
-        if (act && gl == 0) { t.span[0] = (uint8_t)(rk & 0xFF); rootkey = rk; }
-        __syncwarp();
-    }
-    // depth by pointer jumping (aux = ancestor), then a level-ordered backtrack
-    for (int it = lane; it < nodes.total(); it += 32) {
-        const int q = nodes.group(it), i = it - nodes.base(q);
-        const Tabs tt = tabs_of(q);
-        tt.depth[i] = i ? 1 : 0;
-        tt.aux[i] = i ? (uint32_t)tt.par[i] : 0u;
-    }
-    __syncwarp();
-#pragma unroll 1
-    for (int r = 1; r < kMC; r <<= 1) {   // depth < kMC: log2(kMC) pointer-jumping rounds
-        uint32_t nd[G], na[G];
-#pragma unroll
-        for (int s = 0; s < G; s++) {
-            const int it = lane + 32 * s;
-            if (it < nodes.total()) {
-                const int q = nodes.group(it), i = it - nodes.base(q);
-                const Tabs tt = tabs_of(q);
-                const uint32_t an = tt.aux[i];
-                nd[s] = tt.depth[i] + tt.depth[an];
-                na[s] = tt.aux[an];
-            }
-        }
-        __syncwarp();
-#pragma unroll
-        for (int s = 0; s < G; s++) {
-            const int it = lane + 32 * s;
-            if (it < nodes.total()) {
-                const int q = nodes.group(it), i = it - nodes.base(q);
-                const Tabs tt = tabs_of(q);
-                tt.depth[i] = (uint16_t)nd[s];
-                tt.aux[i] = na[s];
-            }
-        }
-        __syncwarp();
-    }
-    int maxd = 0;
-    for (int it = lane; it < nodes.total(); it += 32) {
-        const int q = nodes.group(it), i = it - nodes.base(q);
-        maxd = max(maxd, (int)tabs_of(q).depth[i]);
-    }
-#pragma unroll
-    for (int off = 16; off; off >>= 1) maxd = max(maxd, __shfl_xor_sync(0xffffffffu, maxd, off));
-    for (int d = 1; d <= maxd; d++) {
-        for (int it = lane; it < nodes.total(); it += 32) {
-            const int q = nodes.group(it), i = it - nodes.base(q);
-            const Tabs tt = tabs_of(q);
-            if (tt.depth[i] == d) {
-                const uint32_t s = backtrack_node<LT>(h, tt, i);
-                tt.legH[(size_t)i * 2 * nH] = s;       // keep the route for the outputs and the commit
-            }
-        }
-        __syncwarp();
-    }
-    // outputs and commit
-    for (int it = lane; it < nodes.total(); it += 32) {
-        const int q = nodes.group(it), i = it - nodes.base(q);
-        const Tabs tt = tabs_of(q);
-        const uint32_t s = i ? tt.legH[(size_t)i * 2 * nH] : 0xFFFFFFFFu;
-        int a = 0;
-#pragma unroll
-        for (int k = 0; k < G; k++) a = (k == q) ? aq[k] : a;
-        if (o.rec_seg) o.rec_seg[o.rec_off[o.list_base + idx0 + q] + i] = s;
-        else o.seg[a + i] = s;
-        if (commit && i > 0) {
-            const int u = tt.par[i];
-            commit_edge(g, h, tt.x[i], tt.y[i], tt.x[u], tt.y[u], s, hyb_z(hy, a + i, s, LT));
-        }
-    }
-    if (glane && gl == 0 && my_m >= 1) {
-        const uint32_t total = my_m >= 2 ? (uint32_t)(rootkey >> 8) : 0u;
-        if (o.rec_seg) o.rec_cost[o.list_base + idx0 + gi] = total;
-        else o.cost[list[idx0 + gi]] = total;
-    }
 }
 
 // ------------------------------------------------------------- CTA kernel (nets > 32 nodes)
@@ -1511,33 +1193,21 @@ __global__ void __launch_bounds__(256) k_commit_records(GridView g, NetsView nv,
 }
 
 // ------------------------------------------------------------- host side
-size_t smem_group(int L, int nH, int nV, int mc) {
-    return a16(sizeof(Hdr)) + (size_t)kGroupWarps * groups_of(L) * (tabs_bytes(mc, L, nH, nV, false) + wscr_bytes(L));
-}
-
 size_t smem_large(int L, int nH, int nV, int m) {
     return a16(sizeof(Hdr)) + (size_t)kLargeWarps * wscr_bytes(L) + tabs_bytes(m, L, nH, nV, true) +
            (size_t)kMR * L * ((L + 3) & ~3) * 4;
 }
 
-// FGR_LARGE_KERNEL=old / FGR_GROUP_KERNEL=old select the previous lane-group kernel for nets of 3..32 nodes (A/B runs).
-bool use_old_large() {
-    static int v = -1;
-    if (v < 0) {
-        const char* s = getenv("FGR_LARGE_KERNEL");
-        v = (s && s[0] == 'o') ? 1 : 0;
-    }
-    return v == 1;
+}  // namespace
+
+// Largest net the shared-memory heavy-path kernel (k_dp_large) holds; bigger nets take k_dp_hld.
+int fgr_large_limit(const fgr_grid* g) {
+    int m = 2048;
+    while (m > FGR_SMALL_NET && smem_large(g->L, g->nH, g->nV, m) + 64 > (size_t)g->max_smem) m -= 16;
+    return m;
 }
 
-bool use_old_group() {
-    static int v = -1;
-    if (v < 0) {
-        const char* s = getenv("FGR_GROUP_KERNEL");
-        v = (s && s[0] == 'o') ? 1 : 0;
-    }
-    return v == 1;
-}
+namespace {
 
 template <int LT>
 cudaError_t launch_lt(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int nlarge, int nmidL,
@@ -1554,50 +1224,64 @@ cudaError_t launch_lt(fgr_grid* g, cudaStream_t st, const NetsView& nv, const in
         if (e == cudaSuccess)
             e = cudaFuncSetAttribute(k_large_prep<LT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                      g->max_smem - (int)fa.sharedSizeBytes);
-        if (e == cudaSuccess) e = cudaFuncGetAttributes(&fa, k_dp_group<LT, FGR_SMALL_NET>);
-        if (e == cudaSuccess)
-            e = cudaFuncSetAttribute(k_dp_group<LT, FGR_SMALL_NET>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                     g->max_smem - (int)fa.sharedSizeBytes);
-        if (e == cudaSuccess) e = cudaFuncGetAttributes(&fa, k_dp_group<LT, FGR_MID_NET>);
-        if (e == cudaSuccess)
-            e = cudaFuncSetAttribute(k_dp_group<LT, FGR_MID_NET>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                     g->max_smem - (int)fa.sharedSizeBytes);
         if (e != cudaSuccess) return e;
         configured = true;
     }
     const GridView& v = g->view;
     const HybView hyv = g->hy.view();
-    // Launch units: large-net size buckets 0..4 (the list is in descending size: > 512,
-    // 257..512, 129..256, 65..128, 33..64 nodes; one bucket unless lsplit is given), then
-    // the classes 9..32, 3..8 and 2 nodes.  Units are independent nets: each non-empty
-    // unit gets its own stream (forked from and joined back into the caller's stream).
-    static const int kCap[5] = {1 << 30, 512, 256, 128, 64};
-    int cut[6] = {0, nlarge, nlarge, nlarge, nlarge, nlarge};
-    if (lsplit && !use_old_large())
-        for (int s = 1; s <= 4; s++) cut[s] = max(cut[s - 1], min(lsplit[s - 1], nlarge));
+    // Launch units: large-net size buckets (the list is in descending size): above the heavy-path
+    // kernel's shared-memory limit, then > 512, 257..512, 129..256, 65..128, 33..64 nodes (one bucket
+    // unless lsplit is given), then the classes 9..32, 3..8 and 2 nodes.  Units are independent nets:
+    // each non-empty unit gets its own stream (forked from and joined back into the caller's stream).
+    const int lim = fgr_large_limit(g);
     struct Unit { int kind, off, n, cap; };   // kind: 0 large, 1 midL, 2 midS, 3 two
-    Unit units[8];
+    Unit units[10];
     int nu = 0;
-    for (int s = 0; s < 5; s++)
-        if (cut[s + 1] > cut[s]) units[nu++] = Unit{0, cut[s], cut[s + 1] - cut[s], min(kCap[s], maxm_large)};
+    {
+        // thresholds (descending) with the number of large nets above each
+        int thr[5] = {lim, 512, 256, 128, 64}, above[5] = {0, 0, 0, 0, 0};
+        if (lsplit) for (int k = 0; k < 5; k++) above[k] = min(lsplit[k], nlarge);
+        for (int i = 0; i < 5; i++)
+            for (int j = i + 1; j < 5; j++)
+                if (thr[j] > thr[i]) { int x = thr[i]; thr[i] = thr[j]; thr[j] = x; x = above[i]; above[i] = above[j]; above[j] = x; }
+        int prev = 0, cap = maxm_large;
+        for (int k = 0; k <= 5 && prev < nlarge; k++) {
+            const int end = (k < 5 && lsplit) ? max(prev, above[k]) : nlarge;
+            if (end > prev) units[nu++] = Unit{0, prev, end - prev, min(cap, maxm_large)};
+            prev = end;
+            if (k < 5) cap = thr[k];
+        }
+    }
     if (nmidL > 0) units[nu++] = Unit{1, nlarge, nmidL, 0};
     if (nmidS > 0) units[nu++] = Unit{2, nlarge + nmidL, nmidS, 0};
     if (ntwo > 0) units[nu++] = Unit{3, nlarge + nmidL + nmidS, ntwo, 0};
+    // kernel of a large-net unit (grid policy, fgr_set_dp_policy): the contraction kernel above the
+    // shared-memory limit or under FGR_DP_HLD; else the dataflow kernel up to flow_max nodes (FGR_DP_AUTO)
+    // and the heavy-path kernel
+    auto large_kind = [&](int cap) {   // 0 hld, 1 flow, 2 heavy-path
+        if (cap > lim || g->dp_policy == FGR_DP_HLD) return 0;
+        if (g->dp_policy == FGR_DP_AUTO && cap <= g->flow_max && cap <= fgr_flow_max_nodes(g)) return 1;
+        return 2;
+    };
     const bool fork = nu > 1;
     cudaError_t e;
+    // global workspaces of the large-net units (one region each: the units run concurrently)
+    size_t wsoff[8] = {0}, wstot = 0;
+    unsigned char* wsb = nullptr;
+    {
+        for (int ui = 0; ui < nu; ui++)
+            if (units[ui].kind == 0 && large_kind(units[ui].cap) == 0) { wsoff[ui] = wstot; wstot += (fgr_hld_ws_bytes(g, units[ui].n, units[ui].cap) + 255) & ~(size_t)255; }
+        if (wstot > 0) {
+            wsb = (unsigned char*)fgr_scratch(g->s_hldw, wstot, &e);
+            if (e != cudaSuccess) return e;
+        }
+    }
     if (fork) {
         // recorded before any launch: the side streams wait for the refresh, not for each other
         if ((e = cudaEventRecord(g->ev_fork, st)) != cudaSuccess) return e;
         for (int i = 0; i + 1 < nu; i++)
             if ((e = cudaStreamWaitEvent(g->side[i], g->ev_fork, 0)) != cudaSuccess) return e;
     }
-    // Nets of up to kFlowMax nodes take the dataflow kernel (dp_walk.cu); bigger ones the
-    // heavy-path kernel below, whose root-path transfer matrices shorten the long chains
-    // (measured on t9, 3 interleaved runs each: cut 128 / 64 / 32 = 20.34 / 20.18 / 20.12 ms
-    // per step, profiles/r01h_flowmax_ab2.txt; 64 keeps the flow kernel on the default path).  FGR_FLOW_MAX
-    // overrides the cut for A/B runs.
-    static int flow_cap = -1;
-    if (flow_cap < 0) { const char* s = getenv("FGR_FLOW_MAX"); flow_cap = s ? atoi(s) : kFlowMax; }
     for (int ui = 0; ui < nu; ui++) {
         const Unit& un = units[ui];
         cudaStream_t su = ui == 0 ? st : g->side[ui - 1];
@@ -1606,7 +1290,11 @@ cudaError_t launch_lt(fgr_grid* g, cudaStream_t st, const NetsView& nv, const in
         const int32_t* l = list + un.off;
         const int n = un.n;
         const int ps = fgr_prof_begin(g, un.kind == 0 ? PROF_DP_LARGE : PROF_DP_SMALL, su);
-        if (un.kind == 0 && !use_old_large() && un.cap <= fgr_flow_max_nodes(g) && un.cap <= flow_cap) {
+        const int lk = un.kind == 0 ? large_kind(un.cap) : -1;
+        if (lk == 0) {
+            e = fgr_launch_hld(g, su, nv, l, n, un.cap, os, commit, prep.hld, wsb ? wsb + wsoff[ui] : nullptr);
+            if (e != cudaSuccess) return e;
+        } else if (lk == 1) {
             e = fgr_launch_flow(g, su, nv, l, n, un.cap, os, commit, prep);
             if (e != cudaSuccess) return e;
         } else if (un.kind == 0) {
@@ -1624,20 +1312,8 @@ cudaError_t launch_lt(fgr_grid* g, cudaStream_t st, const NetsView& nv, const in
             e = cudaLaunchKernelEx(&cfg, k_dp_large<LT>, v, nv, l, n, os, commit ? 1 : 0, prep, hyv);
             if (e != cudaSuccess) return e;
         } else if (un.kind <= 2) {
-            if (use_old_group()) {
-                const int per_cta = kGroupWarps * groups_of(LT);
-                if (un.kind == 1)
-                    k_dp_group<LT, FGR_SMALL_NET><<<(n + per_cta - 1) / per_cta, 32 * kGroupWarps,
-                                                     smem_group(LT, g->nH, g->nV, FGR_SMALL_NET), su>>>(
-                        v, nv, l, n, os, commit ? 1 : 0, hyv);
-                else
-                    k_dp_group<LT, FGR_MID_NET><<<(n + per_cta - 1) / per_cta, 32 * kGroupWarps,
-                                                   smem_group(LT, g->nH, g->nV, FGR_MID_NET), su>>>(
-                        v, nv, l, n, os, commit ? 1 : 0, hyv);
-            } else {
-                e = fgr_launch_walk(g, su, nv, l, n, un.kind == 1 ? FGR_SMALL_NET : FGR_MID_NET, os, commit);
-                if (e != cudaSuccess) return e;
-            }
+            e = fgr_launch_walk(g, su, nv, l, n, un.kind == 1 ? FGR_SMALL_NET : FGR_MID_NET, os, commit);
+            if (e != cudaSuccess) return e;
         } else {
             k_dp_two<LT><<<(n + kTwoThreads - 1) / kTwoThreads, kTwoThreads, 0, su>>>(v, nv, l, n, os, commit ? 1 : 0,
                                                                                       hyv);
@@ -1657,7 +1333,6 @@ cudaError_t launch_lt(fgr_grid* g, cudaStream_t st, const NetsView& nv, const in
 
 }  // namespace
 
-size_t fgr_dp_smem_small(const fgr_grid* g) { return smem_group(g->L, g->nH, g->nV, FGR_SMALL_NET); }
 
 size_t fgr_dp_smem_large(const fgr_grid* g, int m) { return smem_large(g->L, g->nH, g->nV, m); }
 
@@ -1665,7 +1340,7 @@ cudaError_t fgr_launch_dp(fgr_grid* g, cudaStream_t st, const NetsView& nv, cons
                           int nmidS, int ntwo, int maxm_large, uint32_t* seg_out, uint32_t* cost_out, uint32_t* rec_seg,
                           const int32_t* rec_off, uint32_t* rec_cost, int list_base, bool commit, const Prep* prep,
                           const int* lsplit) {
-    const Prep pz = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
+    const Prep pz = {};
     const Prep& pp = prep ? *prep : pz;
     Out o;
     o.seg = seg_out; o.cost = cost_out; o.rec_seg = rec_seg; o.rec_off = rec_off; o.rec_cost = rec_cost;

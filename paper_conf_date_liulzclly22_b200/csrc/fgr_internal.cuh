@@ -76,6 +76,23 @@ struct NetsView {
 };
 
 // ------------------------------------------------------------------ host state
+// Heavy-path decomposition of every net routed by k_dp_hld (dp_hld.cu), computed once per
+// stage by k_hld_prep.  Global arrays indexed by global node index (a0 + local), values
+// net-local (uint16): heavy child (0xFFFF = leaf), child CSR (cs[a0+v] .. cs[a0+v+1], with
+// cs of local m implied = m - 1), path nodes pn (paths stored bottom -> head, paths ordered
+// by light depth, deepest first), path starts po[a0 + q] (q < npaths; the end of the last is m),
+// path light depth pr[a0 + q]; info[net] = npaths | rounds << 16.
+struct HldPrep {
+    const uint16_t* hv;
+    const uint16_t* cs;
+    const uint16_t* cl;
+    const uint16_t* pn;
+    const uint16_t* po;
+    const uint8_t* pr;
+    const int32_t* info;
+    const uint8_t* ld;     // light depth of every node (= the round of its path)
+};
+
 // Per-node results of the large-net tree analysis (global, indexed by global node index).
 struct Prep {
     const uint16_t* cs;    // child CSR start (net-local); cs of local m is m - 1 and not stored
@@ -85,6 +102,7 @@ struct Prep {
     const uint16_t* pq;    // path queue (path tops, deepest first)
     const int32_t* npaths; // [num_nets]
     const uint16_t* rpos;  // index along the root path (0xFFFF off it)
+    HldPrep hld;           // heavy-path decomposition for k_dp_hld (the default large-net kernel)
 };
 
 // Hybrid L+Z tables of the current route call (hybrid.cu).  Slots number the hybrid
@@ -130,7 +148,7 @@ struct PlanCache {
     int* h_maxm = nullptr;     // [B] max nodes of a large net in the batch
     int* h_ntwo = nullptr;     // [B] 2-node nets (the tail of each batch in exec order)
     int* h_n9 = nullptr;       // [B] nets with 9..32 nodes
-    int* h_lsplit = nullptr;   // [B][4] large nets with more than 512, 256, 128, 64 nodes
+    int* h_lsplit = nullptr;   // [B][5] large nets with more than fgr_large_limit, 512, 256, 128, 64 nodes
     const int32_t* exec = nullptr;  // exec order actually used (order itself, or a re-sorted copy)
     bool prep_valid = false;        // large-net tree analysis computed for these nets
     Prep prep{};
@@ -180,6 +198,9 @@ struct fgr_grid {
     int rank = 0, world = 1;
     Scratch s_rec[4];
     Scratch s_prep;
+    Scratch s_hldp;             // k_hld_prep outputs (per stage)
+    Scratch s_hldt;             // k_hld_prep temporaries for nets too large for shared memory
+    Scratch s_hldw;             // k_dp_hld global workspaces (per CTA) for large nets
     fgr_stats stats{};
     int max_smem = 0;
     int num_sms = 0;
@@ -189,6 +210,9 @@ struct fgr_grid {
     cudaEvent_t ev_fork = nullptr, ev_join[FGR_SIDE_STREAMS] = {};
     // hybrid L+Z pattern routing (fgr_set_pattern): edges with t1 <= HPWL <= t2; t1 > t2 = L only
     int hyb_t1 = 1, hyb_t2 = 0;
+    // large-net DP kernel selection (fgr_set_dp_policy)
+    int dp_policy = FGR_DP_AUTO;
+    int flow_max = 64;
     HybState hy;
     Scratch s_hyb[3];
     Scratch s_rip[6];          // rip-up extraction and task graph (ripup.cu)
@@ -224,7 +248,6 @@ cudaError_t fgr_launch_large_prep(fgr_grid* g, cudaStream_t st, const NetsView& 
                                   uint16_t* rpos, int32_t* np);
 cudaError_t fgr_launch_commit(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int count,
                               const uint32_t* rec_seg, const int32_t* rec_off, int list_base);
-size_t fgr_dp_smem_small(const fgr_grid* g);
 fgr_status fgr_hyb_prepare(fgr_grid* g, cudaStream_t st, const NetsView& nv, int num_nets, int num_nodes,
                            const int32_t* exec, int R, const int32_t* boff, int nb, int32_t* zmid);
 cudaError_t fgr_launch_hyb_tm(fgr_grid* g, cudaStream_t st, const NetsView& nv, int slot0, int n);
@@ -236,6 +259,14 @@ cudaError_t fgr_launch_walk(fgr_grid* g, cudaStream_t st, const NetsView& nv, co
 cudaError_t fgr_launch_flow(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int n, int maxm,
                             const Out& o, bool commit, const Prep& prep);
 int fgr_flow_max_nodes(const fgr_grid* g);
+int fgr_large_limit(const fgr_grid* g);
+cudaError_t fgr_launch_hld_prep(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int count,
+                                int maxm, uint16_t* hv, uint16_t* cs, uint16_t* cl, uint16_t* pn, uint16_t* po,
+                                uint8_t* pr, int32_t* info, uint8_t* ld);
+// ws: global workspace of fgr_hld_ws_bytes(g, n, maxm) bytes (distinct per concurrent launch)
+cudaError_t fgr_launch_hld(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int n, int maxm,
+                           const Out& o, bool commit, const HldPrep& hp, unsigned char* ws);
+size_t fgr_hld_ws_bytes(const fgr_grid* g, int n, int maxm);
 
 // Output of a DP launch: direct (by node / net id) or route records (multi-GPU).
 struct Out {

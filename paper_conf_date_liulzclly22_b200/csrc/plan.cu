@@ -404,7 +404,7 @@ __global__ void k_finalize(int N, const int* __restrict__ counters, const unsign
                            const unsigned long long* __restrict__ bkeys, const int* __restrict__ msize,
                            const int* __restrict__ segb, int* __restrict__ order, int* __restrict__ batch_of_net,
                            int* __restrict__ nlarge, int* __restrict__ maxm, unsigned long long* __restrict__ segsum,
-                           int* __restrict__ ntwo, int* __restrict__ n9, int* __restrict__ lsplit) {
+                           int* __restrict__ ntwo, int* __restrict__ n9, int* __restrict__ lsplit, int lim) {
     const int i = blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= N) return;
     const int R = N - counters[0];
@@ -419,10 +419,12 @@ __global__ void k_finalize(int N, const int* __restrict__ counters, const unsign
         if (m > FGR_SMALL_NET) {
             atomicAdd(&nlarge[c], 1);
             atomicMax(&maxm[c], m);
-            if (m > 64) atomicAdd(&lsplit[4 * c + 3], 1);   // large-net size buckets (> 512, 256, 128, 64)
-            if (m > 128) atomicAdd(&lsplit[4 * c + 2], 1);
-            if (m > 256) atomicAdd(&lsplit[4 * c + 1], 1);
-            if (m > 512) atomicAdd(&lsplit[4 * c + 0], 1);
+            // large-net size buckets (> fgr_large_limit, 512, 256, 128, 64)
+            if (m > 64) atomicAdd(&lsplit[5 * c + 4], 1);
+            if (m > 128) atomicAdd(&lsplit[5 * c + 3], 1);
+            if (m > 256) atomicAdd(&lsplit[5 * c + 2], 1);
+            if (m > 512) atomicAdd(&lsplit[5 * c + 1], 1);
+            if (m > lim) atomicAdd(&lsplit[5 * c + 0], 1);
         }
         // per-batch sum of dirty-segment bounds (refresh launch sizing); keys are
         // batch-sorted, so a warp almost always shares one batch id
@@ -465,10 +467,8 @@ int bits_for(long long v) {
 }  // namespace
 
 // largest net the CTA path can hold (shared memory), capped by its depth arrays
-static int max_large_nodes(const fgr_grid* g) {
-    int m = 2048;
-    while (m > FGR_SMALL_NET && fgr_dp_smem_large(g, m) + 64 > (size_t)g->max_smem) m -= 16;
-    return m;
+static int max_large_nodes(const fgr_grid*) {
+    return 65535;   // net-local uint16 indices; nets above fgr_large_limit take k_dp_hld (global workspace)
 }
 
 extern "C" FGR_API fgr_status fgr_plan(fgr_grid* g, const fgr_nets* nets, int32_t* batch_of_net, int32_t* order,
@@ -576,7 +576,7 @@ extern "C" FGR_API fgr_status fgr_plan(fgr_grid* g, const fgr_nets* nets, int32_
         FGR_CHECK_CUDA(g, cudaGetLastError());
     }
     // colouring
-    auto* bc = take<int>(g, 11, 9 * ((size_t)R + 1), &e);   // bcount | nlarge | maxm | ntwo | n9 | lsplit[4]
+    auto* bc = take<int>(g, 11, 10 * ((size_t)R + 1), &e);   // bcount | nlarge | maxm | ntwo | n9 | lsplit[5]
     if (e != cudaSuccess) return fgr_cuda_fail(g, e, "plan batch scratch");
     int* d_bcount = bc;
     int* d_nlarge = bc + (R + 1);
@@ -584,7 +584,7 @@ extern "C" FGR_API fgr_status fgr_plan(fgr_grid* g, const fgr_nets* nets, int32_
     int* d_ntwo = bc + 3 * (R + 1);
     int* d_n9 = bc + 4 * (R + 1);
     int* d_ls = bc + 5 * (R + 1);
-    FGR_CHECK_CUDA(g, cudaMemsetAsync(bc, 0, 9 * sizeof(int) * ((size_t)R + 1), st));
+    FGR_CHECK_CUDA(g, cudaMemsetAsync(bc, 0, 10 * sizeof(int) * ((size_t)R + 1), st));
     FGR_CHECK_CUDA(g, cudaMemsetAsync(color, 0xFF, sizeof(int) * ((size_t)N + 1), st));
     FGR_CHECK_CUDA(g, cudaMemsetAsync(batch_of_net, 0xFF, sizeof(int) * (size_t)N, st));
     if (R > 0) {
@@ -627,7 +627,7 @@ extern "C" FGR_API fgr_status fgr_plan(fgr_grid* g, const fgr_nets* nets, int32_
     auto* segsum = (unsigned long long*)box_r;   // box_r no longer needed after colouring
     FGR_CHECK_CUDA(g, cudaMemsetAsync(segsum, 0, sizeof(unsigned long long) * ((size_t)R + 1), st));
     k_finalize<<<(N + 255) / 256, 256, 0, st>>>(N, counters, keys_s, bkeys_s, msize, segb, order, batch_of_net,
-                                                d_nlarge, d_maxm, segsum, d_ntwo, d_n9, d_ls);
+                                                d_nlarge, d_maxm, segsum, d_ntwo, d_n9, d_ls, fgr_large_limit(g));
     FGR_CHECK_CUDA(g, cudaGetLastError());
     g->stats.kernel_launches += 6;
     int B = 0;
@@ -638,7 +638,7 @@ extern "C" FGR_API fgr_status fgr_plan(fgr_grid* g, const fgr_nets* nets, int32_
         free(c.h_off); free(c.h_nlarge); free(c.h_maxm); free(c.h_segb); free(c.h_ntwo); free(c.h_n9);
         free(c.h_lsplit);
         c.cap = B + 1;
-        c.h_lsplit = (int*)malloc(sizeof(int) * 4 * c.cap);
+        c.h_lsplit = (int*)malloc(sizeof(int) * 5 * c.cap);
         c.h_off = (int*)malloc(sizeof(int) * c.cap);
         c.h_nlarge = (int*)malloc(sizeof(int) * c.cap);
         c.h_maxm = (int*)malloc(sizeof(int) * c.cap);
@@ -652,7 +652,7 @@ extern "C" FGR_API fgr_status fgr_plan(fgr_grid* g, const fgr_nets* nets, int32_
         FGR_CHECK_CUDA(g, cudaMemcpy(c.h_maxm, d_maxm, sizeof(int) * B, cudaMemcpyDeviceToHost));
         FGR_CHECK_CUDA(g, cudaMemcpy(c.h_ntwo, d_ntwo, sizeof(int) * B, cudaMemcpyDeviceToHost));
         FGR_CHECK_CUDA(g, cudaMemcpy(c.h_n9, d_n9, sizeof(int) * B, cudaMemcpyDeviceToHost));
-        FGR_CHECK_CUDA(g, cudaMemcpy(c.h_lsplit, d_ls, sizeof(int) * 4 * B, cudaMemcpyDeviceToHost));
+        FGR_CHECK_CUDA(g, cudaMemcpy(c.h_lsplit, d_ls, sizeof(int) * 5 * B, cudaMemcpyDeviceToHost));
         FGR_CHECK_CUDA(g, cudaMemcpy(c.h_segb, segsum, sizeof(long long) * B, cudaMemcpyDeviceToHost));
     }
     c.valid = true;

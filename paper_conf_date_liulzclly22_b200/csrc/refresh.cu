@@ -254,38 +254,13 @@ __device__ __forceinline__ void refresh_body(const GridView& g, int full) {
 template <int WH, int WV>
 __global__ void __launch_bounds__(256) k_refresh(GridView g, int full) { refresh_body<WH, WV, FGR_CHUNK_SEGS>(g, full); }
 
-// task-size variants for A/B runs (FGR_REFRESH_CHUNK: segments per warp task)
-template <int WH, int WV, int CS>
-__global__ void __launch_bounds__(256) k_refresh_cs(GridView g, int full) { refresh_body<WH, WV, CS>(g, full); }
-
-// register-budget variants for A/B runs (FGR_REFRESH_MINB)
-template <int WH, int WV, int MB>
-__global__ void __launch_bounds__(256, MB) k_refresh_mb(GridView g, int full) {
-    refresh_body<WH, WV, FGR_CHUNK_SEGS>(g, full);
-}
-
-static int refresh_chunk_segs() {
-    static int cs = -1;
-    if (cs < 0) {
-        const char* e = getenv("FGR_REFRESH_CHUNK");
-        cs = e ? atoi(e) : FGR_CHUNK_SEGS;
-        if (cs != 4 && cs != 16) cs = FGR_CHUNK_SEGS;
-    }
-    return cs;
-}
-
+// Launch geometry, fixed by the round-1 A/B measurements: 8 segments per warp task
+// (4 / 16: 2.70 / 2.41 ms vs 2.36 ms per t9 step), the compiler's register budget (64 registers, no
+// spills; 48 / 40 spill and run slower) and up to 8 CTAs per SM (a single resident wave is slower).
 template <int WH, int WV>
 static cudaError_t launch_t(fgr_grid* g, cudaStream_t st, bool full, int blocks) {
-    // FGR_REFRESH_MINB (A/B runs): register budget via min resident CTAs per SM; 0 = compiler's choice
-    static int minb = -1;
-    if (minb < 0) { const char* s = getenv("FGR_REFRESH_MINB"); minb = s ? atoi(s) : 0; }
     const int ps = fgr_prof_begin(g, PROF_REFRESH, st);
-    if (minb == 6) k_refresh_mb<WH, WV, 6><<<blocks, 256, 0, st>>>(g->view, full ? 1 : 0);
-    else if (minb == 5) k_refresh_mb<WH, WV, 5><<<blocks, 256, 0, st>>>(g->view, full ? 1 : 0);
-    else if (minb == 4) k_refresh_mb<WH, WV, 4><<<blocks, 256, 0, st>>>(g->view, full ? 1 : 0);
-    else if (refresh_chunk_segs() == 4) k_refresh_cs<WH, WV, 4><<<blocks, 256, 0, st>>>(g->view, full ? 1 : 0);
-    else if (refresh_chunk_segs() == 16) k_refresh_cs<WH, WV, 16><<<blocks, 256, 0, st>>>(g->view, full ? 1 : 0);
-    else k_refresh<WH, WV><<<blocks, 256, 0, st>>>(g->view, full ? 1 : 0);
+    k_refresh<WH, WV><<<blocks, 256, 0, st>>>(g->view, full ? 1 : 0);
     fgr_prof_end(g, ps, st);
     return cudaGetLastError();
 }
@@ -294,14 +269,11 @@ static cudaError_t launch_t(fgr_grid* g, cudaStream_t st, bool full, int blocks)
 cudaError_t fgr_launch_refresh_sized(fgr_grid* g, cudaStream_t st, bool full, long long max_tasks) {
     (void)max_tasks;
     const GridView& v = g->view;
-    const int cs = refresh_chunk_segs();
+    const int cs = FGR_CHUNK_SEGS;
     const long long tasks = (long long)v.h.lines * ((v.h.nseg + cs - 1) / cs) +
                             (long long)v.v.lines * ((v.v.nseg + cs - 1) / cs);
     int blocks = (int)((tasks + 7) / 8);
-    // FGR_REFRESH_CTAS_PER_SM overrides the cap for A/B runs (grid-stride keeps any grid exact)
-    static int per_sm = -1;
-    if (per_sm < 0) { const char* s = getenv("FGR_REFRESH_CTAS_PER_SM"); per_sm = s ? max(1, atoi(s)) : 8; }
-    const int cap_blocks = g->num_sms * per_sm;
+    const int cap_blocks = g->num_sms * 8;   // grid-stride beyond
     if (blocks > cap_blocks) blocks = cap_blocks;
     if (blocks < 1) blocks = 1;
     g->stats.kernel_launches++;

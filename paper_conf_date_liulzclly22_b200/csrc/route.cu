@@ -52,17 +52,17 @@ __global__ void k_batch_info(int B, const int32_t* __restrict__ boff, const int3
                              const int16_t* __restrict__ y, const int32_t* __restrict__ par,
                              int* __restrict__ nlarge, int* __restrict__ maxm, unsigned long long* __restrict__ segb,
                              int* __restrict__ ntwo, int* __restrict__ n9, unsigned long long* __restrict__ keys,
-                             int* __restrict__ lsplit) {
+                             int* __restrict__ lsplit, int lim) {
     // one block per batch
     const int b = blockIdx.x;
     if (b >= B) return;
-    int nl = 0, mm = 0, n2 = 0, nn9 = 0, ls[4] = {0, 0, 0, 0};
+    int nl = 0, mm = 0, n2 = 0, nn9 = 0, ls[5] = {0, 0, 0, 0, 0};
     unsigned long long sb = 0;
     for (int i = boff[b] + threadIdx.x; i < boff[b + 1]; i += blockDim.x) {
         const int id = order[i];
         const int a0 = off[id], m = off[id + 1] - a0;
         if (m > FGR_SMALL_NET) { nl++; mm = max(mm, m); }
-        ls[0] += m > 512; ls[1] += m > 256; ls[2] += m > 128; ls[3] += m > 64;
+        ls[0] += m > lim; ls[1] += m > 512; ls[2] += m > 256; ls[3] += m > 128; ls[4] += m > 64;
         if (m <= 2) n2++;   // the 2-node kernel also finishes trivial nets
         if (m > FGR_MID_NET && m <= FGR_SMALL_NET) nn9++;
         for (int j = 1; j < m; j++) {
@@ -78,15 +78,17 @@ __global__ void k_batch_info(int B, const int32_t* __restrict__ boff, const int3
     atomicAdd(&segb[b], sb);
     atomicAdd(&ntwo[b], n2);
     atomicAdd(&n9[b], nn9);
-    for (int k = 0; k < 4; k++) atomicAdd(&lsplit[4 * b + k], ls[k]);
+    for (int k = 0; k < 5; k++) atomicAdd(&lsplit[5 * b + k], ls[k]);
 }
 
 __global__ void k_large_list(int n, const int32_t* __restrict__ exec, const int32_t* __restrict__ off,
-                             int32_t* __restrict__ out, int* __restrict__ cnt) {
+                             int32_t* __restrict__ out, int* __restrict__ cnt, int minm) {
     const int i = blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= n) return;
     const int id = exec[i];
-    if (off[id + 1] - off[id] > FGR_SMALL_NET) out[atomicAdd(cnt, 1)] = id;
+    const int m = off[id + 1] - off[id];
+    if (m > FGR_SMALL_NET && m <= minm) out[atomicAdd(cnt, 1)] = id;   // the heavy-path / dataflow kernels' nets
+    if (m > minm) out[n + atomicAdd(cnt + 1, 1)] = id;                 // the nets that take k_dp_hld
 }
 
 __global__ void k_keys_to_ids(int n, const unsigned long long* __restrict__ keys, int32_t* __restrict__ ids) {
@@ -105,6 +107,8 @@ __global__ void k_scatter_records(int n, const int32_t* __restrict__ order, cons
     for (int j = lane_id(); j < m; j += 32) seg_out[a0 + j] = rec_seg[rec_off[warp] + j];
     if (lane_id() == 0) cost_out[id] = rec_cost[warp];
 }
+
+inline size_t a16h(size_t b) { return (b + 15) & ~(size_t)15; }
 
 bool nets_equal(const fgr_nets& a, const fgr_nets& b) {
     return a.num_nets == b.num_nets && a.num_nodes == b.num_nodes && a.node_offset == b.node_offset && a.x == b.x &&
@@ -134,6 +138,17 @@ extern "C" FGR_API fgr_status fgr_split_batch(int32_t count, int32_t nlarge, int
     return FGR_OK;
 }
 
+extern "C" FGR_API fgr_status fgr_set_dp_policy(fgr_grid* g, int32_t policy, int32_t flow_max) {
+    if (!g) return fgr_set_error(FGR_ERR_INVALID, "grid is NULL");
+    if (policy != FGR_DP_AUTO && policy != FGR_DP_HEAVY && policy != FGR_DP_HLD)
+        return fgr_set_error(FGR_ERR_INVALID, "unknown DP policy %d", policy);
+    if (flow_max < FGR_SMALL_NET + 1 || flow_max > 65535) return fgr_set_error(FGR_ERR_INVALID, "flow_max %d out of range", flow_max);
+    if (policy != g->dp_policy) g->cache.prep_valid = false;   // the decompositions to build depend on the policy
+    g->dp_policy = policy;
+    g->flow_max = flow_max;
+    return FGR_OK;
+}
+
 extern "C" FGR_API fgr_status fgr_set_pattern(fgr_grid* g, int32_t hybrid_t1, int32_t hybrid_t2) {
     if (!g) return fgr_set_error(FGR_ERR_INVALID, "grid is NULL");
     if (hybrid_t1 <= hybrid_t2 && (hybrid_t1 < 0 || hybrid_t2 > 2 * 32767))
@@ -143,6 +158,9 @@ extern "C" FGR_API fgr_status fgr_set_pattern(fgr_grid* g, int32_t hybrid_t1, in
     g->hy.cached = false;
     return FGR_OK;
 }
+
+static fgr_status hld_prep_list(fgr_grid* g, const fgr_nets* nets, const int32_t* list, int nl, int maxm, cudaStream_t st,
+                                HldPrep* out);
 
 extern "C" FGR_API fgr_status fgr_route_batch(fgr_grid* g, const fgr_nets* nets, const int32_t* net_ids, int32_t count,
                                               uint32_t* seg_out, uint32_t* net_cost, void* stream) {
@@ -174,10 +192,16 @@ extern "C" FGR_API fgr_status fgr_route_batch_ex(fgr_grid* g, const fgr_nets* ne
     g->hy.cached = false;   // the hybrid tables below cover this batch only
     fgr_status s = fgr_hyb_prepare(g, st, nv, nets->num_nets, nets->num_nodes, list, count, nullptr, 1, zmid_out);
     if (s != FGR_OK) return s;
+    Prep bp{};
+    if (hc[0] > 0 && (hc[4] > fgr_large_limit(g) || g->dp_policy == FGR_DP_HLD)) {
+        g->cache.prep_valid = false;   // s_hldp now holds this batch's decomposition
+        s = hld_prep_list(g, nets, list, hc[0], hc[4], st, &bp.hld);
+        if (s != FGR_OK) return s;
+    }
     FGR_CHECK_CUDA(g, refresh_before_dp(g, st, g->total_segs));
     FGR_CHECK_CUDA(g, fgr_launch_hyb_tm(g, st, nv, 0, g->hy.nslots));
     FGR_CHECK_CUDA(g, fgr_launch_dp(g, st, nv, list, hc[0], hc[1], hc[2], hc[3], hc[4], seg_out, net_cost, nullptr,
-                                    nullptr, nullptr, 0, true, nullptr));
+                                    nullptr, nullptr, 0, true, &bp));
     FGR_CHECK_CUDA(g, fgr_launch_hyb_zmid(g, st, seg_out, zmid_out));
     return FGR_OK;
 }
@@ -192,7 +216,7 @@ static fgr_status batch_info(fgr_grid* g, const fgr_nets* nets, const int32_t* o
     cudaError_t e;
     const int R = 0;   // net count of the batches is read back below
     (void)R;
-    void* p = fgr_scratch(g->s_rec[1], (size_t)B * 40 + 64, &e);
+    void* p = fgr_scratch(g->s_rec[1], (size_t)B * 44 + 64, &e);
     if (e != cudaSuccess) return fgr_cuda_fail(g, e, "batch info scratch");
     unsigned long long* d_segb = (unsigned long long*)p;
     int* d_nl = (int*)(d_segb + B);
@@ -200,12 +224,12 @@ static fgr_status batch_info(fgr_grid* g, const fgr_nets* nets, const int32_t* o
     int* d_n2 = d_mm + B;
     int* d_n9 = d_n2 + B;
     int* d_ls = d_n9 + B;
-    FGR_CHECK_CUDA(g, cudaMemsetAsync(p, 0, (size_t)B * 40, st));
+    FGR_CHECK_CUDA(g, cudaMemsetAsync(p, 0, (size_t)B * 44, st));
     if (c.cap < B + 1) {
         free(c.h_off); free(c.h_nlarge); free(c.h_maxm); free(c.h_segb); free(c.h_ntwo); free(c.h_n9);
         free(c.h_lsplit);
         c.cap = B + 1;
-        c.h_lsplit = (int*)malloc(sizeof(int) * 4 * c.cap);
+        c.h_lsplit = (int*)malloc(sizeof(int) * 5 * c.cap);
         c.h_n9 = (int*)malloc(sizeof(int) * c.cap);
         c.h_off = (int*)malloc(sizeof(int) * c.cap);
         c.h_nlarge = (int*)malloc(sizeof(int) * c.cap);
@@ -224,7 +248,7 @@ static fgr_status batch_info(fgr_grid* g, const fgr_nets* nets, const int32_t* o
     if (e != cudaSuccess) return fgr_cuda_fail(g, e, "exec order");
     if (B > 0) {
         k_batch_info<<<B, 256, 0, st>>>(B, batch_offset, order, nets->node_offset, nets->x, nets->y, nets->parent,
-                                        d_nl, d_mm, d_segb, d_n2, d_n9, keys, d_ls);
+                                        d_nl, d_mm, d_segb, d_n2, d_n9, keys, d_ls, fgr_large_limit(g));
         FGR_CHECK_CUDA(g, cudaGetLastError());
         int bits = 42;
         while ((1LL << (bits - 42)) <= B) bits++;
@@ -240,7 +264,7 @@ static fgr_status batch_info(fgr_grid* g, const fgr_nets* nets, const int32_t* o
         FGR_CHECK_CUDA(g, cudaMemcpyAsync(c.h_segb, d_segb, sizeof(long long) * B, cudaMemcpyDeviceToHost, st));
         FGR_CHECK_CUDA(g, cudaMemcpyAsync(c.h_ntwo, d_n2, sizeof(int) * B, cudaMemcpyDeviceToHost, st));
         FGR_CHECK_CUDA(g, cudaMemcpyAsync(c.h_n9, d_n9, sizeof(int) * B, cudaMemcpyDeviceToHost, st));
-        FGR_CHECK_CUDA(g, cudaMemcpyAsync(c.h_lsplit, d_ls, sizeof(int) * 4 * B, cudaMemcpyDeviceToHost, st));
+        FGR_CHECK_CUDA(g, cudaMemcpyAsync(c.h_lsplit, d_ls, sizeof(int) * 5 * B, cudaMemcpyDeviceToHost, st));
     }
     FGR_CHECK_CUDA(g, cudaStreamSynchronize(st));
     c.valid = true;
@@ -255,29 +279,65 @@ static fgr_status batch_info(fgr_grid* g, const fgr_nets* nets, const int32_t* o
 }
 
 // Large-net tree analysis once per stage (k_large_prep), reused by every batch's k_dp_large.
+// Heavy-path decomposition of a list of large nets (k_hld_prep) into g->s_hldp.
+static fgr_status hld_prep_list(fgr_grid* g, const fgr_nets* nets, const int32_t* list, int nl, int maxm, cudaStream_t st,
+                                HldPrep* out) {
+    const size_t M = (size_t)nets->num_nodes, N = (size_t)nets->num_nets;
+    cudaError_t e;
+    char* p = (char*)fgr_scratch(g->s_hldp, 5 * a16h(2 * M) + 2 * a16h(M) + a16h(4 * N) + 64, &e);
+    if (e != cudaSuccess) return fgr_cuda_fail(g, e, "hld prep arrays");
+    auto take = [&](size_t b) { char* q = p; p += a16h(b); return q; };
+    uint16_t* hv = (uint16_t*)take(2 * M); uint16_t* cs = (uint16_t*)take(2 * M); uint16_t* cl = (uint16_t*)take(2 * M);
+    uint16_t* pn = (uint16_t*)take(2 * M); uint16_t* po = (uint16_t*)take(2 * M);
+    uint8_t* pr = (uint8_t*)take(M);
+    int32_t* info = (int32_t*)take(4 * N);
+    uint8_t* ld = (uint8_t*)take(M);
+    FGR_CHECK_CUDA(g, fgr_launch_hld_prep(g, st, fgr_nets_view(nets), list, nl, maxm, hv, cs, cl, pn, po, pr, info, ld));
+    *out = HldPrep{hv, cs, cl, pn, po, pr, info, ld};
+    return FGR_OK;
+}
+
+// Large-net tree analyses once per stage, reused by every batch's large-net DP launches: the
+// heavy-path tables of k_dp_flow / k_dp_large (k_large_prep) for the nets they route, and the
+// decomposition of k_dp_hld (k_hld_prep) for the nets it routes (fgr_set_dp_policy).
 static fgr_status ensure_prep(fgr_grid* g, const fgr_nets* nets, int B, cudaStream_t st) {
     PlanCache& c = g->cache;
     if (c.prep_valid) return FGR_OK;
     const int R = B > 0 ? c.h_off[B] : 0;
-    int maxm = 0, nl = 0;
-    for (int b = 0; b < B; b++) { maxm = c.h_maxm[b] > maxm ? c.h_maxm[b] : maxm; nl += c.h_nlarge[b]; }
-    if (nl == 0) { c.prep = Prep{nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr}; c.prep_valid = true; return FGR_OK; }
+    const int lim = fgr_large_limit(g);
+    int maxm = 0, nl = 0, nh = 0;
+    for (int b = 0; b < B; b++) {
+        maxm = c.h_maxm[b] > maxm ? c.h_maxm[b] : maxm;
+        nl += c.h_nlarge[b];
+        nh += c.h_lsplit[5 * b];
+    }
+    const bool all_hld = g->dp_policy == FGR_DP_HLD;
+    if (all_hld) nh = nl;
+    c.prep = Prep{};
+    if (nl == 0) { c.prep_valid = true; return FGR_OK; }
     const size_t M = (size_t)nets->num_nodes, N = (size_t)nets->num_nets;
     cudaError_t e;
-    char* p = (char*)fgr_scratch(g->s_prep, 6 * 2 * M + 4 * N + 4 * (size_t)nl + 64 + 6 * 16, &e);
+    char* p = (char*)fgr_scratch(g->s_prep, 6 * 2 * M + 4 * N + 8 * (size_t)R + 64 + 6 * 16, &e);
     if (e != cudaSuccess) return fgr_cuda_fail(g, e, "prep arrays");
     auto take16 = [&](size_t n) { uint16_t* q = (uint16_t*)p; p += (2 * n + 15) & ~(size_t)15; return q; };
     uint16_t* cs = take16(M); uint16_t* cl = take16(M); uint16_t* hv = take16(M); uint16_t* bot = take16(M);
     uint16_t* pq = take16(M);
     uint16_t* rpos = take16(M);
     int32_t* np = (int32_t*)p; p += (4 * N + 15) & ~(size_t)15;
-    int32_t* list = (int32_t*)p; p += 4 * (size_t)nl;
+    int32_t* list = (int32_t*)p; p += 8 * (size_t)R;   // [R] nets of k_large_prep | [R] nets of k_hld_prep
     int* cnt = (int*)p;
-    FGR_CHECK_CUDA(g, cudaMemsetAsync(cnt, 0, sizeof(int), st));
-    k_large_list<<<(R + 255) / 256, 256, 0, st>>>(R, c.exec, nets->node_offset, list, cnt);
+    FGR_CHECK_CUDA(g, cudaMemsetAsync(cnt, 0, 2 * sizeof(int), st));
+    k_large_list<<<(R + 255) / 256, 256, 0, st>>>(R, c.exec, nets->node_offset, list, cnt, all_hld ? FGR_SMALL_NET : lim);
     FGR_CHECK_CUDA(g, cudaGetLastError());
-    FGR_CHECK_CUDA(g, fgr_launch_large_prep(g, st, fgr_nets_view(nets), list, nl, maxm, cs, cl, hv, bot, pq, rpos, np));
-    c.prep = Prep{cs, cl, hv, bot, pq, np, rpos};
+    if (!all_hld && nl > nh) {
+        FGR_CHECK_CUDA(g, fgr_launch_large_prep(g, st, fgr_nets_view(nets), list, nl - nh, min(maxm, lim), cs, cl, hv, bot,
+                                                pq, rpos, np));
+        c.prep = Prep{cs, cl, hv, bot, pq, np, rpos, HldPrep{}};
+    }
+    if (nh > 0) {
+        fgr_status s = hld_prep_list(g, nets, list + R, nh, maxm, st, &c.prep.hld);
+        if (s != FGR_OK) return s;
+    }
     c.prep_valid = true;
     return FGR_OK;
 }
@@ -341,7 +401,7 @@ extern "C" FGR_API fgr_status fgr_route_all_ex(fgr_grid* g, const fgr_nets* nets
             const int o0 = c.h_off[b], cnt = c.h_off[b + 1] - o0, nl = c.h_nlarge[b], n2 = c.h_ntwo[b], n9 = c.h_n9[b];
             FGR_CHECK_CUDA(g, fgr_launch_dp(g, st, nv, c.exec + o0, nl, n9, cnt - nl - n9 - n2, n2, c.h_maxm[b],
                                             seg_out, net_cost, nullptr, nullptr, nullptr, 0, true, &c.prep,
-                                            c.h_lsplit + 4 * b));
+                                            c.h_lsplit + 5 * b));
         }
         FGR_CHECK_CUDA(g, fgr_launch_hyb_zmid(g, st, seg_out, zmid_out));
         return FGR_OK;

@@ -19,6 +19,7 @@ LIB_PATH = os.environ.get("FGR_LIB_PATH") or os.path.join(_HERE, "libfastgr.so")
 _LIB = None
 
 FGR_OK, FGR_ERR_INVALID, FGR_ERR_RANGE, FGR_ERR_OOM, FGR_ERR_CUDA, FGR_ERR_NCCL, FGR_ERR_STATE = range(7)
+FGR_DP_AUTO, FGR_DP_HEAVY, FGR_DP_HLD = 0, 1, 2   # large-net DP kernel selection (fgr_set_dp_policy)
 STATUS_NAMES = ["OK", "INVALID", "RANGE", "OOM", "CUDA", "NCCL", "STATE"]
 
 # every entry point include/fastgr.h declares
@@ -26,7 +27,7 @@ EXPORTS = ["fgr_last_error", "fgr_version", "fgr_cost_table", "fgr_grid_create",
            "fgr_grid_set_demand", "fgr_grid_get_demand", "fgr_plan", "fgr_route_batch", "fgr_route_all",
            "fgr_comm_unique_id", "fgr_comm_init", "fgr_run_host", "fgr_get_stats", "fgr_profile_enable",
            "fgr_profile_read", "fgr_split_batch", "fgr_set_pattern", "fgr_route_batch_ex", "fgr_route_all_ex",
-           "fgr_run_host_ex", "fgr_overflow", "fgr_task_graph"]
+           "fgr_run_host_ex", "fgr_overflow", "fgr_task_graph", "fgr_set_dp_policy"]
 PROF_CLASSES = ["refresh", "dp_small", "dp_large", "commit", "plan_preprocess", "plan_sort", "plan_color",
                 "plan_other", "exchange", "hybrid"]
 # the paper's FastGRH selection window: hybrid L+Z on two-pin HPWL in [100, 500]
@@ -86,6 +87,7 @@ def lib():
             "fgr_profile_read": ([P, P, P], S),
             "fgr_split_batch": ([I, I, I, I, P], S),
             "fgr_set_pattern": ([P, I, I], S),
+            "fgr_set_dp_policy": ([P, I, I], S),
             "fgr_route_batch_ex": ([P, P, P, I, P, P, P, P], S),
             "fgr_route_all_ex": ([P, P, P, P, I, P, P, P, P], S),
             "fgr_run_host_ex": ([P, I, I, P, P, P, P, P, P, P, P, P, P, P], S),
@@ -186,6 +188,10 @@ def fgr_set_pattern(h, hybrid_t1, hybrid_t2):
     _check(lib().fgr_set_pattern(h, int(hybrid_t1), int(hybrid_t2)))
 
 
+def fgr_set_dp_policy(h, policy, flow_max=64):
+    _check(lib().fgr_set_dp_policy(h, int(policy), int(flow_max)))
+
+
 def fgr_route_batch_ex(h, nets, net_ids, count, seg_out, zmid_out, net_cost, stream=None):
     _check(lib().fgr_route_batch_ex(h, ctypes.byref(nets), _ptr(net_ids), int(count), _ptr(seg_out), _ptr(zmid_out),
                                     _ptr(net_cost), _stream(stream)))
@@ -273,7 +279,7 @@ def fgr_profile_read(h) -> dict:
 class Router:
     """Owns a grid handle plus device copies of one design's nets (torch tensors)."""
 
-    def __init__(self, design, device: int = 0, stream=None, hybrid=None):
+    def __init__(self, design, device: int = 0, stream=None, hybrid=None, dp_policy=None):
         import torch
         if not torch.cuda.is_available():
             raise RuntimeError("fastgr needs a CUDA device (no CPU fallback)")
@@ -291,6 +297,8 @@ class Router:
         self.hybrid = hybrid
         if hybrid is not None:
             fgr_set_pattern(self.h, hybrid[0], hybrid[1])
+        if dp_policy is not None:   # (policy, flow_max)
+            fgr_set_dp_policy(self.h, dp_policy[0], dp_policy[1])
         self._ecap = ecap
         t = lambda a: torch.from_numpy(np.ascontiguousarray(a)).to(self.dev)
         self.t_off, self.t_x, self.t_y = t(design.node_offset), t(design.x), t(design.y)

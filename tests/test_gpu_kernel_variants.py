@@ -1,86 +1,90 @@
-"""GPU parity of every DP kernel selection: the environment switches
-FGR_FLOW_MAX (largest net of the dataflow kernel), FGR_LARGE_KERNEL=old and
-FGR_GROUP_KERNEL=old are read once per process, so each selection runs in its own
-subprocess and is checked element by element against the oracle, through fgr_route_all
-(with the once-per-stage tree analysis) and fgr_route_batch (without it).
+"""GPU parity of every large-net DP kernel selection (fgr_set_dp_policy, include/fastgr.h;
+DESIGN.md §5): the tree-dataflow kernel (k_dp_flow) up to flow_max nodes, the heavy-path
+kernel (k_dp_large) up to its shared-memory limit, the heavy-path contraction kernel
+(k_dp_hld) above it or for every net.  Each selection is checked element by element against
+the oracle through fgr_route_all (with the once-per-stage tree analyses) and fgr_route_batch
+(without them).
 
-The "chains" design has large nets with long root paths (>= 64 nodes), so under
-FGR_FLOW_MAX=100000 the flow kernel's root-path walker (transfer matrices built by the
-worker groups, walker-inline fallback, kicks) is exercised.
+The "chains" design has large nets with long root paths (>= 64 nodes, the flow kernel's
+root-path walker); "huge" has nets of 1.5k-4.4k nodes, above the shared-memory kernels' limit.
 """
-import os
-import subprocess
 import sys
 
+import numpy as np
 import pytest
+
+import gen
+from oracle import Oracle
+from paper_conf_date_liulzclly22_b200 import fastgr as F
 
 pytestmark = pytest.mark.gpu
 
-ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-
-SCRIPT = r"""
-import sys, numpy as np, torch
-sys.path.insert(0, ".")
-import gen
-from oracle import Oracle
-from tests.test_gpu_parity import check_against_oracle, first_diff, _router
-
-designs = {
+DESIGNS = {
     "t5": lambda: gen.make_config("t5", num_nets=20000),
     "bignets": lambda: gen.generate(nx=120, ny=110, nlayers=9, num_nets=400, seed=77, caps=gen.CAP9, pin_dist=1,
                                     kmin=30, kmax=400, hpwl_base=20.0, hpwl_sigma=0.5, name="bignets"),
     "chains": lambda: gen.generate(nx=160, ny=150, nlayers=9, num_nets=120, seed=91, caps=gen.CAP9, pin_dist=1,
                                    kmin=300, kmax=900, hpwl_base=60.0, hpwl_sigma=0.3, name="chains"),
+    "huge": lambda: gen.generate(nx=300, ny=300, nlayers=9, num_nets=12, seed=5, caps=gen.CAP9, pin_dist=1,
+                                 kmin=1400, kmax=5000, hpwl_base=160.0, hpwl_sigma=0.2, name="huge"),
 }
-for name in sys.argv[1].split(","):
-    d = designs[name]()
-    check_against_oracle(d)
-    # fgr_route_batch: no tree analysis (the kernels build their child CSR themselves)
-    o = Oracle(d)
-    ob, onb = o.plan()
-    oseg, ocost, odem = o.route(ob, onb)
-    r = _router(d)
+
+POLICIES = {
+    "auto": (F.FGR_DP_AUTO, 64),
+    "flow_all": (F.FGR_DP_AUTO, 65535),
+    "flow_40": (F.FGR_DP_AUTO, 40),
+    "heavy": (F.FGR_DP_HEAVY, 64),
+    "hld": (F.FGR_DP_HLD, 64),
+}
+
+_cache = {}
+
+
+def _oracle(name):
+    if name not in _cache:
+        d = DESIGNS[name]()
+        o = Oracle(d)
+        ob, onb = o.plan()
+        _cache[name] = (d, ob, onb) + tuple(o.route(ob, onb))
+    return _cache[name]
+
+
+def first_diff(a, b):
+    idx = np.nonzero(a != b)[0]
+    return None if len(idx) == 0 else (int(idx[0]), a[idx[0]], b[idx[0]], len(idx))
+
+
+@pytest.mark.parametrize("policy", sorted(POLICIES))
+@pytest.mark.parametrize("design", sorted(DESIGNS))
+def test_kernel_selection_bit_exact(policy, design):
+    import torch
+    d, ob, onb, oseg, ocost, odem = _oracle(design)
+    r = F.Router(d, device=0, dp_policy=POLICIES[policy])
+    r.reset_demand(None)
+    nb = r.plan()
+    r.route_all()
+    b, nb, seg, cost, dem = r.results()
+    assert nb == onb
+    assert np.array_equal(seg, oseg), first_diff(seg, oseg)
+    assert np.array_equal(cost, ocost), first_diff(cost, ocost)
+    assert np.array_equal(dem, odem)
+    # fgr_route_batch: no once-per-stage analyses (the kernels build their tables themselves)
     r.reset_demand(None)
     r.seg.fill_(-1)
     r.cost.zero_()
-    for b in range(onb):
-        r.route_batch(torch.from_numpy(np.nonzero(ob == b)[0].astype(np.int32)).cuda())
+    for bb in range(onb):
+        r.route_batch(torch.from_numpy(np.nonzero(ob == bb)[0].astype(np.int32)).cuda())
     torch.cuda.synchronize()
     seg = r.seg.cpu().numpy().view(np.uint32)
-    assert np.array_equal(seg, oseg), (name, first_diff(seg, oseg))
-    assert np.array_equal(r.cost.cpu().numpy().view(np.uint32), ocost), name
-    assert np.array_equal(r.demand().cpu().numpy(), odem), name
+    assert np.array_equal(seg, oseg), first_diff(seg, oseg)
+    assert np.array_equal(r.cost.cpu().numpy().view(np.uint32), ocost)
+    assert np.array_equal(r.demand().cpu().numpy(), odem)
     r.close()
-    print("ok", name, int((d.net_sizes() > 32).sum()), "large nets")
-"""
-
-VARIANTS = {
-    "flow_all": {"FGR_FLOW_MAX": "100000"},
-    "flow_40": {"FGR_FLOW_MAX": "40"},
-    "flow_128": {"FGR_FLOW_MAX": "128"},    # the previous default cut
-    "large_old": {"FGR_LARGE_KERNEL": "old"},
-    "group_old": {"FGR_GROUP_KERNEL": "old"},
-}
 
 
-@pytest.mark.parametrize("variant", sorted(VARIANTS))
-def test_kernel_selection_bit_exact(variant):
-    env = dict(os.environ)
-    env.update(VARIANTS[variant])
-    designs = "t5,bignets,chains"
-    p = subprocess.run([sys.executable, "-c", SCRIPT, designs], cwd=ROOT, env=env, capture_output=True, text=True,
-                       timeout=900)
-    assert p.returncode == 0, p.stdout[-3000:] + p.stderr[-3000:]
-    assert p.stdout.count("ok ") == 3, p.stdout
-
-
-def test_chains_design_has_long_root_paths():
-    """The chains design must reach the walker (root path >= 64 nodes)."""
-    import numpy as np
-    sys.path.insert(0, ROOT)
-    import gen
-    d = gen.generate(nx=160, ny=150, nlayers=9, num_nets=120, seed=91, caps=gen.CAP9, pin_dist=1, kmin=300, kmax=900,
-                     hpwl_base=60.0, hpwl_sigma=0.3, name="chains")
+def test_designs_reach_the_intended_kernels():
+    """chains: root paths >= 64 nodes (flow kernel's walker); huge: nets above the 1.3k-node shared-memory limit."""
+    d = DESIGNS["chains"]()
     sizes = d.net_sizes()
     deepest = 0
     for n in np.nonzero(sizes > 128)[0][:20]:
@@ -91,3 +95,17 @@ def test_chains_design_has_long_root_paths():
             depth[i] = depth[par[i]] + 1
         deepest = max(deepest, int(depth.max()))
     assert deepest >= 64, deepest
+    assert (DESIGNS["huge"]().net_sizes() > 1400).sum() >= 10
+
+
+def test_dp_policy_validation():
+    d = gen.make_config("tiny", num_nets=5)
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("needs a GPU")
+    r = F.Router(d, device=0)
+    with pytest.raises(F.FgrError):
+        F.fgr_set_dp_policy(r.h, 7, 64)
+    with pytest.raises(F.FgrError):
+        F.fgr_set_dp_policy(r.h, F.FGR_DP_AUTO, 8)
+    r.close()

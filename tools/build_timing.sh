@@ -1,14 +1,12 @@
 #!/bin/bash
-# Debug build with in-kernel phase timers (-DFGR_TIMING) into tbuild/libfastgr.so (use FGR_LIB_PATH=...).
+# Build build_t/libfastgr_t.so: the library with FGR_HLD_TIMING per-phase clock64 prints in k_dp_hld
+# (use with FGR_LIB_PATH=build_t/libfastgr_t.so).  Reuses the other objects of build/.
 set -e
 cd "$(dirname "$0")/.."
-NI=$(python -c "import nvidia.nccl,os;print(os.path.dirname(nvidia.nccl.__path__[0]))")/nccl
-mkdir -p tbuild
-for f in paper_conf_date_liulzclly22_b200/csrc/*.cu; do
-  b=$(basename $f .cu)
-  /usr/local/cuda/bin/nvcc -DFGR_TIMING -O3 -std=c++17 -gencode arch=compute_100a,code=sm_100a -lineinfo \
-    -Xcompiler -fPIC -Xcompiler -fvisibility=hidden -Iinclude -I$NI/include --expt-relaxed-constexpr -c -o tbuild/$b.o $f &
-done
-wait
-/usr/local/cuda/bin/nvcc -gencode arch=compute_100a,code=sm_100a -shared -o tbuild/libfastgr.so tbuild/*.o \
-  -L$NI/lib -l:libnccl.so.2 -Xlinker -rpath=$NI/lib
+SITE=$(python -c "import nvidia.nccl,os;print(os.path.dirname(nvidia.nccl.__path__[0]))")
+mkdir -p build_t
+/usr/local/cuda/bin/nvcc -DFGR_HLD_TIMING -O3 -std=c++17 -gencode arch=compute_100a,code=sm_100a -lineinfo -Xcompiler -fPIC \
+  -Xcompiler -fvisibility=hidden -Iinclude -I$SITE/nccl/include --expt-relaxed-constexpr -c -o build_t/dp_hld.o \
+  paper_conf_date_liulzclly22_b200/csrc/dp_hld.cu
+/usr/local/cuda/bin/nvcc -gencode arch=compute_100a,code=sm_100a -shared -o build_t/libfastgr_t.so \
+  $(ls build/*.o | grep -v dp_hld) build_t/dp_hld.o -L$SITE/nccl/lib -l:libnccl.so.2 -Xlinker -rpath=$SITE/nccl/lib -Xcompiler -fPIC
