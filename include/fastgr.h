@@ -198,11 +198,17 @@ FGR_API fgr_status fgr_route_batch_ex(fgr_grid* grid, const fgr_nets* nets, cons
  * order/batch_offset/num_batches as returned by fgr_plan for the same nets.
  * seg_out [num_nodes] and net_cost [num_nets] are fully written (trivial nets:
  * seg 0xFFFFFFFF, cost 0).  With a communicator (fgr_comm_init, world > 1),
- * each batch's nets are split across ranks (fgr_split_batch) and the routes are
- * exchanged with one NCCL all-reduce per batch; every rank ends with identical
- * outputs and demand, bitwise equal to world = 1.  (A communicator of world 1
- * takes the same exchange path, which is how it is tested on one GPU.)  No host synchronisation when the
- * arguments are those of the grid's last fgr_plan call.
+ * each batch of at least split_min nets is split across ranks by tree edges
+ * (fgr_split_batch) and the routes are exchanged with one NCCL all-reduce per
+ * batch; smaller batches are routed whole on every rank (fgr_set_exchange).  Every
+ * rank ends with identical outputs and demand, bitwise equal to world = 1.  (A
+ * communicator of world 1 takes the same exchange path; fgr_set_exchange's
+ * emulate_world runs it with k emulated ranks on one GPU.)  The exchange path
+ * synchronises the stream once per call (record offsets and the edge split);
+ * without it there is no host synchronisation when the arguments are those of
+ * the grid's last fgr_plan call.  The plan cache is keyed on the identity of the
+ * `nets` device pointers and order/batch_offset: after rewriting those buffers in
+ * place, call fgr_plan again.
  */
 FGR_API fgr_status fgr_route_all(fgr_grid* grid, const fgr_nets* nets, const int32_t* order,
                                  const int32_t* batch_offset, int32_t num_batches, uint32_t* seg_out,
@@ -215,11 +221,34 @@ FGR_API fgr_status fgr_route_all_ex(fgr_grid* grid, const fgr_nets* nets, const 
                                     const int32_t* batch_offset, int32_t num_batches, uint32_t* seg_out,
                                     int32_t* zmid_out, uint32_t* net_cost, void* stream);
 
-/* The multi-GPU split rule fgr_route_all applies to one batch (host-only, no GPU):
- * the batch's `count` nets are ordered large nets first (`nlarge` of them); rank r
- * of `world` routes the large nets [out[0], out[1]) and the small nets
- * [out[2], out[3]) (indices into the batch).  Contiguous, disjoint, covering. */
-FGR_API fgr_status fgr_split_batch(int32_t count, int32_t nlarge, int32_t rank, int32_t world, int32_t* out4);
+/*
+ * fgr_split_batch — the multi-GPU split rule fgr_route_all applies to one batch
+ * (host-only, no GPU).  The batch's `count` nets are in exec
+ * order, large nets first (`nlarge` of them).  edge_prefix [count+1] HOST in (may
+ * be NULL): edge_prefix[i] = tree edges of the batch's first i nets.  Rank r of
+ * `world` routes the large nets [out[0], out[1]) and the small nets [out[2],
+ * out[3]) (indices into the batch): contiguous, disjoint and covering, balanced by
+ * tree edges (by net count when edge_prefix is NULL).  A batch of fewer than
+ * split_min nets is not split: out = {0, nlarge, nlarge, count} on every rank and
+ * out[4] = 1 (every rank routes it whole and no exchange is needed); else out[4] = 0.
+ * out5 [5] HOST out.  Errors: INVALID.
+ */
+FGR_API fgr_status fgr_split_batch(int32_t count, int32_t nlarge, const int64_t* edge_prefix, int32_t split_min,
+                                   int32_t rank, int32_t world, int32_t* out5);
+
+/*
+ * fgr_set_exchange — multi-GPU exchange settings of later fgr_route_all(_ex) calls.
+ *   split_min (default 2048): batches of fewer nets are routed whole on every
+ *       rank instead of split + all-reduced (a batch's latency is its biggest
+ *       net; a collective per small batch only adds latency).  0 = split every batch.
+ *   emulate_world: 0 or 1 = off; k > 1 = TEST MODE on a grid without a
+ *       communicator: fgr_route_all takes the exchange path with k emulated ranks on
+ *       this device (every rank's chunk routed into the shared route records, which
+ *       then hold what the NCCL SUM all-reduce would; then the commit from the
+ *       records), so the split, record and commit code runs on one GPU.
+ * Host-only; takes effect at the next route call.  Errors: INVALID.
+ */
+FGR_API fgr_status fgr_set_exchange(fgr_grid* grid, int32_t split_min, int32_t emulate_world);
 
 /* Multi-GPU (one process per GPU).  fgr_comm_unique_id fills 128 bytes on the
  * root rank; broadcast them (e.g. torch.distributed) and call fgr_comm_init on
@@ -289,6 +318,7 @@ typedef struct {
     int64_t dp_nets, dp_edges;         /* nets and tree edges routed                            */
     int64_t kernel_launches;           /* kernels launched by the library                       */
     int32_t num_batches, world, rank;
+    int32_t exchanged_batches;         /* multi-GPU: batches split across ranks (others routed whole) */
 } fgr_stats;
 FGR_API fgr_status fgr_get_stats(fgr_grid* grid, fgr_stats* out);
 

@@ -213,6 +213,10 @@ struct fgr_grid {
     // large-net DP kernel selection (fgr_set_dp_policy)
     int dp_policy = FGR_DP_AUTO;
     int flow_max = 64;
+    // multi-GPU exchange (fgr_set_exchange): batches below split_min nets are routed whole on every
+    // rank; emu_world > 1 runs the exchange path with that many emulated ranks on one device
+    int split_min = 2048;
+    int emu_world = 0;
     HybState hy;
     Scratch s_hyb[3];
     Scratch s_rip[6];          // rip-up extraction and task graph (ripup.cu)

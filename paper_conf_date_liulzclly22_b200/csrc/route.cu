@@ -127,14 +127,48 @@ static cudaError_t refresh_before_dp(fgr_grid* g, cudaStream_t st, long long max
     return fgr_launch_refresh_sized(g, st, false, max_tasks);
 }
 
-extern "C" FGR_API fgr_status fgr_split_batch(int32_t count, int32_t nlarge, int32_t rank, int32_t world, int32_t* out) {
+// first index i in [lo, hi] with pre[i] - pre[lo] >= target (pre non-decreasing)
+static int32_t split_point(const int64_t* pre, int32_t lo, int32_t hi, int64_t target) {
+    int32_t a = lo, b = hi;
+    while (a < b) {
+        const int32_t mid = a + (b - a) / 2;
+        if (pre[mid] - pre[lo] >= target) b = mid; else a = mid + 1;
+    }
+    return a;
+}
+
+extern "C" FGR_API fgr_status fgr_split_batch(int32_t count, int32_t nlarge, const int64_t* edge_prefix, int32_t split_min,
+                                              int32_t rank, int32_t world, int32_t* out) {
     if (!out || count < 0 || nlarge < 0 || nlarge > count || world < 1 || rank < 0 || rank >= world)
         return fgr_set_error(FGR_ERR_INVALID, "bad split arguments");
-    const long long ns = count - nlarge;
-    out[0] = (int32_t)((long long)nlarge * rank / world);
-    out[1] = (int32_t)((long long)nlarge * (rank + 1) / world);
-    out[2] = nlarge + (int32_t)(ns * rank / world);
-    out[3] = nlarge + (int32_t)(ns * (rank + 1) / world);
+    if (count < split_min) {   // too small to pay an exchange: every rank routes the whole batch
+        out[0] = 0; out[1] = nlarge; out[2] = nlarge; out[3] = count; out[4] = 1;
+        return FGR_OK;
+    }
+    out[4] = 0;
+    if (!edge_prefix) {
+        const long long ns = count - nlarge;
+        out[0] = (int32_t)((long long)nlarge * rank / world);
+        out[1] = (int32_t)((long long)nlarge * (rank + 1) / world);
+        out[2] = nlarge + (int32_t)(ns * rank / world);
+        out[3] = nlarge + (int32_t)(ns * (rank + 1) / world);
+        return FGR_OK;
+    }
+    // balanced by tree edges: contiguous chunks of the large and of the small nets
+    const int64_t el = edge_prefix[nlarge] - edge_prefix[0], es = edge_prefix[count] - edge_prefix[nlarge];
+    out[0] = rank == 0 ? 0 : split_point(edge_prefix, 0, nlarge, (el * rank + world - 1) / world);
+    out[1] = rank == world - 1 ? nlarge : split_point(edge_prefix, 0, nlarge, (el * (rank + 1) + world - 1) / world);
+    out[2] = rank == 0 ? nlarge : split_point(edge_prefix, nlarge, count, (es * rank + world - 1) / world);
+    out[3] = rank == world - 1 ? count : split_point(edge_prefix, nlarge, count, (es * (rank + 1) + world - 1) / world);
+    return FGR_OK;
+}
+
+extern "C" FGR_API fgr_status fgr_set_exchange(fgr_grid* g, int32_t split_min, int32_t emulate_world) {
+    if (!g) return fgr_set_error(FGR_ERR_INVALID, "grid is NULL");
+    if (split_min < 0 || emulate_world < 0 || emulate_world > 1024)
+        return fgr_set_error(FGR_ERR_INVALID, "bad exchange settings %d / %d", split_min, emulate_world);
+    g->split_min = split_min;
+    g->emu_world = emulate_world;
     return FGR_OK;
 }
 
@@ -391,9 +425,12 @@ extern "C" FGR_API fgr_status fgr_route_all_ex(fgr_grid* g, const fgr_nets* nets
     g->stats.world = g->world;
     g->stats.rank = g->rank;
     g->stats.dp_nets = B > 0 ? c.h_off[B] : 0;
+    g->stats.dp_edges = (int64_t)M - N;   // every net is a tree: sum of (nodes - 1)
+    g->stats.exchanged_batches = 0;
     g->stats.kernel_launches = 0;
     FGR_CHECK_CUDA(g, cudaMemsetAsync(g->d_stats, 0, 4 * sizeof(unsigned long long), st));
-    if (!g->comm) {
+    const bool emu = !g->comm && g->emu_world > 1;
+    if (!g->comm && !emu) {
         for (int b = 0; b < B; b++) {
             const long long bound = b > 0 ? c.h_segb[b - 1] : (long long)g->total_segs;
             FGR_CHECK_CUDA(g, refresh_before_dp(g, st, bound));
@@ -406,7 +443,11 @@ extern "C" FGR_API fgr_status fgr_route_all_ex(fgr_grid* g, const fgr_nets* nets
         FGR_CHECK_CUDA(g, fgr_launch_hyb_zmid(g, st, seg_out, zmid_out));
         return FGR_OK;
     }
-    // ---- multi-GPU: split each batch, exchange route records, commit everywhere
+    // ---- multi-GPU: split each batch by tree edges, exchange route records, commit everywhere.
+    // Batches with fewer than split_min nets are routed whole on every rank (no exchange: the
+    // routes are deterministic).  emu: all `world` ranks' chunks run on this device into the
+    // shared records, which then hold what the NCCL SUM would (test mode, fgr_set_exchange).
+    const int W = emu ? g->emu_world : g->world;
     cudaError_t e;
     const int R = B > 0 ? c.h_off[B] : 0;
     int32_t* rec_off = (int32_t*)fgr_scratch(g->s_rec[2], sizeof(int32_t) * ((size_t)R + 1) * 2 + 64, &e);
@@ -417,63 +458,73 @@ extern "C" FGR_API fgr_status fgr_route_all_ex(fgr_grid* g, const fgr_nets* nets
         FGR_CHECK_CUDA(g, cudaGetLastError());
     }
     FGR_CHECK_CUDA(g, cudaMemsetAsync(sizes + R, 0, sizeof(int32_t), st));
+    std::vector<int32_t> h_sz((size_t)R + 1);
+    if (R > 0) FGR_CHECK_CUDA(g, cudaMemcpyAsync(h_sz.data(), sizes, sizeof(int32_t) * (size_t)R, cudaMemcpyDeviceToHost, st));
     size_t tb = 0;
     cub::DeviceScan::ExclusiveSum(nullptr, tb, sizes, rec_off, R + 1, st);
     void* tmp = fgr_scratch(g->s_plan[8], tb, &e);
     if (e != cudaSuccess) return fgr_cuda_fail(g, e, "scan scratch");
     FGR_CHECK_CUDA(g, cub::DeviceScan::ExclusiveSum(tmp, tb, sizes, rec_off, R + 1, st));
-    int* h_roff = (int*)malloc(sizeof(int) * (B + 1));
+    std::vector<int> h_roff((size_t)B + 1);
     for (int b = 0; b <= B; b++)
-        FGR_CHECK_CUDA(g, cudaMemcpyAsync(h_roff + b, rec_off + c.h_off[b], sizeof(int), cudaMemcpyDeviceToHost, st));
+        FGR_CHECK_CUDA(g, cudaMemcpyAsync(h_roff.data() + b, rec_off + c.h_off[b], sizeof(int), cudaMemcpyDeviceToHost, st));
     FGR_CHECK_CUDA(g, cudaStreamSynchronize(st));
+    std::vector<int64_t> h_epre((size_t)R + 1);   // tree-edge prefix over the exec order
+    h_epre[0] = 0;
+    for (int i = 0; i < R; i++) h_epre[(size_t)i + 1] = h_epre[i] + (h_sz[i] - 1);
     const size_t nrec = (size_t)h_roff[B];
     uint32_t* rec = (uint32_t*)fgr_scratch(g->s_rec[3], sizeof(uint32_t) * (nrec + (size_t)R + 1), &e);
-    if (e != cudaSuccess) { free(h_roff); return fgr_cuda_fail(g, e, "records"); }
+    if (e != cudaSuccess) return fgr_cuda_fail(g, e, "records");
     uint32_t* rec_cost = rec + nrec;
     FGR_CHECK_CUDA(g, cudaMemsetAsync(rec, 0, sizeof(uint32_t) * (nrec + (size_t)R + 1), st));
-    fgr_status rs = FGR_OK;
-    for (int b = 0; b < B && rs == FGR_OK; b++) {
+    g->stats.exchanged_batches = 0;
+    for (int b = 0; b < B; b++) {
         const long long bound = b > 0 ? c.h_segb[b - 1] : (long long)g->total_segs;
-        cudaError_t ce = refresh_before_dp(g, st, bound);
-        if (ce != cudaSuccess) { rs = fgr_cuda_fail(g, ce, "refresh"); break; }
+        FGR_CHECK_CUDA(g, refresh_before_dp(g, st, bound));
         // every rank builds the batch's hybrid matrices: the commit of remote routes reads their Z argmins
-        if (hy.active) ce = fgr_launch_hyb_tm(g, st, nv, hy.boff[b], hy.boff[b + 1] - hy.boff[b]);
-        if (ce != cudaSuccess) { rs = fgr_cuda_fail(g, ce, "hybrid"); break; }
+        if (hy.active) FGR_CHECK_CUDA(g, fgr_launch_hyb_tm(g, st, nv, hy.boff[b], hy.boff[b + 1] - hy.boff[b]));
         const int o0 = c.h_off[b], cnt = c.h_off[b + 1] - o0, nl = c.h_nlarge[b], n2 = c.h_ntwo[b], n9 = c.h_n9[b];
-        int32_t sp[4];
-        fgr_split_batch(cnt, nl, g->rank, g->world, sp);
-        if (sp[1] > sp[0])
-            ce = fgr_launch_dp(g, st, nv, c.exec + o0 + sp[0], sp[1] - sp[0], 0, 0, 0, c.h_maxm[b], nullptr, nullptr,
-                               rec, rec_off, rec_cost, o0 + sp[0], false, &c.prep);
-        if (ce == cudaSuccess && sp[3] > sp[2]) {
-            // the rank's small chunk [sp2, sp3) crosses the class boundaries nl+n9 and cnt-n2
-            const int b1 = nl + n9, b2 = cnt - n2;
-            const int cL = max(0, min(sp[3], b1) - sp[2]);
-            const int cS = max(0, min(sp[3], b2) - max(sp[2], b1));
-            const int cT = sp[3] - sp[2] - cL - cS;
-            ce = fgr_launch_dp(g, st, nv, c.exec + o0 + sp[2], 0, cL, cS, cT, 0, nullptr, nullptr, rec, rec_off,
-                               rec_cost, o0 + sp[2], false, &c.prep);
+        int32_t sp[5];
+        fgr_split_batch(cnt, nl, h_epre.data() + o0, g->split_min, 0, W, sp);
+        if (sp[4]) {   // routed whole on every rank, committed by the DP kernels themselves
+            FGR_CHECK_CUDA(g, fgr_launch_dp(g, st, nv, c.exec + o0, nl, n9, cnt - nl - n9 - n2, n2, c.h_maxm[b], nullptr,
+                                            nullptr, rec, rec_off, rec_cost, o0, true, &c.prep, c.h_lsplit + 5 * b));
+            continue;
         }
-        if (ce != cudaSuccess) { rs = fgr_cuda_fail(g, ce, "dp"); break; }
-        const int ps = fgr_prof_begin(g, PROF_EXCHANGE, st);
-        ncclResult_t nr = ncclGroupStart();
-        if (nr == ncclSuccess)
-            nr = ncclAllReduce(rec + h_roff[b], rec + h_roff[b], (size_t)(h_roff[b + 1] - h_roff[b]), ncclUint32,
-                               ncclSum, g->comm, st);
-        if (nr == ncclSuccess)
-            nr = ncclAllReduce(rec_cost + o0, rec_cost + o0, (size_t)cnt, ncclUint32, ncclSum, g->comm, st);
-        ncclResult_t ne = ncclGroupEnd();
-        fgr_prof_end(g, ps, st);
-        if (nr != ncclSuccess || ne != ncclSuccess) {
-            g->broken = true;
-            rs = fgr_set_error(FGR_ERR_NCCL, "NCCL all-reduce failed: %s", ncclGetErrorString(nr != ncclSuccess ? nr : ne));
-            break;
+        for (int r = emu ? 0 : g->rank; r < (emu ? W : g->rank + 1); r++) {
+            fgr_split_batch(cnt, nl, h_epre.data() + o0, g->split_min, r, W, sp);
+            if (sp[1] > sp[0])
+                FGR_CHECK_CUDA(g, fgr_launch_dp(g, st, nv, c.exec + o0 + sp[0], sp[1] - sp[0], 0, 0, 0, c.h_maxm[b], nullptr,
+                                                nullptr, rec, rec_off, rec_cost, o0 + sp[0], false, &c.prep));
+            if (sp[3] > sp[2]) {
+                // the rank's small chunk [sp2, sp3) crosses the class boundaries nl+n9 and cnt-n2
+                const int b1 = nl + n9, b2 = cnt - n2;
+                const int cL = max(0, min(sp[3], b1) - sp[2]);
+                const int cS = max(0, min(sp[3], b2) - max(sp[2], b1));
+                const int cT = sp[3] - sp[2] - cL - cS;
+                FGR_CHECK_CUDA(g, fgr_launch_dp(g, st, nv, c.exec + o0 + sp[2], 0, cL, cS, cT, 0, nullptr, nullptr, rec,
+                                                rec_off, rec_cost, o0 + sp[2], false, &c.prep));
+            }
         }
-        ce = fgr_launch_commit(g, st, nv, c.exec + o0, cnt, rec, rec_off, o0);
-        if (ce != cudaSuccess) { rs = fgr_cuda_fail(g, ce, "commit"); break; }
+        g->stats.exchanged_batches++;
+        if (!emu) {
+            const int ps = fgr_prof_begin(g, PROF_EXCHANGE, st);
+            ncclResult_t nr = ncclGroupStart();
+            if (nr == ncclSuccess)
+                nr = ncclAllReduce(rec + h_roff[b], rec + h_roff[b], (size_t)(h_roff[b + 1] - h_roff[b]), ncclUint32,
+                                   ncclSum, g->comm, st);
+            if (nr == ncclSuccess)
+                nr = ncclAllReduce(rec_cost + o0, rec_cost + o0, (size_t)cnt, ncclUint32, ncclSum, g->comm, st);
+            ncclResult_t ne = ncclGroupEnd();
+            fgr_prof_end(g, ps, st);
+            if (nr != ncclSuccess || ne != ncclSuccess) {
+                g->broken = true;
+                return fgr_set_error(FGR_ERR_NCCL, "NCCL all-reduce failed: %s",
+                                     ncclGetErrorString(nr != ncclSuccess ? nr : ne));
+            }
         }
-    free(h_roff);
-    if (rs != FGR_OK) return rs;
+        FGR_CHECK_CUDA(g, fgr_launch_commit(g, st, nv, c.exec + o0, cnt, rec, rec_off, o0));
+    }
     if (R > 0) {
         k_scatter_records<<<(unsigned)(((size_t)R * 32 + 255) / 256), 256, 0, st>>>(R, c.exec, nets->node_offset,
                                                                                      rec_off, rec, rec_cost, seg_out,
@@ -526,15 +577,16 @@ extern "C" FGR_API fgr_status fgr_run_host_ex(fgr_grid* g, int32_t N, int32_t M,
         return fgr_set_error(FGR_ERR_INVALID, "bad host arrays");
     cudaStream_t st = (cudaStream_t)stream;
     FGR_CHECK_CUDA(g, cudaSetDevice(g->device));
-    // one device slab: off | par | seg | x | y | plo | phi | cost | batch | order | boff
-    const size_t bytes = 4 * ((size_t)N + 1) + 4 * (size_t)M + 4 * (size_t)M + 2 * (size_t)M + 2 * (size_t)M + M + M +
-                         4 * (size_t)N + 4 * (size_t)N + 4 * (size_t)N + 4 * ((size_t)N + 1) + 256;
+    // one device slab: off | par | seg | zmid | batch | order | boff | cost | x | y | plo | phi
+    const size_t bytes = 4 * ((size_t)N + 1) + 4 * (size_t)M + 4 * (size_t)M + 4 * (size_t)M + 4 * (size_t)N +
+                         4 * (size_t)N + 4 * ((size_t)N + 1) + 4 * (size_t)N + 2 * (size_t)M + 2 * (size_t)M + M + M + 256;
     cudaError_t e;
     char* p = (char*)fgr_scratch(g->s_rec[0], bytes + 64, &e);
     if (e != cudaSuccess) return fgr_cuda_fail(g, e, "run_host buffers");
     int32_t* d_off = (int32_t*)p; p += 4 * ((size_t)N + 1);
     int32_t* d_par = (int32_t*)p; p += 4 * (size_t)M;
     uint32_t* d_seg = (uint32_t*)p; p += 4 * (size_t)M;
+    int32_t* d_zmid = (int32_t*)p; p += 4 * (size_t)M;
     int32_t* d_bat = (int32_t*)p; p += 4 * (size_t)N;
     int32_t* d_ord = (int32_t*)p; p += 4 * (size_t)N;
     int32_t* d_boff = (int32_t*)p; p += 4 * ((size_t)N + 1);
@@ -559,9 +611,10 @@ extern "C" FGR_API fgr_status fgr_run_host_ex(fgr_grid* g, int32_t N, int32_t M,
     int32_t B = 0;
     s = fgr_plan(g, &n, d_bat, d_ord, d_boff, &B, stream);
     if (s != FGR_OK) return s;
-    s = fgr_route_all(g, &n, d_ord, d_boff, B, d_seg, d_cost, stream);
+    s = fgr_route_all_ex(g, &n, d_ord, d_boff, B, d_seg, h_zmid ? d_zmid : nullptr, d_cost, stream);
     if (s != FGR_OK) return s;
     if (h_seg && M > 0) FGR_CHECK_CUDA(g, cudaMemcpyAsync(h_seg, d_seg, 4 * (size_t)M, cudaMemcpyDeviceToHost, st));
+    if (h_zmid && M > 0) FGR_CHECK_CUDA(g, cudaMemcpyAsync(h_zmid, d_zmid, 4 * (size_t)M, cudaMemcpyDeviceToHost, st));
     if (h_cost && N > 0) FGR_CHECK_CUDA(g, cudaMemcpyAsync(h_cost, d_cost, 4 * (size_t)N, cudaMemcpyDeviceToHost, st));
     FGR_CHECK_CUDA(g, cudaStreamSynchronize(st));
     if (h_nb) *h_nb = B;

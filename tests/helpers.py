@@ -186,19 +186,31 @@ def route_cost(d: Design, pc: PyCost, n, segs, zs=None):
     return total
 
 
-def edge_options(d: Design, n, i, hybrid=None):
+def edge_options(d: Design, n, i, hybrid=None, general_straight=False):
     """Every route of local node i's edge: [(seg, z)].  With hybrid=(t1, t2) and t1 <= HPWL <= t2
-    (bent edges only), every Z shape with both bend points strictly inside the box is added."""
+    (bent edges only), every Z shape with both bend points strictly inside the box is added.
+
+    general_straight=True (the check of reading R7): a straight edge also gets both degenerate
+    L shapes with any layer pair — one leg along the edge on a layer of its direction, a
+    zero-length leg on ANY layer at an endpoint, and the bend via between the two (so the
+    via stack at that endpoint may be paid at the "bend" instead of in the node hull)."""
     a = d.node_offset[n]
     v, u = a + i, a + int(d.parent[a + i])
     xv, yv, xu, yu = int(d.x[v]), int(d.y[v]), int(d.x[u]), int(d.y[u])
     L = d.nlayers
     H = [l for l in range(L) if d.dir[l] == 0]
     V = [l for l in range(L) if d.dir[l] == 1]
-    if yv == yu:
-        return [(make_seg(0, l, l, 1), -1) for l in H]
-    if xv == xu:
-        return [(make_seg(0, l, l, 1), -1) for l in V]
+    if yv == yu or xv == xu:
+        D = H if yv == yu else V
+        out = [(make_seg(0, l, l, 1), -1) for l in D]
+        if general_straight:
+            # bend 0 (bend point (x_u, y_v)) and bend 1 (bend point (x_v, y_u)); for a horizontal edge
+            # bend 0 = full leg 1 on ls in H then zero-length leg 2 at u on any lt, bend 1 = zero-length
+            # leg 1 at v on any ls then full leg 2 on lt in H (vertical edges: the mirror image)
+            full_first = 0 if yv == yu else 1
+            out += [(make_seg(full_first, ls, lt, 0), -1) for ls in D for lt in range(L) if lt != ls]
+            out += [(make_seg(1 - full_first, ls, lt, 0), -1) for lt in D for ls in range(L) if ls != lt]
+        return out
     out = [(make_seg(0, ls, lt, 0), -1) for ls in H for lt in V] + [(make_seg(1, ls, lt, 0), -1) for ls in V for lt in H]
     h = abs(xv - xu) + abs(yv - yu)
     if hybrid is not None and hybrid[0] <= h <= hybrid[1]:
@@ -209,11 +221,11 @@ def edge_options(d: Design, n, i, hybrid=None):
     return out
 
 
-def brute_force_min(d: Design, n, demand, hybrid=None):
+def brute_force_min(d: Design, n, demand, hybrid=None, general_straight=False):
     """Min over every per-edge route assignment of the full route cost."""
     pc = PyCost(d, demand)
     m = d.node_offset[n + 1] - d.node_offset[n]
-    opts = [edge_options(d, n, i, hybrid) for i in range(1, m)]
+    opts = [edge_options(d, n, i, hybrid, general_straight) for i in range(1, m)]
     best = None
     for combo in itertools.product(*opts):
         c = route_cost(d, pc, n, [None] + [s for s, _ in combo], [None] + [z for _, z in combo])

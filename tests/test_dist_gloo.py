@@ -1,12 +1,15 @@
 """World-size-2 CPU (gloo) tests of the multi-GPU protocol of fgr_route_all.
 
 The device path (include/fastgr.h, fgr_route_all with a communicator) does, per
-batch: split the batch with fgr_split_batch, route the rank's chunk into
-zero-padded route records, SUM-all-reduce the records, then commit every net of
-the batch from the records.  Here the same protocol runs on CPU with gloo, the
+batch: split the batch by tree edges with fgr_split_batch, route the rank's chunk
+into zero-padded route records, SUM-all-reduce the records, then commit every net
+of the batch from the records; a batch of fewer than split_min nets is routed whole
+on every rank with no exchange.  Here the same protocol runs on CPU with gloo, the
 split taken from the library's host-only fgr_split_batch and the per-net routing
 from the oracle; the result must equal the single-process oracle bit for bit
-(nets of one batch are independent: reading R13).
+(nets of one batch are independent: reading R13).  The library's own exchange path
+(split arithmetic, record offsets, partial launches, commit from records) runs on
+one GPU under fgr_set_exchange's emulated ranks: tests/test_gpu_exchange.py.
 """
 import os
 import socket
@@ -63,7 +66,18 @@ def _worker(rank, world, port, cfg, q):
                 seg[d.node_offset[n]] = 0xFFFFFFFF
         for bb, ids in enumerate(batch_order(d, b, nb)):
             nl = int((sizes[ids] > 32).sum())
-            l0, l1, s0, s1 = F.fgr_split_batch(len(ids), nl, rank, world)
+            ep = np.concatenate([[0], np.cumsum(sizes[ids] - 1)])
+            l0, l1, s0, s1, whole = F.fgr_split_batch(len(ids), nl, rank, world, ep, SPLIT_MIN)
+            if whole:   # routed whole on every rank, no exchange
+                assert (l0, l1, s0, s1) == (0, nl, nl, len(ids))
+                for n in ids:
+                    s_, c_ = o.route_net(int(n), demand)
+                    a, e = d.node_offset[n], d.node_offset[n + 1]
+                    seg[a:e] = s_[a:e]
+                    cost[n] = c_
+                for n in ids:
+                    o.commit_net(int(n), seg, demand)
+                continue
             mine = list(ids[l0:l1]) + list(ids[s0:s1])
             rec = np.zeros(d.num_nodes, np.int64)
             rc = np.zeros(d.num_nets, np.int64)
@@ -85,6 +99,9 @@ def _worker(rank, world, port, cfg, q):
         q.put((rank, seg.tobytes(), cost.tobytes(), demand.tobytes()))
     finally:
         dist.destroy_process_group()
+
+
+SPLIT_MIN = 20   # small enough that tiny/t1 exercise both the split and the whole-batch path
 
 
 def _run(cfg, world=2):
@@ -135,10 +152,35 @@ def test_split_covers_batch(world):
         nl = int(rng.integers(0, count + 1))
         seen = []
         for r in range(world):
-            l0, l1, s0, s1 = F.fgr_split_batch(count, nl, r, world)
+            l0, l1, s0, s1, whole = F.fgr_split_batch(count, nl, r, world)
+            assert whole == 0
             assert 0 <= l0 <= l1 <= nl <= s0 <= s1 <= count
             seen += list(range(l0, l1)) + list(range(s0, s1))
             assert abs((l1 - l0) - nl / world) <= 1 and abs((s1 - s0) - (count - nl) / world) <= 1
         assert sorted(seen) == list(range(count))
     with pytest.raises(F.FgrError):
         F.fgr_split_batch(10, 11, 0, 1)
+
+
+@pytest.mark.parametrize("world", [1, 2, 3, 8])
+def test_split_balances_tree_edges(world):
+    """Edge-balanced split: covering, and each rank's share of the large
+    (small) nets' edges is within one net's edges of the ideal."""
+    rng = np.random.default_rng(10 + world)
+    for _ in range(200):
+        count = int(rng.integers(1, 400))
+        nl = int(rng.integers(0, count + 1))
+        edges = np.concatenate([np.sort(rng.integers(33, 1000, size=nl))[::-1], rng.integers(1, 32, size=count - nl)])
+        ep = np.concatenate([[0], np.cumsum(edges)])
+        seen = []
+        for r in range(world):
+            l0, l1, s0, s1, whole = F.fgr_split_batch(count, nl, r, world, ep, 0)
+            assert whole == 0 and 0 <= l0 <= l1 <= nl <= s0 <= s1 <= count
+            seen += list(range(l0, l1)) + list(range(s0, s1))
+            el = edges[:nl].sum() / world
+            es = edges[nl:].sum() / world
+            assert abs(edges[l0:l1].sum() - el) <= (edges[:nl].max() if nl else 0)
+            assert abs(edges[s0:s1].sum() - es) <= (edges[nl:].max() if count > nl else 0)
+        assert sorted(seen) == list(range(count))
+        for r in range(world):   # below split_min: every rank takes the whole batch
+            assert F.fgr_split_batch(count, nl, r, world, ep, count + 1) == (0, nl, nl, count, 1)

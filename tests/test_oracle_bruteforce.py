@@ -67,3 +67,31 @@ def test_bruteforce_with_pin_spans_and_vias():
                 continue
             _, cost = o.route_net(n, demand)
             assert cost == brute_force_min(d, n, demand), (seed, n)
+
+
+def test_straight_edge_reading_R7():
+    """Reading R7: a straight tree edge takes the single candidate ls = lt with
+    one leg.  Pinned against the general degenerate L shapes (a zero-length leg on any layer at an
+    endpoint plus the bend via, on both bends): over random tiny trees with pins, Steiner nodes,
+    unequal via costs and congestion, the minimum over the general candidate set equals the
+    oracle's cost (sub-additivity of the via stack makes the extra candidates never better)."""
+    checked = straight = 0
+    for seed in range(60):
+        L = 3 + seed % 3
+        d = gen.random_small(seed=7000 + seed, nx=6, ny=5, nlayers=L, num_nets=5, kmax=4, literal_frac=0.3,
+                             caps=[1] * L)
+        rng = np.random.default_rng(seed)
+        d.via_cost = rng.integers(0, 60, size=L - 1).astype(np.int32)
+        o = Oracle(d)
+        demand = rng.integers(0, 3, size=(L, d.ny, d.nx)).astype(np.int32)
+        for n in range(d.num_nets):
+            a, m = d.node_offset[n], d.node_offset[n + 1] - d.node_offset[n]
+            if m < 2 or m > 4:
+                continue
+            ns = sum(1 for i in range(1, m) if d.x[a + i] == d.x[a + d.parent[a + i]] or
+                     d.y[a + i] == d.y[a + d.parent[a + i]])
+            _, cost = o.route_net(n, demand)
+            assert cost == brute_force_min(d, n, demand, general_straight=True), (seed, n)
+            checked += 1
+            straight += ns
+    assert checked > 40 and straight > 20, (checked, straight)
