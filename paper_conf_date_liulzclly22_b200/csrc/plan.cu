@@ -162,8 +162,10 @@ __global__ void __launch_bounds__(256) k_color(int R, const int* __restrict__ rl
     __shared__ uint32_t bits[8][COLOR_BITS / 32];
     __shared__ int defer[8][COLOR_DEFER];
     __shared__ int ndefer[8];
-    __shared__ int s_base, s_next;
-    if (threadIdx.x == 0) { s_base = 0; s_next = COLOR_CHUNK; }   // empty block: first taker refills
+    // CTA ticket block: base << 32 | next, one 64-bit word so that a rank's (base, index) pair is
+    // read atomically (a separate base word could be replaced by a refill between the two reads)
+    __shared__ unsigned long long s_tk;
+    if (threadIdx.x == 0) s_tk = (unsigned long long)COLOR_CHUNK;   // empty block: first taker refills
     __syncthreads();
     R = *rlim;   // phase 1: the ranks below the big-box threshold (k_color_big does the rest)
     const int w = threadIdx.x >> 5, lane = lane_id();
@@ -177,16 +179,15 @@ __global__ void __launch_bounds__(256) k_color(int R, const int* __restrict__ rl
         int r = 0;
         if (lane == 0) {
             for (;;) {
-                const int k = atomicAdd(&s_next, 1);
-                if (k < COLOR_CHUNK) { r = s_base + k; break; }
+                const unsigned long long tk = atomicAdd(&s_tk, 1ull);
+                const int k = (int)(tk & 0xFFFFFFFFull);
+                if (k < COLOR_CHUNK) { r = (int)(tk >> 32) + k; break; }
                 // block exhausted: one warp refills it; the others spin until the new block is published
                 if (k == COLOR_CHUNK) {
                     const int nb = atomicAdd(ticket, COLOR_CHUNK);
-                    s_base = nb;
-                    __threadfence_block();
-                    atomicExch(&s_next, 0);
+                    atomicExch(&s_tk, (unsigned long long)(unsigned)nb << 32);
                 } else {
-                    while (*(volatile int*)&s_next >= COLOR_CHUNK) __nanosleep(20);
+                    while ((int)(*(volatile unsigned long long*)&s_tk & 0xFFFFFFFFull) >= COLOR_CHUNK) __nanosleep(20);
                 }
             }
         }
