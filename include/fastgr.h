@@ -171,14 +171,15 @@ FGR_API fgr_status fgr_set_pattern(fgr_grid* grid, int32_t hybrid_t1, int32_t hy
  * fgr_set_dp_policy — which tree-DP kernel routes nets of more than 32 nodes
  * (all kernels compute the same DP, §III-D Eqs. (1)-(7), and give
  * bit-identical routes; the choice only changes speed):
- *   FGR_DP_AUTO  (default) nets of up to flow_max nodes: the tree-dataflow
- *                kernel; bigger nets: the heavy-path kernel while the net fits
- *                its shared-memory tables (~1.3k nodes at L = 9), above that the
- *                heavy-path contraction kernel (global workspace, any size up to
- *                65535 nodes);
- *   FGR_DP_HEAVY as AUTO without the tree-dataflow kernel;
- *   FGR_DP_HLD   the heavy-path contraction kernel for every net of > 32 nodes.
- * flow_max in [33, 65535] (default 64; ignored unless AUTO).  Errors: INVALID.
+ *   FGR_DP_AUTO  (default) the leaf-to-root dataflow kernel k_dp_tree while the
+ *                net's tables fit one SM's shared memory (~1.1k nodes at L = 9),
+ *                above that the heavy-path contraction kernel k_dp_hld (global
+ *                workspace, any size up to 65535 nodes);
+ *   FGR_DP_HEAVY the previous kernels: nets of up to flow_max nodes the tree-
+ *                dataflow kernel k_dp_flow, bigger nets the heavy-path kernel
+ *                k_dp_large (~1.3k nodes at L = 9), above that k_dp_hld;
+ *   FGR_DP_HLD   k_dp_hld for every net of > 32 nodes.
+ * flow_max in [33, 65535] (default 64; used by FGR_DP_HEAVY).  Errors: INVALID.
  * Host-only; takes effect at the next route call.
  */
 #define FGR_DP_AUTO 0

@@ -1207,6 +1207,12 @@ int fgr_large_limit(const fgr_grid* g) {
     return m;
 }
 
+// Largest net routed by a shared-memory kernel under the grid's DP policy (k_dp_tree for
+// FGR_DP_AUTO, k_dp_large for FGR_DP_HEAVY); bigger nets take k_dp_hld.
+int fgr_top_limit(const fgr_grid* g) {
+    return g->dp_policy == FGR_DP_AUTO ? fgr_tree_cap(g) : fgr_large_limit(g);
+}
+
 namespace {
 
 template <int LT>
@@ -1233,19 +1239,26 @@ cudaError_t launch_lt(fgr_grid* g, cudaStream_t st, const NetsView& nv, const in
     // kernel's shared-memory limit, then > 512, 257..512, 129..256, 65..128, 33..64 nodes (one bucket
     // unless lsplit is given), then the classes 9..32, 3..8 and 2 nodes.  Units are independent nets:
     // each non-empty unit gets its own stream (forked from and joined back into the caller's stream).
-    const int lim = fgr_large_limit(g);
+    const int lim = fgr_top_limit(g);
+    const bool tree = g->dp_policy == FGR_DP_AUTO;
     struct Unit { int kind, off, n, cap; };   // kind: 0 large, 1 midL, 2 midS, 3 two
     Unit units[10];
     int nu = 0;
     {
-        // thresholds (descending) with the number of large nets above each
+        // thresholds (descending) with the number of large nets above each; the tree kernel
+        // (FGR_DP_AUTO) takes three buckets: (512, lim], (128, 512], (32, 128]
         int thr[5] = {lim, 512, 256, 128, 64}, above[5] = {0, 0, 0, 0, 0};
+        bool use[5] = {true, true, !tree, true, !tree};
         if (lsplit) for (int k = 0; k < 5; k++) above[k] = min(lsplit[k], nlarge);
         for (int i = 0; i < 5; i++)
             for (int j = i + 1; j < 5; j++)
-                if (thr[j] > thr[i]) { int x = thr[i]; thr[i] = thr[j]; thr[j] = x; x = above[i]; above[i] = above[j]; above[j] = x; }
+                if (thr[j] > thr[i]) {
+                    int x = thr[i]; thr[i] = thr[j]; thr[j] = x; x = above[i]; above[i] = above[j]; above[j] = x;
+                    bool y = use[i]; use[i] = use[j]; use[j] = y;
+                }
         int prev = 0, cap = maxm_large;
         for (int k = 0; k <= 5 && prev < nlarge; k++) {
+            if (k < 5 && !use[k]) continue;
             const int end = (k < 5 && lsplit) ? max(prev, above[k]) : nlarge;
             if (end > prev) units[nu++] = Unit{0, prev, end - prev, min(cap, maxm_large)};
             prev = end;
@@ -1255,12 +1268,13 @@ cudaError_t launch_lt(fgr_grid* g, cudaStream_t st, const NetsView& nv, const in
     if (nmidL > 0) units[nu++] = Unit{1, nlarge, nmidL, 0};
     if (nmidS > 0) units[nu++] = Unit{2, nlarge + nmidL, nmidS, 0};
     if (ntwo > 0) units[nu++] = Unit{3, nlarge + nmidL + nmidS, ntwo, 0};
-    // kernel of a large-net unit (grid policy, fgr_set_dp_policy): the contraction kernel above the
-    // shared-memory limit or under FGR_DP_HLD; else the dataflow kernel up to flow_max nodes (FGR_DP_AUTO)
-    // and the heavy-path kernel
-    auto large_kind = [&](int cap) {   // 0 hld, 1 flow, 2 heavy-path
+    // kernel of a large-net unit (fgr_set_dp_policy): the contraction kernel above lim or under
+    // FGR_DP_HLD; FGR_DP_AUTO: the tree kernel; FGR_DP_HEAVY: the dataflow kernel up to flow_max
+    // nodes, then the heavy-path kernel
+    auto large_kind = [&](int cap) {   // 0 hld, 1 flow, 2 heavy-path, 3 tree
         if (cap > lim || g->dp_policy == FGR_DP_HLD) return 0;
-        if (g->dp_policy == FGR_DP_AUTO && cap <= g->flow_max && cap <= fgr_flow_max_nodes(g)) return 1;
+        if (tree) return 3;
+        if (cap <= g->flow_max && cap <= fgr_flow_max_nodes(g)) return 1;
         return 2;
     };
     const bool fork = nu > 1;
@@ -1293,6 +1307,9 @@ cudaError_t launch_lt(fgr_grid* g, cudaStream_t st, const NetsView& nv, const in
         const int lk = un.kind == 0 ? large_kind(un.cap) : -1;
         if (lk == 0) {
             e = fgr_launch_hld(g, su, nv, l, n, un.cap, os, commit, prep.hld, wsb ? wsb + wsoff[ui] : nullptr);
+            if (e != cudaSuccess) return e;
+        } else if (lk == 3) {
+            e = fgr_launch_tree(g, su, nv, l, n, un.cap, os, commit, prep.hld);
             if (e != cudaSuccess) return e;
         } else if (lk == 1) {
             e = fgr_launch_flow(g, su, nv, l, n, un.cap, os, commit, prep);

@@ -712,11 +712,13 @@ __global__ void __launch_bounds__(512, 1) k_dp_hld(GridView g, NetsView nv, cons
 // hd / len (path head and length by path position).
 constexpr int kPrepT = 256;
 
-__host__ __device__ inline size_t hprep_bytes(int m) { return 6 * a16((size_t)(m + 1) * 4) + a16((size_t)m + 1); }
+__host__ __device__ inline size_t hprep_bytes(int m) { return 8 * a16((size_t)(m + 1) * 4) + a16((size_t)m + 1); }
+constexpr int kLeafOrderMax = 4096;   // nets up to this size get the deepest-first leaf order (k_dp_tree)
 
 __global__ void __launch_bounds__(kPrepT) k_hld_prep(NetsView nv, const int32_t* __restrict__ list, uint16_t* hv_o,
                                                      uint16_t* cs_o, uint16_t* cl_o, uint16_t* pn_o, uint16_t* po_o,
-                                                     uint8_t* pr_o, int32_t* info_o, uint8_t* ld_o, unsigned char* gtmp,
+                                                     uint8_t* pr_o, int32_t* info_o, uint8_t* ld_o, uint16_t* lf_o,
+                                                     unsigned char* gtmp,
                                                      size_t gstride, int smem_cap) {
     extern __shared__ __align__(16) unsigned char smem[];
     __shared__ int s_cnt[kHldMaxRounds + 1], s_start[kHldMaxRounds + 1], s_nr, s_np;
@@ -733,7 +735,9 @@ __global__ void __launch_bounds__(kPrepT) k_hld_prep(NetsView nv, const int32_t*
     int* hd = (int*)(base + 3 * a16((size_t)(m + 1) * 4));
     int* len = (int*)(base + 4 * a16((size_t)(m + 1) * 4));
     int* par = (int*)(base + 5 * a16((size_t)(m + 1) * 4));
-    uint8_t* ld = base + 6 * a16((size_t)(m + 1) * 4);
+    int* dep = (int*)(base + 6 * a16((size_t)(m + 1) * 4));
+    unsigned* lk = (unsigned*)(base + 7 * a16((size_t)(m + 1) * 4));
+    uint8_t* ld = base + 8 * a16((size_t)(m + 1) * 4);
     for (int i = tid; i < m; i += kPrepT) { sub[i] = 1; hk[i] = 0; cnt[i] = 0; par[i] = nv.par[a0 + i]; }
     if (tid <= kHldMaxRounds) s_cnt[tid] = 0;
     __syncthreads();
@@ -763,9 +767,11 @@ __global__ void __launch_bounds__(kPrepT) k_hld_prep(NetsView nv, const int32_t*
     if (tid == 0) {
         // light depth: a light edge adds one (parent index < child index: one forward pass)
         ld[0] = 0;
+        dep[0] = 0;
         int mx = 0;
         for (int i = 1; i < m; i++) {
             const int p = par[i];
+            dep[i] = dep[p] + 1;
             const int hvp = hk[p] ? (int)(0xFFFFu - (hk[p] & 0xFFFFu)) : -1;
             const int d = ld[p] + (hvp != i ? 1 : 0);
             ld[i] = (uint8_t)d;
@@ -827,6 +833,22 @@ __global__ void __launch_bounds__(kPrepT) k_hld_prep(NetsView nv, const int32_t*
     }
     for (int v = tid; v < m; v += kPrepT) ld_o[a0 + v] = ld[v];
     if (tid == 0) info_o[net] = np | (s_nr << 16);
+    // leaves (= path bottoms) deepest first, ties by index: the start order of k_dp_tree's
+    // leaf-to-root dataflow (long chains start first)
+    if (m > kLeafOrderMax) return;
+    __syncthreads();
+    for (int q = tid; q < np; q += kPrepT) {
+        int w = hd[q];
+        while (hk[w]) w = (int)(0xFFFFu - (hk[w] & 0xFFFFu));
+        lk[q] = ((unsigned)(0xFFFF - dep[w]) << 16) | (unsigned)w;
+    }
+    __syncthreads();
+    for (int q = tid; q < np; q += kPrepT) {
+        const unsigned key = lk[q];
+        int rank = 0;
+        for (int j = 0; j < np; j++) rank += lk[j] < key;
+        lf_o[a0 + rank] = (uint16_t)(key & 0xFFFFu);
+    }
 }
 
 struct HldPlan {
@@ -917,7 +939,7 @@ cudaError_t fgr_launch_hld(fgr_grid* g, cudaStream_t st, const NetsView& nv, con
 
 cudaError_t fgr_launch_hld_prep(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int count,
                                 int maxm, uint16_t* hv, uint16_t* cs, uint16_t* cl, uint16_t* pn, uint16_t* po,
-                                uint8_t* pr, int32_t* info, uint8_t* ld) {
+                                uint8_t* pr, int32_t* info, uint8_t* ld, uint16_t* lf) {
     if (count <= 0) return cudaSuccess;
     static int configured = 0;
     if (!configured) {
@@ -937,7 +959,7 @@ cudaError_t fgr_launch_hld_prep(fgr_grid* g, cudaStream_t st, const NetsView& nv
         if (e != cudaSuccess) return e;
         dyn = cap;   // smaller nets of the launch still use shared memory
     }
-    k_hld_prep<<<count, kPrepT, dyn, st>>>(nv, list, hv, cs, cl, pn, po, pr, info, ld, gtmp, stride, (int)dyn);
+    k_hld_prep<<<count, kPrepT, dyn, st>>>(nv, list, hv, cs, cl, pn, po, pr, info, ld, lf, gtmp, stride, (int)dyn);
     g->stats.kernel_launches++;
     return cudaGetLastError();
 }

@@ -1,0 +1,584 @@
+// dp_tree.cu — S4 tree DP + S5 backtrack for nets of FGR_SMALL_NET+1 .. tree_cap(L)
+// nodes (the large nets whose tables fit one SM's shared memory; bigger nets take
+// k_dp_hld).  One CTA per net; the S6 commit of these nets runs afterwards in the
+// grid-wide k_commit_nets so that a lone large net does not push its tens of
+// thousands of unit-edge REDs through a single SM.
+//
+// Recurrences (§III-D, Eqs. (1)-(7), L582-756; readings R3, R5-R11 in
+// DESIGN.md §3).  For node v with children Ch(v), pin span [plo, phi]:
+//     F_v(lo,hi) = V(lo,hi) + Σ_{c∈Ch(v)} min_{l∈[lo,hi]} E_c(l)                  (Eq. (2), R3)
+//     B_v(ls)    = min_{lo <= a(ls), hi >= b(ls)} F_v(lo,hi),  a = min(ls,plo), b = max(ls,phi)
+//     E_v(lt)    = min_ls C_v(ls,lt) + B_v(ls)                                 (Eqs. (1),(3), R5, R7)
+// and at the root the generalised Eq. (4) (R9): min over spans containing the pin span.
+// With at most one child c the span minimum has the closed form
+//     B_v(ls) = min_l E_c(l) + V(min(a,l), max(b,l))
+//             = min_l E_c(l) + max(vp[b], vp[l]) - min(vp[a], vp[l])   (vp = via prefix, non-decreasing)
+// (a leaf is the case E_c ≡ 0), and for a bent L edge (R5: ls and lt of different directions)
+//     E_v(lt) = leg2(lt) + min_{ls: dir(ls) != dir(lt)} [B_v(ls) + leg1(ls) + |vp[ls] - vp[lt]|].
+//
+// Organisation (the paper's kernel walks a net's nodes in DFS order with one block per
+// net and the L parallel computation flows in its threads):
+//   P0  topology and the per-stage decomposition (k_hld_prep) into shared memory;
+//   P1  every edge's leg costs gathered at once (costs are fixed during a batch);
+//   P2  values, leaf-to-root dataflow: a lane group (lane = layer) takes leaves by ticket
+//       (deepest first) and walks upwards; at a node with several children only the last
+//       child to finish (pending-child counter) continues with the parent, so no group
+//       ever waits and the critical path is the tree height, not a sum over levels;
+//   P3  argmin tables in parallel over all nodes (R11 order): for every node the child
+//       span phi_v[span of the parent] (the whole S5 decision for that edge) and recE;
+//   P4  top-down backtrack along heavy paths (one byte load per node);
+//   P5  outputs (seg, cost).
+// All per-net tables live in shared memory at compile-time offsets (no pointer
+// arithmetic in the hot loops), values are 32-bit with DPX min-plus (VIADDMNMX).
+#include "dp_common.cuh"
+
+#ifdef FGR_TREE_TIMING
+#define TMARK(i) do { if (threadIdx.x == 0) tmk[i] = clock64(); } while (0)
+#else
+#define TMARK(i) do { } while (0)
+#endif
+
+namespace {
+
+constexpr int kTreeMaxRounds = 17;
+
+__host__ __device__ constexpr int tr_ns(int LT) { return LT * (LT + 1) / 2; }
+__host__ __device__ __forceinline__ int tr_tri(int LT, int lo, int hi) { return lo * LT - (lo * (lo - 1)) / 2 + (hi - lo); }
+__host__ __device__ constexpr int tr_a16(int b) { return (b + 15) & ~15; }
+
+enum { TE_BENT = 0, TE_SH = 1, TE_SV = 2, TE_HYB = 3 };
+
+// Bytes of the shared-memory layout below (TL<LT, NT, CAP>::BYTES).
+__host__ __device__ constexpr int tl_bytes(int LT, int NT, int CAP) {
+    return 3 * tr_a16(4 * LT * CAP) + tr_a16(4 * CAP) + 4 * tr_a16(2 * CAP) + 2 * tr_a16(2 * CAP + 2) + tr_a16(tr_ns(LT) * CAP) +
+           tr_a16(LT * CAP) + 4 * tr_a16(CAP) + (NT / 32) * groups_of(LT) * tr_a16(5 * LT * LT);
+}
+
+// Shared-memory layout for capacity CAP nodes (all offsets compile-time constants).
+template <int LT, int NT, int CAP>
+struct TL {
+    static constexpr int NS = tr_ns(LT);
+    static constexpr int GPW = groups_of(LT);
+    static constexpr int NW = NT / 32;
+    static constexpr int E = 0;                                   // uint32 [CAP][LT]  E_v(lt)
+    static constexpr int LG1 = E + tr_a16(4 * LT * CAP);          // uint32 [CAP][LT]  leg 1 by ls (straight: the leg, INF off-direction)
+    static constexpr int LG2 = LG1 + tr_a16(4 * LT * CAP);        // uint32 [CAP][LT]  leg 2 by lt
+    static constexpr int PEND = LG2 + tr_a16(4 * LT * CAP);       // uint32 [CAP]      children still pending (P2)
+    static constexpr int PAR = PEND + tr_a16(4 * CAP);            // uint16 [CAP]
+    static constexpr int CS = PAR + tr_a16(2 * CAP);              // uint16 [CAP + 1]  child CSR
+    static constexpr int CL = CS + tr_a16(2 * CAP + 2);           // uint16 [CAP]
+    static constexpr int LF = CL + tr_a16(2 * CAP);               // uint16 [CAP]      leaves, deepest first
+    static constexpr int PN = LF + tr_a16(2 * CAP);               // uint16 [CAP]      heavy-path nodes (bottom -> head)
+    static constexpr int PO = PN + tr_a16(2 * CAP);               // uint16 [CAP + 1]  path starts
+    static constexpr int PHI = PO + tr_a16(2 * CAP + 2);          // uint8 [CAP][NS]   span of v for each span of its parent
+    static constexpr int RECE = PHI + tr_a16(NS * CAP);           // uint8 [CAP][LT]   argmin ls of E_v(lt)
+    static constexpr int ET = RECE + tr_a16(LT * CAP);            // uint8 [CAP]       edge type
+    static constexpr int PLO = ET + tr_a16(CAP);                  // int8 [CAP]
+    static constexpr int PHIP = PLO + tr_a16(CAP);                // int8 [CAP]
+    static constexpr int SPAN = PHIP + tr_a16(CAP);               // uint8 [CAP]       chosen span (S5)
+    static constexpr int SCR = SPAN + tr_a16(CAP);                // per group: uint32 [LT][LT] suffix minima + uint8 [LT][LT] argmin hi
+    static constexpr int SCR_G = tr_a16(5 * LT * LT);
+    static constexpr int BYTES = SCR + NW * GPW * SCR_G;
+    static_assert(BYTES == tl_bytes(LT, NT, CAP), "layout size");
+};
+
+// Largest capacity of the 512-thread variant that fits the opt-in shared memory of an SM
+// (227 KB less the kernel's static shared memory and a margin).
+__host__ __device__ constexpr int tree_cap512(int LT) {
+    int cap = 4096;
+    while (cap > 64 && tl_bytes(LT, 512, cap) + 4096 > 227 * 1024) cap -= 16;
+    return cap;
+}
+
+template <int LT>
+struct Lane {                       // per-lane constants of a lane group (lane = layer gl)
+    int gl, gbase;
+    unsigned gmask;
+    uint32_t myvp;                  // vp[gl]
+    uint32_t D[LT];                 // |vp[ls] - vp[gl]| if dir(ls) != dir(gl), else INF  (bent-edge via + direction rule)
+};
+
+// C_v argmin / values for a hybrid edge: M[lt][ls] (transfer matrix of the L + Z candidates).
+template <int LT>
+__device__ __forceinline__ const uint32_t* hyb_row(const HybView& hy, int gnode, int lt) {
+    return hy.M + ((size_t)hy.slot[gnode] * LT + lt) * LT;
+}
+
+template <int LT, int NT, int CAP>
+__global__ void __launch_bounds__(NT, (NT >= 512 ? 1 : (NT >= 256 ? 2 : 4)))
+k_dp_tree(GridView g, NetsView nv, const int32_t* __restrict__ list, int count, Out o, HldPrep hp, HybView hy) {
+    using T = TL<LT, NT, CAP>;
+    constexpr int NS = T::NS, GPW = T::GPW, NW = T::NW;
+    extern __shared__ __align__(16) unsigned char sm[];
+    __shared__ uint8_t s_los[2][FGR_MAXL];
+    __shared__ uint8_t s_tlo[NS], s_thi[NS];
+    __shared__ int s_rb[kTreeMaxRounds + 1];
+    __shared__ int s_ticket;
+    __shared__ uint32_t s_root_span, s_root_cost;
+    uint32_t* const sE = reinterpret_cast<uint32_t*>(sm + T::E);
+    uint32_t* const sLG1 = reinterpret_cast<uint32_t*>(sm + T::LG1);
+    uint32_t* const sLG2 = reinterpret_cast<uint32_t*>(sm + T::LG2);
+    uint32_t* const sPEND = reinterpret_cast<uint32_t*>(sm + T::PEND);
+    uint16_t* const sPAR = reinterpret_cast<uint16_t*>(sm + T::PAR);
+    uint16_t* const sCS = reinterpret_cast<uint16_t*>(sm + T::CS);
+    uint16_t* const sCL = reinterpret_cast<uint16_t*>(sm + T::CL);
+    uint16_t* const sLF = reinterpret_cast<uint16_t*>(sm + T::LF);
+    uint16_t* const sPN = reinterpret_cast<uint16_t*>(sm + T::PN);
+    uint16_t* const sPO = reinterpret_cast<uint16_t*>(sm + T::PO);
+    uint8_t* const sPHI = sm + T::PHI;
+    uint8_t* const sRECE = sm + T::RECE;
+    uint8_t* const sET = sm + T::ET;
+    int8_t* const sPLO = reinterpret_cast<int8_t*>(sm + T::PLO);
+    int8_t* const sPHIP = reinterpret_cast<int8_t*>(sm + T::PHIP);
+    uint8_t* const sSPAN = sm + T::SPAN;
+
+    const int tid = threadIdx.x;
+    const int warp = tid >> 5, lane = lane_id();
+    const int gi = lane / LT;
+    const bool glane = gi < GPW;
+    Lane<LT> ln;
+    ln.gl = glane ? lane - gi * LT : 0;
+    ln.gbase = glane ? gi * LT : 0;
+    ln.gmask = glane ? (((1u << LT) - 1u) << ln.gbase) : (1u << lane);
+    uint32_t hmask = 0;
+#pragma unroll
+    for (int l = 0; l < LT; l++) hmask |= (g.dir[l] == 0 ? 1u : 0u) << l;
+    ln.myvp = 0;
+#pragma unroll
+    for (int l = 0; l < LT; l++) ln.myvp = (l == ln.gl) ? g.viapre[l] : ln.myvp;
+    {
+        const bool myh = (hmask >> ln.gl) & 1u;
+#pragma unroll
+        for (int l = 0; l < LT; l++) {
+            const uint32_t vl = g.viapre[l];
+            const bool lh = (hmask >> l) & 1u;
+            ln.D[l] = lh != myh ? (vl >= ln.myvp ? vl - ln.myvp : ln.myvp - vl) : FGR_INF;
+        }
+    }
+    uint32_t* const scrF = reinterpret_cast<uint32_t*>(sm + T::SCR + (warp * GPW + (glane ? gi : 0)) * T::SCR_G);
+    uint8_t* const scrH = reinterpret_cast<uint8_t*>(scrF + LT * LT);
+    for (int i = tid; i < 2 * FGR_MAXL; i += NT) s_los[i / FGR_MAXL][i % FGR_MAXL] = g.layer_of_slot[i / FGR_MAXL][i % FGR_MAXL];
+    for (int lo = 0; lo < LT; lo++)
+        for (int hi = lo + tid; hi < LT; hi += NT) { s_tlo[tr_tri(LT, lo, hi)] = (uint8_t)lo; s_thi[tr_tri(LT, lo, hi)] = (uint8_t)hi; }
+    bool waited = false;
+
+    for (int idx = blockIdx.x; idx < count; idx += gridDim.x) {
+#ifdef FGR_TREE_TIMING
+        long long tmk[8];
+#endif
+        TMARK(0);
+        const int net = list[idx];
+        const int a0 = nv.off[net];
+        const int m = nv.off[net + 1] - a0;
+        const int info = hp.info[net];
+        const int np = info & 0xFFFF, nr = info >> 16;   // np = number of heavy paths = number of leaves
+        const int hnet = hy.net ? hy.net[net] : -1;
+        // ---- P0: topology (demand-independent: overlaps the refresh under PDL)
+        for (int i = tid; i < m; i += NT) {
+            int et = TE_BENT;
+            int u = 0xFFFF;
+            if (i) {
+                u = nv.par[a0 + i];
+                const int xv = nv.x[a0 + i], yv = nv.y[a0 + i], xu = nv.x[a0 + u], yu = nv.y[a0 + u];
+                et = (yv == yu) ? TE_SH : (xv == xu) ? TE_SV : TE_BENT;
+                if (et == TE_BENT && hnet >= 0 && hy.slot[a0 + i] >= 0) et = TE_HYB;
+            }
+            sPAR[i] = (uint16_t)u;
+            sET[i] = (uint8_t)et;
+            sPLO[i] = nv.plo[a0 + i];
+            sPHIP[i] = nv.phi[a0 + i];
+            const int c0 = hp.cs[a0 + i];
+            const int c1 = i + 1 < m ? hp.cs[a0 + i + 1] : m - 1;
+            sCS[i] = (uint16_t)c0;
+            sPEND[i] = (uint32_t)(c1 - c0);
+            if (i + 1 < m) sCL[i] = hp.cl[a0 + i];
+            sPN[i] = hp.pn[a0 + i];
+            if (i < np) { sLF[i] = hp.lf[a0 + i]; sPO[i] = hp.po[a0 + i]; }
+            if (et == TE_SH || et == TE_SV) {   // the off-direction layers of a straight edge stay impossible (R6, R7)
+#pragma unroll
+                for (int l = 0; l < LT; l++) sLG1[i * LT + l] = FGR_INF;
+            }
+        }
+        for (int q = tid; q < np; q += NT) {
+            const int r = hp.pr[a0 + q];
+            if (q == 0 || hp.pr[a0 + q - 1] != r) s_rb[r] = q;
+        }
+        if (tid == 0) { sCS[m] = (uint16_t)(m - 1); sPO[np] = (uint16_t)m; s_ticket = 0; }
+        if (!waited) { pdl_wait(); waited = true; }   // the refresh must be complete before the gathers
+        __syncthreads();
+        TMARK(1);
+        // ---- P1: leg gathers, 4 tasks per edge:
+        //   0: leg 1 H on row y_v, 1: leg 1 V on col x_v, 2: leg 2 V on col x_u, 3: leg 2 H on row y_u
+        for (int task = tid; task < 4 * (m - 1); task += NT) {
+            const int v = 1 + (task >> 2), type = task & 3;
+            const int et = sET[v];
+            if (et == TE_HYB || (et == TE_SH && type != 0) || (et == TE_SV && type != 1)) continue;
+            const int u = sPAR[v];
+            const int xv = nv.x[a0 + v], yv = nv.y[a0 + v], xu = nv.x[a0 + u], yu = nv.y[a0 + u];
+            const bool H = type == 0 || type == 3;
+            const int line = type == 0 ? yv : type == 1 ? xv : type == 2 ? xu : yu;
+            const int pa = H ? min(xv, xu) : min(yv, yu);
+            const int pb = H ? max(xv, xu) : max(yv, yu);
+            const uint32_t* P = H ? g.h.P : g.v.P;
+            const uint32_t* SB = H ? g.h.SB : g.v.SB;
+            const int len = H ? g.h.len : g.v.len, W = H ? g.h.W : g.v.W, nseg = H ? g.h.nseg : g.v.nseg;
+            const int cnt = H ? g.h.cnt : g.v.cnt;
+            uint32_t* dst = (type >= 2 ? sLG2 : sLG1) + v * LT;
+            const uint8_t* los = s_los[H ? 0 : 1];
+            const size_t ia = ((size_t)line * len + pa) * W, ib = ((size_t)line * len + pb) * W;
+            const size_t sa = ((size_t)line * nseg + (pa >> FGR_SEG_SHIFT)) * W;
+            const size_t sb = ((size_t)line * nseg + (pb >> FGR_SEG_SHIFT)) * W;
+            const int nq = W >> 2;
+#pragma unroll
+            for (int q = 0; q < 4; q++) {
+                if (q < nq) {
+                    const uint4 Pa = __ldg(reinterpret_cast<const uint4*>(P + ia) + q);
+                    const uint4 Pb = __ldg(reinterpret_cast<const uint4*>(P + ib) + q);
+                    const uint4 Sa = __ldg(reinterpret_cast<const uint4*>(SB + sa) + q);
+                    const uint4 Sb = __ldg(reinterpret_cast<const uint4*>(SB + sb) + q);
+                    if (4 * q + 0 < cnt) dst[los[4 * q + 0]] = (Sb.x + Pb.x) - (Sa.x + Pa.x);
+                    if (4 * q + 1 < cnt) dst[los[4 * q + 1]] = (Sb.y + Pb.y) - (Sa.y + Pa.y);
+                    if (4 * q + 2 < cnt) dst[los[4 * q + 2]] = (Sb.z + Pb.z) - (Sa.z + Pa.z);
+                    if (4 * q + 3 < cnt) dst[los[4 * q + 3]] = (Sb.w + Pb.w) - (Sa.w + Pa.w);
+                }
+            }
+        }
+        __syncthreads();
+        TMARK(2);
+        // ---- P2: values, leaf-to-root dataflow.  cur = node of the group (-1: take a ticket, -2: done)
+        if (glane) {
+            int cur = -1;
+            while (true) {
+                if (cur == -1) {
+                    int t = 0;
+                    if (ln.gl == 0) t = atomicAdd(&s_ticket, 1);
+                    t = __shfl_sync(ln.gmask, t, ln.gbase);
+                    cur = t < np ? (int)sLF[t] : -2;
+                }
+                if (cur < 0) break;
+                const int v = cur;
+                const int k0 = sCS[v], k1 = sCS[v + 1];
+                const int plo = sPLO[v], phi = sPHIP[v];
+                const bool pin = plo >= 0;
+                uint32_t B;
+                if (v == 0 || k1 - k0 >= 2) {
+                    // span table: lane lo builds F(lo, hi) over all children, suffix minima over hi
+                    uint32_t acc[LT];
+#pragma unroll
+                    for (int hi = 0; hi < LT; hi++) acc[hi] = hi >= ln.gl ? g.viapre[hi] - ln.myvp : FGR_INF;
+                    for (int k = k0; k < k1; k++) {
+                        const uint32_t* Ec = sE + sCL[k] * LT;
+                        uint32_t run = FGR_INF;
+#pragma unroll
+                        for (int hi = 0; hi < LT; hi++) {
+                            run = min(run, hi >= ln.gl ? Ec[hi] : FGR_INF);
+                            acc[hi] = sat_add(acc[hi], run);
+                        }
+                    }
+                    if (v == 0) {
+                        // generalised Eq. (4) (R9): first (lo, hi) in lexicographic order among the minimal
+                        // spans containing the root's pin span (any span for a Steiner root)
+                        const int ra = pin ? plo : LT - 1, rb = pin ? phi : 0;
+                        uint32_t bv = FGR_INF, bh = 0;
+#pragma unroll
+                        for (int hi = LT - 1; hi >= 0; hi--)
+                            if (hi >= rb && acc[hi] <= bv) { bv = acc[hi]; bh = (uint32_t)hi; }
+                        if (ln.gl > ra) bv = FGR_INF;
+                        uint32_t best = FGR_INF, blo = 0, bhi = 0;
+                        for (int lo = 0; lo < LT; lo++) {
+                            const uint32_t x = __shfl_sync(ln.gmask, bv, ln.gbase + lo);
+                            const uint32_t h = __shfl_sync(ln.gmask, bh, ln.gbase + lo);
+                            if (x < best) { best = x; blo = (uint32_t)lo; bhi = h; }
+                        }
+                        if (ln.gl == 0) { s_root_cost = best; s_root_span = (uint32_t)tr_tri(LT, (int)blo, (int)bhi); }
+                        cur = -2;
+                        continue;
+                    }
+                    uint32_t run = FGR_INF;
+#pragma unroll
+                    for (int b = LT - 1; b >= 0; b--) {
+                        run = min(run, acc[b]);
+                        scrF[ln.gl * LT + b] = run;
+                    }
+                    __syncwarp(ln.gmask);
+                    const int a = pin ? min(ln.gl, plo) : ln.gl, b = pin ? max(ln.gl, phi) : ln.gl;
+                    B = FGR_INF;
+#pragma unroll
+                    for (int lo = 0; lo < LT; lo++)
+                        if (lo <= a) B = min(B, scrF[lo * LT + b]);
+                    __syncwarp(ln.gmask);
+                } else {
+                    // at most one child: B(ls) = min_l X(l) + max(vp[b], vp[l]) - min(vp[a], vp[l])
+                    uint32_t vpa = ln.myvp, vpb = ln.myvp;
+                    if (pin) {
+                        vpa = min(vpa, g.viapre[plo]);
+                        vpb = max(vpb, g.viapre[phi]);
+                    }
+                    const uint32_t* Ec = sE + (k1 > k0 ? sCL[k0] : 0) * LT;
+                    const bool leaf = k1 == k0;
+                    uint32_t b0 = 0xFFFFFFFFu, b1 = 0xFFFFFFFFu;
+#pragma unroll
+                    for (int l = 0; l < LT; l++) {
+                        const uint32_t vl = g.viapre[l];
+                        const uint32_t w = max(vpb, vl) - min(vpa, vl);
+                        const uint32_t x = leaf ? 0u : Ec[l];
+                        if (l & 1) b1 = __viaddmin_u32(x, w, b1);
+                        else b0 = __viaddmin_u32(x, w, b0);
+                    }
+                    B = min(min(b0, b1), FGR_INF);
+                }
+                // edge step: E_v(lt), lane = lt
+                const int et = sET[v];
+                uint32_t Ev;
+                if (et == TE_BENT) {
+                    const uint32_t bp = sat_add(B, sLG1[v * LT + ln.gl]);
+                    uint32_t e0 = 0xFFFFFFFFu, e1 = 0xFFFFFFFFu;
+#pragma unroll
+                    for (int ls = 0; ls < LT; ls++) {
+                        const uint32_t x = __shfl_sync(ln.gmask, bp, ln.gbase + ls);
+                        if (ls & 1) e1 = __viaddmin_u32(x, ln.D[ls], e1);
+                        else e0 = __viaddmin_u32(x, ln.D[ls], e0);
+                    }
+                    Ev = sat_add(min(min(e0, e1), FGR_INF), sLG2[v * LT + ln.gl]);
+                } else if (et == TE_HYB) {
+                    const uint32_t* M = hyb_row<LT>(hy, a0 + v, ln.gl);
+                    uint32_t e0 = FGR_INF;
+#pragma unroll
+                    for (int ls = 0; ls < LT; ls++) {
+                        const uint32_t x = __shfl_sync(ln.gmask, B, ln.gbase + ls);
+                        e0 = min(e0, sat_add(x, __ldg(M + ls)));
+                    }
+                    Ev = e0;
+                } else {
+                    Ev = sat_add(B, sLG1[v * LT + ln.gl]);
+                }
+                sE[v * LT + ln.gl] = Ev;
+                __syncwarp(ln.gmask);
+                int last = 0;
+                if (ln.gl == 0) {
+                    __threadfence_block();
+                    last = atomicSub(&sPEND[sPAR[v]], 1u) == 1u;
+                    __threadfence_block();
+                }
+                last = __shfl_sync(ln.gmask, last, ln.gbase);
+                cur = last ? (int)sPAR[v] : -1;
+            }
+        }
+        __syncthreads();
+        TMARK(3);
+        // ---- P3: argmin tables (R11), one lane group per node
+        for (int base = 1 + warp * GPW; base < m; base += NW * GPW) {
+            const int vq = base + gi;
+            if (!glane || vq >= m) continue;
+            const int v = vq;
+            const int k0 = sCS[v], k1 = sCS[v + 1];
+            const int plo = sPLO[v], phi = sPHIP[v];
+            const bool pin = plo >= 0;
+            // F row lo = gl, then suffix minima over hi with the smallest attaining hi
+            uint32_t acc[LT];
+#pragma unroll
+            for (int hi = 0; hi < LT; hi++) acc[hi] = hi >= ln.gl ? g.viapre[hi] - ln.myvp : FGR_INF;
+            for (int k = k0; k < k1; k++) {
+                const uint32_t* Ec = sE + sCL[k] * LT;
+                uint32_t run = FGR_INF;
+#pragma unroll
+                for (int hi = 0; hi < LT; hi++) {
+                    run = min(run, hi >= ln.gl ? Ec[hi] : FGR_INF);
+                    acc[hi] = sat_add(acc[hi], run);
+                }
+            }
+            {
+                uint32_t run = 0xFFFFFFFFu, rh = 0;
+#pragma unroll
+                for (int b = LT - 1; b >= 0; b--) {
+                    if (acc[b] <= run) { run = acc[b]; rh = (uint32_t)b; }
+                    scrF[ln.gl * LT + b] = run;
+                    scrH[ln.gl * LT + b] = (uint8_t)rh;
+                }
+            }
+            __syncwarp(ln.gmask);
+            // B(ls) and its span: smallest lo (then that lo's smallest hi) among the minimal spans
+            const int a = pin ? min(ln.gl, plo) : ln.gl, b = pin ? max(ln.gl, phi) : ln.gl;
+            uint32_t B = FGR_INF;
+            int blo = -1;
+#pragma unroll
+            for (int lo = 0; lo < LT; lo++) {
+                const uint32_t f = scrF[lo * LT + b];
+                if (lo <= a && f < B) { B = f; blo = lo; }
+            }
+            const int spanB = blo >= 0 ? tr_tri(LT, blo, scrH[blo * LT + b]) : 0;
+            __syncwarp(ln.gmask);
+            // recE(lt): smallest ls minimising B(ls) + C(ls, lt)
+            const int et = sET[v];
+            int bls = 0;
+            if (et == TE_BENT) {
+                const uint32_t bp = sat_add(B, sLG1[v * LT + ln.gl]);
+                uint32_t best = FGR_INF;
+#pragma unroll
+                for (int ls = 0; ls < LT; ls++) {
+                    const uint32_t x = __viaddmin_u32(__shfl_sync(ln.gmask, bp, ln.gbase + ls), ln.D[ls], FGR_INF);
+                    if (x < best) { best = x; bls = ls; }
+                }
+            } else if (et == TE_HYB) {
+                const uint32_t* M = hyb_row<LT>(hy, a0 + v, ln.gl);
+                uint32_t best = FGR_INF;
+#pragma unroll
+                for (int ls = 0; ls < LT; ls++) {
+                    const uint32_t x = sat_add(__shfl_sync(ln.gmask, B, ln.gbase + ls), __ldg(M + ls));
+                    if (x < best) { best = x; bls = ls; }
+                }
+            } else {
+                bls = ln.gl;   // R7: one candidate, ls = lt
+            }
+            sRECE[v * LT + ln.gl] = (uint8_t)bls;
+            // phi row lo = gl: child layer = smallest l in [lo, hi] minimising E_v(l) (R11), then its span
+            const int sol = __shfl_sync(ln.gmask, spanB, ln.gbase + bls);
+            const uint32_t* Ev = sE + v * LT;
+            uint8_t* ph = sPHI + v * NS;
+            uint32_t be = FGR_INF;
+            int curs = 0;
+#pragma unroll
+            for (int hi = 0; hi < LT; hi++) {
+                const int sh = __shfl_sync(ln.gmask, sol, ln.gbase + hi);
+                const uint32_t ev = Ev[hi];
+                if (hi == ln.gl || (hi > ln.gl && ev < be)) { be = ev; curs = sh; }
+                if (hi >= ln.gl) ph[tr_tri(LT, ln.gl, hi)] = (uint8_t)curs;
+            }
+        }
+        __syncthreads();
+        TMARK(4);
+        // ---- P4: top-down backtrack (S5) along heavy paths, shallowest light depth first
+        for (int r = 0; r < nr; r++) {
+            const int q0 = s_rb[r], q1 = r > 0 ? s_rb[r - 1] : np;
+            for (int q = q0 + tid; q < q1; q += NT) {
+                const int kb = sPO[q], ke = sPO[q + 1];
+                int k = ke - 1;
+                int v = sPN[k];
+                int s;
+                if (v == 0) s = (int)s_root_span;
+                else { s = sPHI[v * NS + sSPAN[sPAR[v]]]; sSPAN[v] = (uint8_t)s; }
+                if (v == 0) sSPAN[0] = (uint8_t)s;
+                for (k = ke - 2; k >= kb; k--) {
+                    v = sPN[k];
+                    s = sPHI[v * NS + s];
+                    sSPAN[v] = (uint8_t)s;
+                }
+            }
+            __syncthreads();
+        }
+        TMARK(5);
+        // ---- P5: outputs; the S6 commit follows in k_commit_nets
+        for (int i = 1 + tid; i < m; i += NT) {
+            const int su = sSPAN[sPAR[i]];
+            const int lo = s_tlo[su], hi = s_thi[su];
+            const uint32_t* Ei = sE + i * LT;
+            uint32_t be = Ei[lo];
+            int lt = lo;
+            for (int l = lo + 1; l <= hi; l++) {
+                const uint32_t e = Ei[l];
+                if (e < be) { be = e; lt = l; }
+            }
+            const int ls = sRECE[i * LT + lt];
+            const int et = sET[i];
+            const bool straight = et == TE_SH || et == TE_SV;
+            const uint32_t bend = seg_bend(((hmask >> ls) & 1u) ? 0 : 1, ((hmask >> lt) & 1u) ? 0 : 1, straight);
+            const uint32_t s = bend | ((uint32_t)ls << 8) | ((uint32_t)lt << 16) | ((uint32_t)straight << 24);
+            if (o.rec_seg) o.rec_seg[o.rec_off[o.list_base + idx] + i] = s;
+            else o.seg[a0 + i] = s;
+        }
+        if (tid == 0) {
+            if (o.rec_seg) { o.rec_seg[o.rec_off[o.list_base + idx]] = 0xFFFFFFFFu; o.rec_cost[o.list_base + idx] = s_root_cost; }
+            else { o.seg[a0] = 0xFFFFFFFFu; o.cost[net] = s_root_cost; }
+        }
+        __syncthreads();
+        TMARK(6);
+#ifdef FGR_TREE_TIMING
+        if (threadIdx.x == 0 && m > 400)
+            printf("TREE m=%d np=%d nr=%d NT=%d load=%lld gather=%lld values=%lld argmin=%lld back=%lld out=%lld total=%lld\n",
+                   m, np, nr, NT, tmk[1] - tmk[0], tmk[2] - tmk[1], tmk[3] - tmk[2], tmk[4] - tmk[3], tmk[5] - tmk[4],
+                   tmk[6] - tmk[5], tmk[6] - tmk[0]);
+#endif
+    }
+}
+
+// S6 for the nets of a tree-kernel launch: one thread per tree edge, blocks of 256 edges.
+__global__ void __launch_bounds__(256) k_commit_nets(GridView g, NetsView nv, const int32_t* __restrict__ list, int count,
+                                                     int chunks, Out o, HybView hy) {
+    __shared__ Hdr hs;
+    init_hdr(&hs, g);
+    __syncthreads();
+    const int idx = blockIdx.x / chunks;
+    if (idx >= count) return;
+    const int net = list[idx];
+    const int a0 = nv.off[net], m = nv.off[net + 1] - a0;
+    const int i = 1 + (blockIdx.x % chunks) * 256 + threadIdx.x;
+    if (i >= m) return;
+    const uint32_t s = o.rec_seg ? o.rec_seg[o.rec_off[o.list_base + idx] + i] : o.seg[a0 + i];
+    const int u = nv.par[a0 + i];
+    commit_edge(g, &hs, nv.x[a0 + i], nv.y[a0 + i], nv.x[a0 + u], nv.y[a0 + u], s, hyb_z(hy, a0 + i, s, g.L));
+}
+
+template <int LT, int NT, int CAP>
+cudaError_t launch_tree_v(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int n, const Out& o,
+                          const HldPrep& hp) {
+    using T = TL<LT, NT, CAP>;
+    static int configured = 0;
+    if (!configured) {
+        cudaError_t e = cudaFuncSetAttribute(k_dp_tree<LT, NT, CAP>, cudaFuncAttributeMaxDynamicSharedMemorySize, T::BYTES);
+        if (e != cudaSuccess) return e;
+        configured = 1;
+    }
+    int per_sm = NT >= 512 ? 1 : (NT >= 256 ? 2 : 4);
+    const int by_smem = g->max_smem / (T::BYTES + 2048);
+    if (by_smem < per_sm) per_sm = by_smem < 1 ? 1 : by_smem;
+    const int grid = n < per_sm * g->num_sms ? n : per_sm * g->num_sms;
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(grid);
+    cfg.blockDim = dim3(NT);
+    cfg.dynamicSmemBytes = T::BYTES;
+    cfg.stream = st;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, k_dp_tree<LT, NT, CAP>, g->view, nv, list, n, o, hp, g->hy.view());
+}
+
+template <int LT>
+cudaError_t launch_tree_lt(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int n, int maxm,
+                           const Out& o, const HldPrep& hp) {
+    if (maxm <= 128) return launch_tree_v<LT, 128, 128>(g, st, nv, list, n, o, hp);
+    if (maxm <= 512) return launch_tree_v<LT, 256, 512>(g, st, nv, list, n, o, hp);
+    return launch_tree_v<LT, 512, tree_cap512(LT)>(g, st, nv, list, n, o, hp);
+}
+
+}  // namespace
+
+int fgr_tree_cap(const fgr_grid* g) {
+    switch (g->L) {
+#define FGR_LT(k) case k: return tree_cap512(k);
+        FGR_LT(2) FGR_LT(3) FGR_LT(4) FGR_LT(5) FGR_LT(6) FGR_LT(7) FGR_LT(8) FGR_LT(9) FGR_LT(10) FGR_LT(11)
+        FGR_LT(12) FGR_LT(13) FGR_LT(14) FGR_LT(15) FGR_LT(16)
+#undef FGR_LT
+        default: return 0;
+    }
+}
+
+cudaError_t fgr_launch_tree(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int n, int maxm,
+                            const Out& o, bool commit, const HldPrep& hp) {
+    if (n <= 0) return cudaSuccess;
+    cudaError_t e;
+    switch (g->L) {
+#define FGR_LT(k) case k: e = launch_tree_lt<k>(g, st, nv, list, n, maxm, o, hp); break;
+        FGR_LT(2) FGR_LT(3) FGR_LT(4) FGR_LT(5) FGR_LT(6) FGR_LT(7) FGR_LT(8) FGR_LT(9) FGR_LT(10) FGR_LT(11)
+        FGR_LT(12) FGR_LT(13) FGR_LT(14) FGR_LT(15) FGR_LT(16)
+#undef FGR_LT
+        default: return cudaErrorInvalidValue;
+    }
+    if (e != cudaSuccess || !commit) return e;
+    g->stats.kernel_launches++;
+    const int chunks = (maxm - 1 + 255) / 256;
+    k_commit_nets<<<n * chunks, 256, 0, st>>>(g->view, nv, list, n, chunks, o, g->hy.view());
+    return cudaGetLastError();
+}

@@ -91,6 +91,7 @@ struct HldPrep {
     const uint8_t* pr;
     const int32_t* info;
     const uint8_t* ld;     // light depth of every node (= the round of its path)
+    const uint16_t* lf;    // leaves (path bottoms) by descending depth, ties by index (k_dp_tree), [a0 + q], q < npaths
 };
 
 // Per-node results of the large-net tree analysis (global, indexed by global node index).
@@ -264,9 +265,14 @@ cudaError_t fgr_launch_flow(fgr_grid* g, cudaStream_t st, const NetsView& nv, co
                             const Out& o, bool commit, const Prep& prep);
 int fgr_flow_max_nodes(const fgr_grid* g);
 int fgr_large_limit(const fgr_grid* g);
+int fgr_top_limit(const fgr_grid* g);   // size above which nets take k_dp_hld (policy dependent)
 cudaError_t fgr_launch_hld_prep(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int count,
                                 int maxm, uint16_t* hv, uint16_t* cs, uint16_t* cl, uint16_t* pn, uint16_t* po,
-                                uint8_t* pr, int32_t* info, uint8_t* ld);
+                                uint8_t* pr, int32_t* info, uint8_t* ld, uint16_t* lf);
+// k_dp_tree (dp_tree.cu): nets of FGR_SMALL_NET+1 .. fgr_tree_cap(g) nodes; commit = launch k_commit_nets after it
+cudaError_t fgr_launch_tree(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int n, int maxm,
+                            const Out& o, bool commit, const HldPrep& hp);
+int fgr_tree_cap(const fgr_grid* g);
 // ws: global workspace of fgr_hld_ws_bytes(g, n, maxm) bytes (distinct per concurrent launch)
 cudaError_t fgr_launch_hld(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int n, int maxm,
                            const Out& o, bool commit, const HldPrep& hp, unsigned char* ws);

@@ -420,7 +420,7 @@ __global__ void k_finalize(int N, const int* __restrict__ counters, const unsign
         if (m > FGR_SMALL_NET) {
             atomicAdd(&nlarge[c], 1);
             atomicMax(&maxm[c], m);
-            // large-net size buckets (> fgr_large_limit, 512, 256, 128, 64)
+            // large-net size buckets (> fgr_top_limit, 512, 256, 128, 64)
             if (m > 64) atomicAdd(&lsplit[5 * c + 4], 1);
             if (m > 128) atomicAdd(&lsplit[5 * c + 3], 1);
             if (m > 256) atomicAdd(&lsplit[5 * c + 2], 1);
@@ -628,7 +628,7 @@ extern "C" FGR_API fgr_status fgr_plan(fgr_grid* g, const fgr_nets* nets, int32_
     auto* segsum = (unsigned long long*)box_r;   // box_r no longer needed after colouring
     FGR_CHECK_CUDA(g, cudaMemsetAsync(segsum, 0, sizeof(unsigned long long) * ((size_t)R + 1), st));
     k_finalize<<<(N + 255) / 256, 256, 0, st>>>(N, counters, keys_s, bkeys_s, msize, segb, order, batch_of_net,
-                                                d_nlarge, d_maxm, segsum, d_ntwo, d_n9, d_ls, fgr_large_limit(g));
+                                                d_nlarge, d_maxm, segsum, d_ntwo, d_n9, d_ls, fgr_top_limit(g));
     FGR_CHECK_CUDA(g, cudaGetLastError());
     g->stats.kernel_launches += 6;
     int B = 0;

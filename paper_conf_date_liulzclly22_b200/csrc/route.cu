@@ -177,7 +177,10 @@ extern "C" FGR_API fgr_status fgr_set_dp_policy(fgr_grid* g, int32_t policy, int
     if (policy != FGR_DP_AUTO && policy != FGR_DP_HEAVY && policy != FGR_DP_HLD)
         return fgr_set_error(FGR_ERR_INVALID, "unknown DP policy %d", policy);
     if (flow_max < FGR_SMALL_NET + 1 || flow_max > 65535) return fgr_set_error(FGR_ERR_INVALID, "flow_max %d out of range", flow_max);
-    if (policy != g->dp_policy) g->cache.prep_valid = false;   // the decompositions to build depend on the policy
+    if (policy != g->dp_policy) {   // the decompositions and the size buckets depend on the policy
+        g->cache.prep_valid = false;
+        g->cache.valid = false;
+    }
     g->dp_policy = policy;
     g->flow_max = flow_max;
     return FGR_OK;
@@ -227,7 +230,7 @@ extern "C" FGR_API fgr_status fgr_route_batch_ex(fgr_grid* g, const fgr_nets* ne
     fgr_status s = fgr_hyb_prepare(g, st, nv, nets->num_nets, nets->num_nodes, list, count, nullptr, 1, zmid_out);
     if (s != FGR_OK) return s;
     Prep bp{};
-    if (hc[0] > 0 && (hc[4] > fgr_large_limit(g) || g->dp_policy == FGR_DP_HLD)) {
+    if (hc[0] > 0 && (hc[4] > fgr_top_limit(g) || g->dp_policy != FGR_DP_HEAVY)) {
         g->cache.prep_valid = false;   // s_hldp now holds this batch's decomposition
         s = hld_prep_list(g, nets, list, hc[0], hc[4], st, &bp.hld);
         if (s != FGR_OK) return s;
@@ -282,7 +285,7 @@ static fgr_status batch_info(fgr_grid* g, const fgr_nets* nets, const int32_t* o
     if (e != cudaSuccess) return fgr_cuda_fail(g, e, "exec order");
     if (B > 0) {
         k_batch_info<<<B, 256, 0, st>>>(B, batch_offset, order, nets->node_offset, nets->x, nets->y, nets->parent,
-                                        d_nl, d_mm, d_segb, d_n2, d_n9, keys, d_ls, fgr_large_limit(g));
+                                        d_nl, d_mm, d_segb, d_n2, d_n9, keys, d_ls, fgr_top_limit(g));
         FGR_CHECK_CUDA(g, cudaGetLastError());
         int bits = 42;
         while ((1LL << (bits - 42)) <= B) bits++;
@@ -318,7 +321,7 @@ static fgr_status hld_prep_list(fgr_grid* g, const fgr_nets* nets, const int32_t
                                 HldPrep* out) {
     const size_t M = (size_t)nets->num_nodes, N = (size_t)nets->num_nets;
     cudaError_t e;
-    char* p = (char*)fgr_scratch(g->s_hldp, 5 * a16h(2 * M) + 2 * a16h(M) + a16h(4 * N) + 64, &e);
+    char* p = (char*)fgr_scratch(g->s_hldp, 6 * a16h(2 * M) + 2 * a16h(M) + a16h(4 * N) + 64, &e);
     if (e != cudaSuccess) return fgr_cuda_fail(g, e, "hld prep arrays");
     auto take = [&](size_t b) { char* q = p; p += a16h(b); return q; };
     uint16_t* hv = (uint16_t*)take(2 * M); uint16_t* cs = (uint16_t*)take(2 * M); uint16_t* cl = (uint16_t*)take(2 * M);
@@ -326,8 +329,9 @@ static fgr_status hld_prep_list(fgr_grid* g, const fgr_nets* nets, const int32_t
     uint8_t* pr = (uint8_t*)take(M);
     int32_t* info = (int32_t*)take(4 * N);
     uint8_t* ld = (uint8_t*)take(M);
-    FGR_CHECK_CUDA(g, fgr_launch_hld_prep(g, st, fgr_nets_view(nets), list, nl, maxm, hv, cs, cl, pn, po, pr, info, ld));
-    *out = HldPrep{hv, cs, cl, pn, po, pr, info, ld};
+    uint16_t* lf = (uint16_t*)take(2 * M);
+    FGR_CHECK_CUDA(g, fgr_launch_hld_prep(g, st, fgr_nets_view(nets), list, nl, maxm, hv, cs, cl, pn, po, pr, info, ld, lf));
+    *out = HldPrep{hv, cs, cl, pn, po, pr, info, ld, lf};
     return FGR_OK;
 }
 
@@ -338,14 +342,14 @@ static fgr_status ensure_prep(fgr_grid* g, const fgr_nets* nets, int B, cudaStre
     PlanCache& c = g->cache;
     if (c.prep_valid) return FGR_OK;
     const int R = B > 0 ? c.h_off[B] : 0;
-    const int lim = fgr_large_limit(g);
+    const int lim = fgr_top_limit(g);
     int maxm = 0, nl = 0, nh = 0;
     for (int b = 0; b < B; b++) {
         maxm = c.h_maxm[b] > maxm ? c.h_maxm[b] : maxm;
         nl += c.h_nlarge[b];
         nh += c.h_lsplit[5 * b];
     }
-    const bool all_hld = g->dp_policy == FGR_DP_HLD;
+    const bool all_hld = g->dp_policy != FGR_DP_HEAVY;   // k_dp_tree and k_dp_hld both read the HLD decomposition
     if (all_hld) nh = nl;
     c.prep = Prep{};
     if (nl == 0) { c.prep_valid = true; return FGR_OK; }

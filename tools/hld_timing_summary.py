@@ -5,5 +5,5 @@ rows = [{k: int(v) for k, v in re.findall(r'(\w+)=(\d+)', l)} for l in t.split('
 rows.sort(key=lambda r: -r['m'])
 for r in rows[:5]:
     print(r)
-for k in ['load', 'gather', 'p2', 'p3a', 'p3b', 'p4', 'p5', 'p6', 'total']:
+for k in ["load","gather","p2","p3a","p3b","p4","p5","p6","total"]:
     print(k, int(statistics.mean(r[k] for r in rows)))

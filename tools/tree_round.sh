@@ -1,0 +1,13 @@
+#!/bin/bash
+# GPU check of the large-net kernels: parity (hld_check + variant tests), bench, per-phase timing.
+TAG=${1:-r02e}
+mkdir -p gpurun_out
+timeout 600 python tools/hld_check.py bignets,chains,t5,huge,t1 > gpurun_out/${TAG}_check.txt 2>&1
+echo "check rc=$?" >> gpurun_out/${TAG}_check.txt
+tail -12 gpurun_out/${TAG}_check.txt
+timeout 300 python bench.py --steps 10 --warmup 3 --no-cpu-baseline --no-e2e > gpurun_out/${TAG}_bench.json 2> gpurun_out/${TAG}_bench.err
+python -c "import json;d=json.load(open('gpurun_out/${TAG}_bench.json'));print('bench', d['ms_per_step'], d['route_ms'], d['plan_ms'], d.get('kernels_ms_per_step'))"
+FGR_LIB_PATH=build_t/libfastgr_tt.so timeout 300 python bench.py --steps 1 --warmup 0 --no-cpu-baseline --no-e2e > gpurun_out/${TAG}_timing.txt 2>&1
+grep "TREE" gpurun_out/${TAG}_timing.txt | sort -t= -k2 -n -r | head -5
+timeout 300 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/${TAG}_launches.csv python bench.py --steps 1 --warmup 1 --no-cpu-baseline --no-e2e > /dev/null 2>&1
+python tools/launch_batches.py gpurun_out/${TAG}_launches.csv > gpurun_out/${TAG}_batches.txt 2>&1; head -3 gpurun_out/${TAG}_batches.txt
