@@ -1280,11 +1280,16 @@ cudaError_t launch_lt(fgr_grid* g, cudaStream_t st, const NetsView& nv, const in
     const bool fork = nu > 1;
     cudaError_t e;
     // global workspaces of the large-net units (one region each: the units run concurrently)
-    size_t wsoff[8] = {0}, wstot = 0;
+    size_t wsoff[10] = {0}, wstot = 0;
     unsigned char* wsb = nullptr;
     {
-        for (int ui = 0; ui < nu; ui++)
-            if (units[ui].kind == 0 && large_kind(units[ui].cap) == 0) { wsoff[ui] = wstot; wstot += (fgr_hld_ws_bytes(g, units[ui].n, units[ui].cap) + 255) & ~(size_t)255; }
+        for (int ui = 0; ui < nu; ui++) {
+            if (units[ui].kind != 0) continue;
+            const int lk = large_kind(units[ui].cap);
+            const size_t b = lk == 0 ? fgr_hld_ws_bytes(g, units[ui].n, units[ui].cap) : 0;
+            wsoff[ui] = wstot;
+            wstot += (b + 255) & ~(size_t)255;
+        }
         if (wstot > 0) {
             wsb = (unsigned char*)fgr_scratch(g->s_hldw, wstot, &e);
             if (e != cudaSuccess) return e;
