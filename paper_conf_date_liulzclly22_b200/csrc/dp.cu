@@ -1279,6 +1279,7 @@ cudaError_t launch_lt(fgr_grid* g, cudaStream_t st, const NetsView& nv, const in
     };
     const bool fork = nu > 1;
     cudaError_t e;
+    int tree_off = 0, tree_n = 0, tree_cap = 0;   // the tree-kernel units (contiguous in the list) share one commit
     // global workspaces of the large-net units (one region each: the units run concurrently)
     size_t wsoff[10] = {0}, wstot = 0;
     unsigned char* wsb = nullptr;
@@ -1314,7 +1315,9 @@ cudaError_t launch_lt(fgr_grid* g, cudaStream_t st, const NetsView& nv, const in
             e = fgr_launch_hld(g, su, nv, l, n, un.cap, os, commit, prep.hld, wsb ? wsb + wsoff[ui] : nullptr);
             if (e != cudaSuccess) return e;
         } else if (lk == 3) {
-            e = fgr_launch_tree(g, su, nv, l, n, un.cap, os, commit, prep.hld);
+            e = fgr_launch_tree(g, su, nv, l, n, un.cap, os, false, prep.hld);   // committed after the join
+            if (tree_n == 0) { tree_off = un.off; tree_cap = un.cap; }
+            tree_n += n;
             if (e != cudaSuccess) return e;
         } else if (lk == 1) {
             e = fgr_launch_flow(g, su, nv, l, n, un.cap, os, commit, prep);
@@ -1349,6 +1352,14 @@ cudaError_t launch_lt(fgr_grid* g, cudaStream_t st, const NetsView& nv, const in
             if ((e = cudaEventRecord(g->ev_join[i], g->side[i])) != cudaSuccess) return e;
             if ((e = cudaStreamWaitEvent(st, g->ev_join[i], 0)) != cudaSuccess) return e;
         }
+    }
+    if (commit && tree_n > 0) {
+        Out os = o;
+        os.list_base = o.list_base + tree_off;
+        const int ps = fgr_prof_begin(g, PROF_COMMIT, st);
+        e = fgr_launch_commit_nets(g, st, nv, list + tree_off, tree_n, tree_cap, os);
+        fgr_prof_end(g, ps, st);
+        if (e != cudaSuccess) return e;
     }
     return cudaSuccess;
 }

@@ -112,11 +112,13 @@ struct TL {
 
 // Largest capacity of the 512-thread variant that fits the opt-in shared memory of an SM
 // (227 KB less the kernel's static shared memory and a margin).
-__host__ __device__ constexpr int tree_cap512(int LT) {
+__host__ __device__ constexpr int tree_cap_nt(int LT, int NT) {
     int cap = 4096;
-    while (cap > 64 && tl_bytes(LT, 512, cap) + 4096 > 227 * 1024) cap -= 16;
+    while (cap > 64 && tl_bytes(LT, NT, cap) + 4096 > 227 * 1024) cap -= 16;
     return cap;
 }
+constexpr int kTreeBigNT = 384;   // threads of the variant for the largest nets (up to 168 registers per thread)
+__host__ __device__ constexpr int tree_cap512(int LT) { return tree_cap_nt(LT, kTreeBigNT); }
 
 template <int LT>
 struct Lane {                       // per-lane constants of a lane group (lane = layer gl)
@@ -321,7 +323,7 @@ __device__ __forceinline__ void tree_node_argmin(const GridView& g, const HybVie
 }
 
 template <int LT, int NT, int CAP>
-__global__ void __launch_bounds__(NT, (NT >= 512 ? 1 : (NT >= 256 ? 2 : 4)))
+__global__ void __launch_bounds__(NT, (NT >= 384 ? 1 : (NT >= 256 ? 2 : 4)))
 k_dp_tree(GridView g, NetsView nv, const int32_t* __restrict__ list, int count, Out o, HldPrep hp, HybView hy) {
     using T = TL<LT, NT, CAP>;
     constexpr int NS = T::NS, GPW = T::GPW, NW = T::NW;
@@ -446,26 +448,17 @@ k_dp_tree(GridView g, NetsView nv, const int32_t* __restrict__ list, int count, 
             const size_t ia = ((size_t)line * len + pa) * W, ib = ((size_t)line * len + pb) * W;
             const size_t sa = ((size_t)line * nseg + (pa >> FGR_SEG_SHIFT)) * W;
             const size_t sb = ((size_t)line * nseg + (pb >> FGR_SEG_SHIFT)) * W;
-            const int nq = W >> 2;
-            const bool oneseg = (pa >> FGR_SEG_SHIFT) == (pb >> FGR_SEG_SHIFT);   // segment bases cancel
-#pragma unroll
-            for (int q = 0; q < 4; q++) {
-                if (q < nq) {
-                    const uint4 Pa = __ldg(reinterpret_cast<const uint4*>(P + ia) + q);
-                    const uint4 Pb = __ldg(reinterpret_cast<const uint4*>(P + ib) + q);
-                    uint4 Sa = make_uint4(0, 0, 0, 0), Sb = make_uint4(0, 0, 0, 0);
-                    if (!oneseg) {
-                        Sa = __ldg(reinterpret_cast<const uint4*>(SB + sa) + q);
-                        Sb = __ldg(reinterpret_cast<const uint4*>(SB + sb) + q);
-                    }
-                    if (4 * q + 0 < cnt) dst[los[4 * q + 0]] = (Sb.x + Pb.x) - (Sa.x + Pa.x);
-                    if (4 * q + 1 < cnt) dst[los[4 * q + 1]] = (Sb.y + Pb.y) - (Sa.y + Pa.y);
-                    if (4 * q + 2 < cnt) dst[los[4 * q + 2]] = (Sb.z + Pb.z) - (Sa.z + Pa.z);
-                    if (4 * q + 3 < cnt) dst[los[4 * q + 3]] = (Sb.w + Pb.w) - (Sa.w + Pa.w);
-                }
+            for (int q = 0; q < (W >> 2); q++) {
+                const uint4 Pa = __ldg(reinterpret_cast<const uint4*>(P + ia) + q);
+                const uint4 Pb = __ldg(reinterpret_cast<const uint4*>(P + ib) + q);
+                const uint4 Sa = __ldg(reinterpret_cast<const uint4*>(SB + sa) + q);
+                const uint4 Sb = __ldg(reinterpret_cast<const uint4*>(SB + sb) + q);
+                if (4 * q + 0 < cnt) dst[los[4 * q + 0]] = (Sb.x + Pb.x) - (Sa.x + Pa.x);
+                if (4 * q + 1 < cnt) dst[los[4 * q + 1]] = (Sb.y + Pb.y) - (Sa.y + Pa.y);
+                if (4 * q + 2 < cnt) dst[los[4 * q + 2]] = (Sb.z + Pb.z) - (Sa.z + Pa.z);
+                if (4 * q + 3 < cnt) dst[los[4 * q + 3]] = (Sb.w + Pb.w) - (Sa.w + Pa.w);
             }
         }
-        cta_sync();
         cta_sync();
         TMARK(2);
         // ---- P2 + P3: values (leaf-to-root dataflow, one walking group per warp) and, on warps
@@ -753,7 +746,7 @@ __global__ void __launch_bounds__(256) k_commit_nets(GridView g, NetsView nv, co
 template <int LT, int NT, int CAP>
 int tree_grid(const fgr_grid* g, int n) {
     using T = TL<LT, NT, CAP>;
-    int per_sm = NT >= 512 ? 1 : (NT >= 256 ? 2 : 4);
+    int per_sm = NT >= 384 ? 1 : (NT >= 256 ? 2 : 4);
     const int by_smem = g->max_smem / (T::BYTES + 2048);
     if (by_smem < per_sm) per_sm = by_smem < 1 ? 1 : by_smem;
     return n < per_sm * g->num_sms ? n : per_sm * g->num_sms;
@@ -787,7 +780,7 @@ cudaError_t launch_tree_lt(fgr_grid* g, cudaStream_t st, const NetsView& nv, con
                            const Out& o, const HldPrep& hp) {
     if (maxm <= 128) return launch_tree_v<LT, 128, 128>(g, st, nv, list, n, o, hp);
     if (maxm <= 512) return launch_tree_v<LT, 256, 512>(g, st, nv, list, n, o, hp);
-    return launch_tree_v<LT, 512, tree_cap512(LT)>(g, st, nv, list, n, o, hp);
+    return launch_tree_v<LT, kTreeBigNT, tree_cap512(LT)>(g, st, nv, list, n, o, hp);
 }
 
 }  // namespace
@@ -814,6 +807,12 @@ cudaError_t fgr_launch_tree(fgr_grid* g, cudaStream_t st, const NetsView& nv, co
         default: return cudaErrorInvalidValue;
     }
     if (e != cudaSuccess || !commit) return e;
+    return fgr_launch_commit_nets(g, st, nv, list, n, maxm, o);
+}
+
+cudaError_t fgr_launch_commit_nets(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int n, int maxm,
+                                   const Out& o) {
+    if (n <= 0 || maxm < 2) return cudaSuccess;
     g->stats.kernel_launches++;
     const int chunks = (maxm - 1 + 255) / 256;
     k_commit_nets<<<n * chunks, 256, 0, st>>>(g->view, nv, list, n, chunks, o, g->hy.view());

@@ -272,6 +272,9 @@ cudaError_t fgr_launch_hld_prep(fgr_grid* g, cudaStream_t st, const NetsView& nv
 // k_dp_tree (dp_tree.cu): nets of FGR_SMALL_NET+1 .. fgr_tree_cap(g) nodes; commit = launch k_commit_nets after it
 cudaError_t fgr_launch_tree(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int n, int maxm,
                             const Out& o, bool commit, const HldPrep& hp);
+// S6 for nets routed without an in-kernel commit: one thread per tree edge (reads seg or the route records)
+cudaError_t fgr_launch_commit_nets(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int n, int maxm,
+                                   const Out& o);
 int fgr_tree_cap(const fgr_grid* g);
 // ws: global workspace of fgr_hld_ws_bytes(g, n, maxm) bytes (distinct per concurrent launch)
 cudaError_t fgr_launch_hld(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int n, int maxm,
