@@ -454,6 +454,7 @@ def main():
             "kernels_ms_per_step": {c: v[0] / steps for c, v in prof.items() if v[1]},
             "kernels_launches_per_step": {c: v[1] / steps for c, v in prof.items() if v[1]},
             "refresh_segments_per_step": stats["refresh_segments"],
+            "batch_loop": {0: "direct launches", 1: "captured", 2: "CUDA Graph replay"}.get(stats.get("graph_mode", 0)),
             "ripup": ripup,
             "wall_s": t_wall,
         }

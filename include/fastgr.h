@@ -251,6 +251,19 @@ FGR_API fgr_status fgr_split_batch(int32_t count, int32_t nlarge, const int64_t*
  */
 FGR_API fgr_status fgr_set_exchange(fgr_grid* grid, int32_t split_min, int32_t emulate_world);
 
+/*
+ * fgr_set_graph — replay the single-GPU batch loop of fgr_route_all(_ex) as a CUDA
+ * Graph (on = 1, the default) or issue it launch by launch (on = 0).  The batches
+ * run in sequence either way (one kernel invocation per batch);
+ * the graph only removes the host issue cost and the inter-launch gaps.  A call
+ * whose plan (host batch sizes), nets/output pointers, stream, DP policy and
+ * pattern equal those of the previous call is captured once and then replayed;
+ * any change re-runs the loop directly.  Not used with a communicator, with
+ * emulated ranks or while the profiler is on.  Routes are identical in both modes.
+ * Errors: INVALID (NULL grid).  Host-only.
+ */
+FGR_API fgr_status fgr_set_graph(fgr_grid* grid, int32_t on);
+
 /* Multi-GPU (one process per GPU).  fgr_comm_unique_id fills 128 bytes on the
  * root rank; broadcast them (e.g. torch.distributed) and call fgr_comm_init on
  * every rank with the grid already created on that rank's device. */
@@ -320,6 +333,8 @@ typedef struct {
     int64_t kernel_launches;           /* kernels launched by the library                       */
     int32_t num_batches, world, rank;
     int32_t exchanged_batches;         /* multi-GPU: batches split across ranks (others routed whole) */
+    int32_t graph_mode;                /* batch loop of the call: 0 direct, 1 captured, 2 replayed (fgr_set_graph) */
+    int32_t reserved;
 } fgr_stats;
 FGR_API fgr_status fgr_get_stats(fgr_grid* grid, fgr_stats* out);
 

@@ -27,9 +27,12 @@ fgr_status fgr_cuda_fail(fgr_grid* g, cudaError_t e, const char* where) {
     return fgr_set_error(FGR_ERR_CUDA, "CUDA error %s (%s) at %s", cudaGetErrorName(e), cudaGetErrorString(e), where);
 }
 
+unsigned long long g_scratch_gen = 0;
+
 void* fgr_scratch(Scratch& s, size_t bytes, cudaError_t* err) {
     *err = cudaSuccess;
     if (bytes <= s.bytes && s.p) return s.p;
+    g_scratch_gen++;
     if (s.p) cudaFree(s.p);
     s.p = nullptr;
     s.bytes = 0;
@@ -235,6 +238,8 @@ extern "C" FGR_API fgr_status fgr_grid_create(const fgr_grid_desc* d, int device
 extern "C" FGR_API fgr_status fgr_grid_destroy(fgr_grid* g) {
     if (!g) return FGR_OK;
     cudaSetDevice(g->device);
+    if (g->rg.exec) cudaGraphExecDestroy(g->rg.exec);
+    if (g->rg.cap) cudaStreamDestroy(g->rg.cap);
     if (g->comm) ncclCommDestroy(g->comm);
     cudaFree(g->mem);
     cudaFree(g->d_table);

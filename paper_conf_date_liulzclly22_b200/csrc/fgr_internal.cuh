@@ -157,6 +157,20 @@ struct PlanCache {
     int cap = 0;
 };
 
+extern unsigned long long g_scratch_gen;   // bumped whenever a scratch buffer is (re)allocated
+
+// Captured single-GPU batch loop of fgr_route_all (route.cu): valid while every input of
+// the loop's launches is unchanged (key, host batch mirrors, scratch generation).
+struct RouteGraph {
+    bool use = true;
+    cudaGraphExec_t exec = nullptr;
+    cudaStream_t cap = nullptr;       // private stream the loop is captured on
+    std::vector<long long> key;       // pointers, sizes, policy, pattern, initial full-dirty flag, scratch gen
+    std::vector<long long> mirror;    // h_off, h_nlarge, h_maxm, h_ntwo, h_n9, h_lsplit, h_segb
+    long long launches = 0;           // library kernel launches in the captured loop
+    std::vector<long long> seen_key, seen_mirror;   // the previous direct run (capture on the next equal call)
+};
+
 struct Scratch {            // grow-only device scratch
     void* p = nullptr;
     size_t bytes = 0;
@@ -219,6 +233,7 @@ struct fgr_grid {
     int split_min = 2048;
     int emu_world = 0;
     HybState hy;
+    RouteGraph rg;
     Scratch s_hyb[3];
     Scratch s_rip[6];          // rip-up extraction and task graph (ripup.cu)
 };

@@ -10,6 +10,7 @@
 #include <cub/cub.cuh>
 
 #include <cstdlib>
+#include <cstdint>
 #include <cstring>
 
 #include "fgr_internal.cuh"
@@ -169,6 +170,15 @@ extern "C" FGR_API fgr_status fgr_set_exchange(fgr_grid* g, int32_t split_min, i
         return fgr_set_error(FGR_ERR_INVALID, "bad exchange settings %d / %d", split_min, emulate_world);
     g->split_min = split_min;
     g->emu_world = emulate_world;
+    return FGR_OK;
+}
+
+extern "C" FGR_API fgr_status fgr_set_graph(fgr_grid* g, int32_t on) {
+    if (!g) return fgr_set_error(FGR_ERR_INVALID, "grid is NULL");
+    g->rg.use = on != 0;
+    if (!g->rg.use && g->rg.exec) { cudaGraphExecDestroy(g->rg.exec); g->rg.exec = nullptr; }
+    g->rg.key.clear();
+    g->rg.seen_key.clear();
     return FGR_OK;
 }
 
@@ -435,16 +445,96 @@ extern "C" FGR_API fgr_status fgr_route_all_ex(fgr_grid* g, const fgr_nets* nets
     FGR_CHECK_CUDA(g, cudaMemsetAsync(g->d_stats, 0, 4 * sizeof(unsigned long long), st));
     const bool emu = !g->comm && g->emu_world > 1;
     if (!g->comm && !emu) {
-        for (int b = 0; b < B; b++) {
-            const long long bound = b > 0 ? c.h_segb[b - 1] : (long long)g->total_segs;
-            FGR_CHECK_CUDA(g, refresh_before_dp(g, st, bound));
-            if (hy.active) FGR_CHECK_CUDA(g, fgr_launch_hyb_tm(g, st, nv, hy.boff[b], hy.boff[b + 1] - hy.boff[b]));
-            const int o0 = c.h_off[b], cnt = c.h_off[b + 1] - o0, nl = c.h_nlarge[b], n2 = c.h_ntwo[b], n9 = c.h_n9[b];
-            FGR_CHECK_CUDA(g, fgr_launch_dp(g, st, nv, c.exec + o0, nl, n9, cnt - nl - n9 - n2, n2, c.h_maxm[b],
-                                            seg_out, net_cost, nullptr, nullptr, nullptr, 0, true, &c.prep,
-                                            c.h_lsplit + 5 * b));
+        // the batch loop (batches in sequence), replayed as a CUDA Graph when
+        // nothing its launches depend on changed since the previous call (fgr_set_graph)
+        auto loop = [&](cudaStream_t st) -> cudaError_t {
+            cudaError_t e2;
+            for (int b = 0; b < B; b++) {
+                const long long bound = b > 0 ? c.h_segb[b - 1] : (long long)g->total_segs;
+                if ((e2 = refresh_before_dp(g, st, bound)) != cudaSuccess) return e2;
+                if (hy.active && (e2 = fgr_launch_hyb_tm(g, st, nv, hy.boff[b], hy.boff[b + 1] - hy.boff[b])) != cudaSuccess)
+                    return e2;
+                const int o0 = c.h_off[b], cnt = c.h_off[b + 1] - o0, nl = c.h_nlarge[b], n2 = c.h_ntwo[b], n9 = c.h_n9[b];
+                if ((e2 = fgr_launch_dp(g, st, nv, c.exec + o0, nl, n9, cnt - nl - n9 - n2, n2, c.h_maxm[b], seg_out,
+                                        net_cost, nullptr, nullptr, nullptr, 0, true, &c.prep, c.h_lsplit + 5 * b)) !=
+                    cudaSuccess)
+                    return e2;
+            }
+            return fgr_launch_hyb_zmid(g, st, seg_out, zmid_out);
+        };
+        RouteGraph& rg = g->rg;
+        g->stats.graph_mode = 0;
+        if (!rg.use || g->prof.on || B == 0) {
+            FGR_CHECK_CUDA(g, loop(st));
+            return FGR_OK;
         }
-        FGR_CHECK_CUDA(g, fgr_launch_hyb_zmid(g, st, seg_out, zmid_out));
+        std::vector<long long> key = {(long long)(uintptr_t)c.exec, B, (long long)(uintptr_t)nets->node_offset,
+                                      (long long)(uintptr_t)nets->x, (long long)(uintptr_t)nets->y,
+                                      (long long)(uintptr_t)nets->pin_lo, (long long)(uintptr_t)nets->pin_hi,
+                                      (long long)(uintptr_t)nets->parent, N, M, (long long)(uintptr_t)seg_out,
+                                      (long long)(uintptr_t)zmid_out, (long long)(uintptr_t)net_cost,
+                                      (long long)(uintptr_t)st, g->dp_policy, g->flow_max, hy.active ? 1 : 0,
+                                      g->hyb_t1, g->hyb_t2, g->full_dirty ? 1 : 0, (long long)g_scratch_gen};
+        std::vector<long long> mir;
+        mir.reserve((size_t)B * 12 + 1);
+        for (int b = 0; b <= B; b++) mir.push_back(c.h_off[b]);
+        for (int b = 0; b < B; b++) {
+            mir.push_back(c.h_nlarge[b]); mir.push_back(c.h_maxm[b]); mir.push_back(c.h_ntwo[b]);
+            mir.push_back(c.h_n9[b]); mir.push_back(c.h_segb[b]);
+            for (int k = 0; k < 5; k++) mir.push_back(c.h_lsplit[5 * b + k]);
+        }
+        if (hy.active)
+            for (int x : hy.boff) mir.push_back(x);
+        if (rg.exec && key == rg.key && mir == rg.mirror) {
+            FGR_CHECK_CUDA(g, cudaGraphLaunch(rg.exec, st));
+            g->full_dirty = false;
+            g->stats.kernel_launches += rg.launches;
+            g->stats.graph_mode = 2;
+            return FGR_OK;
+        }
+        if (key == rg.seen_key && mir == rg.seen_mirror) {
+            // second call with these inputs (every scratch buffer is sized): capture the loop on the
+            // grid's private stream (the caller's may be the legacy stream, which cannot be captured),
+            // then launch the graph on the caller's stream
+            if (rg.exec) { cudaGraphExecDestroy(rg.exec); rg.exec = nullptr; }
+            const bool fd = g->full_dirty;
+            const long long l0 = g->stats.kernel_launches;
+            cudaGraph_t graph = nullptr;
+            cudaError_t e2 = cudaSuccess;
+            if (!rg.cap) e2 = cudaStreamCreateWithFlags(&rg.cap, cudaStreamNonBlocking);
+            if (e2 == cudaSuccess) e2 = cudaStreamBeginCapture(rg.cap, cudaStreamCaptureModeThreadLocal);
+            if (e2 == cudaSuccess) {
+                const cudaError_t el = loop(rg.cap);
+                e2 = cudaStreamEndCapture(rg.cap, &graph);
+                if (el != cudaSuccess) e2 = el;
+            }
+            if (e2 == cudaSuccess && g_scratch_gen == (unsigned long long)key[key.size() - 1])
+                e2 = cudaGraphInstantiate(&rg.exec, graph, 0);
+            else if (e2 == cudaSuccess)
+                e2 = cudaErrorStreamCaptureInvalidated;   // a buffer moved during capture: not reusable
+            if (graph) cudaGraphDestroy(graph);
+            if (e2 == cudaSuccess) {
+                rg.key = key;
+                rg.mirror = mir;
+                rg.launches = g->stats.kernel_launches - l0;
+                FGR_CHECK_CUDA(g, cudaGraphLaunch(rg.exec, st));
+                g->stats.graph_mode = 1;
+                return FGR_OK;
+            }
+            // capture failed: clear the sticky error state of this attempt and run the loop directly
+            // (the reason stays readable through fgr_last_error; the call itself succeeds)
+            if (rg.exec) { cudaGraphExecDestroy(rg.exec); rg.exec = nullptr; }
+            (void)cudaGetLastError();
+            fgr_set_error(FGR_OK, "batch-loop graph capture failed (%s); direct launches from now on",
+                          cudaGetErrorString(e2));
+            g->full_dirty = fd;
+            g->stats.kernel_launches = l0;
+            rg.use = false;
+        }
+        FGR_CHECK_CUDA(g, loop(st));
+        key.back() = (long long)g_scratch_gen;   // buffers the direct run sized are in place for the next call
+        rg.seen_key = key;
+        rg.seen_mirror = mir;
         return FGR_OK;
     }
     // ---- multi-GPU: split each batch by tree edges, exchange route records, commit everywhere.

@@ -27,7 +27,7 @@ EXPORTS = ["fgr_last_error", "fgr_version", "fgr_cost_table", "fgr_grid_create",
            "fgr_grid_set_demand", "fgr_grid_get_demand", "fgr_plan", "fgr_route_batch", "fgr_route_all",
            "fgr_comm_unique_id", "fgr_comm_init", "fgr_run_host", "fgr_get_stats", "fgr_profile_enable",
            "fgr_profile_read", "fgr_split_batch", "fgr_set_pattern", "fgr_route_batch_ex", "fgr_route_all_ex",
-           "fgr_run_host_ex", "fgr_overflow", "fgr_task_graph", "fgr_set_dp_policy", "fgr_set_exchange"]
+           "fgr_run_host_ex", "fgr_overflow", "fgr_task_graph", "fgr_set_dp_policy", "fgr_set_exchange", "fgr_set_graph"]
 PROF_CLASSES = ["refresh", "dp_small", "dp_large", "commit", "plan_preprocess", "plan_sort", "plan_color",
                 "plan_other", "exchange", "hybrid"]
 # the paper's FastGRH selection window: hybrid L+Z on two-pin HPWL in [100, 500]
@@ -56,7 +56,8 @@ class fgr_nets(ctypes.Structure):
 class fgr_stats(ctypes.Structure):
     _fields_ = [("refresh_segments", ctypes.c_int64), ("refresh_bytes", ctypes.c_int64), ("dp_nets", ctypes.c_int64),
                 ("dp_edges", ctypes.c_int64), ("kernel_launches", ctypes.c_int64), ("num_batches", ctypes.c_int32),
-                ("world", ctypes.c_int32), ("rank", ctypes.c_int32), ("exchanged_batches", ctypes.c_int32)]
+                ("world", ctypes.c_int32), ("rank", ctypes.c_int32), ("exchanged_batches", ctypes.c_int32),
+                ("graph_mode", ctypes.c_int32), ("reserved", ctypes.c_int32)]
 
 
 def lib():
@@ -87,6 +88,7 @@ def lib():
             "fgr_profile_read": ([P, P, P], S),
             "fgr_split_batch": ([I, I, P, I, I, I, P], S),
             "fgr_set_exchange": ([P, I, I], S),
+            "fgr_set_graph": ([P, I], S),
             "fgr_set_pattern": ([P, I, I], S),
             "fgr_set_dp_policy": ([P, I, I], S),
             "fgr_route_batch_ex": ([P, P, P, I, P, P, P, P], S),
@@ -269,6 +271,11 @@ def fgr_split_batch(count, nlarge, rank, world, edge_prefix=None, split_min=0):
 
 def fgr_set_exchange(h, split_min=2048, emulate_world=0):
     _check(lib().fgr_set_exchange(h, int(split_min), int(emulate_world)))
+
+
+def fgr_set_graph(h, on=True):
+    """Replay the single-GPU batch loop as a CUDA Graph (default on); routes are identical either way."""
+    _check(lib().fgr_set_graph(h, 1 if on else 0))
 
 
 def fgr_profile_enable(h, enable=True):
