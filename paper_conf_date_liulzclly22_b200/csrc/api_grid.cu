@@ -29,6 +29,32 @@ fgr_status fgr_cuda_fail(fgr_grid* g, cudaError_t e, const char* where) {
 
 unsigned long long g_scratch_gen = 0;
 
+void fgr_mirrors_free(PlanCache& c) {
+    int* ip[6] = {c.h_off, c.h_nlarge, c.h_maxm, c.h_ntwo, c.h_n9, c.h_lsplit};
+    for (int* q : ip)
+        if (q) cudaFreeHost(q);
+    if (c.h_segb) cudaFreeHost(c.h_segb);
+    c.h_off = c.h_nlarge = c.h_maxm = c.h_ntwo = c.h_n9 = c.h_lsplit = nullptr;
+    c.h_segb = nullptr;
+    c.cap = 0;
+}
+
+cudaError_t fgr_mirrors_reserve(PlanCache& c, int B) {
+    if (c.cap >= B + 1) return cudaSuccess;
+    fgr_mirrors_free(c);
+    const int cap = B + 1;
+    cudaError_t e = cudaMallocHost(&c.h_off, sizeof(int) * cap);
+    if (e == cudaSuccess) e = cudaMallocHost(&c.h_nlarge, sizeof(int) * cap);
+    if (e == cudaSuccess) e = cudaMallocHost(&c.h_maxm, sizeof(int) * cap);
+    if (e == cudaSuccess) e = cudaMallocHost(&c.h_ntwo, sizeof(int) * cap);
+    if (e == cudaSuccess) e = cudaMallocHost(&c.h_n9, sizeof(int) * cap);
+    if (e == cudaSuccess) e = cudaMallocHost(&c.h_lsplit, sizeof(int) * 5 * cap);
+    if (e == cudaSuccess) e = cudaMallocHost(&c.h_segb, sizeof(long long) * cap);
+    if (e != cudaSuccess) { fgr_mirrors_free(c); return e; }
+    c.cap = cap;
+    return cudaSuccess;
+}
+
 void* fgr_scratch(Scratch& s, size_t bytes, cudaError_t* err) {
     *err = cudaSuccess;
     if (bytes <= s.bytes && s.p) return s.p;
@@ -255,13 +281,7 @@ extern "C" FGR_API fgr_status fgr_grid_destroy(fgr_grid* g) {
         if (g->ev_join[i]) cudaEventDestroy(g->ev_join[i]);
     }
     if (g->ev_fork) cudaEventDestroy(g->ev_fork);
-    free(g->cache.h_off);
-    free(g->cache.h_nlarge);
-    free(g->cache.h_maxm);
-    free(g->cache.h_segb);
-    free(g->cache.h_ntwo);
-    free(g->cache.h_n9);
-    free(g->cache.h_lsplit);
+    fgr_mirrors_free(g->cache);
     delete g;
     return FGR_OK;
 }

@@ -429,6 +429,7 @@ k_dp_tree(GridView g, NetsView nv, const int32_t* __restrict__ list, int count, 
         TMARK(1);
         // ---- P1: leg gathers, 4 tasks per edge:
         //   0: leg 1 H on row y_v, 1: leg 1 V on col x_v, 2: leg 2 V on col x_u, 3: leg 2 H on row y_u
+#pragma unroll 4
         for (int task = tid; task < 4 * (m - 1); task += NT) {
             const int v = 1 + (task >> 2), type = task & 3;
             const int et = sET[v];

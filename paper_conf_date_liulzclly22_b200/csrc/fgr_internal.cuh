@@ -246,6 +246,9 @@ enum { PROF_REFRESH = 0, PROF_DP_SMALL, PROF_DP_LARGE, PROF_COMMIT, PROF_PRE, PR
 
 // ------------------------------------------------------------------ host helpers
 fgr_status fgr_set_error(fgr_status s, const char* fmt, ...);
+// host mirrors of the plan's per-batch sizes, pinned (async D2H copies); capacity >= B + 1 batches
+cudaError_t fgr_mirrors_reserve(PlanCache& c, int B);
+void fgr_mirrors_free(PlanCache& c);
 fgr_status fgr_cuda_fail(fgr_grid* g, cudaError_t e, const char* where);
 void* fgr_scratch(Scratch& s, size_t bytes, cudaError_t* err);
 

@@ -635,26 +635,16 @@ extern "C" FGR_API fgr_status fgr_plan(fgr_grid* g, const fgr_nets* nets, int32_
     FGR_CHECK_CUDA(g, cudaMemcpyAsync(&B, counters + 4, sizeof(int), cudaMemcpyDeviceToHost, st));
     FGR_CHECK_CUDA(g, cudaStreamSynchronize(st));  // sync 2 of 2
     PlanCache& c = g->cache;
-    if (c.cap < B + 1) {
-        free(c.h_off); free(c.h_nlarge); free(c.h_maxm); free(c.h_segb); free(c.h_ntwo); free(c.h_n9);
-        free(c.h_lsplit);
-        c.cap = B + 1;
-        c.h_lsplit = (int*)malloc(sizeof(int) * 5 * c.cap);
-        c.h_off = (int*)malloc(sizeof(int) * c.cap);
-        c.h_nlarge = (int*)malloc(sizeof(int) * c.cap);
-        c.h_maxm = (int*)malloc(sizeof(int) * c.cap);
-        c.h_segb = (long long*)malloc(sizeof(long long) * c.cap);
-        c.h_ntwo = (int*)malloc(sizeof(int) * c.cap);
-        c.h_n9 = (int*)malloc(sizeof(int) * c.cap);
-    }
-    if (B > 0) {
-        FGR_CHECK_CUDA(g, cudaMemcpy(c.h_off, batch_offset, sizeof(int) * (B + 1), cudaMemcpyDeviceToHost));
-        FGR_CHECK_CUDA(g, cudaMemcpy(c.h_nlarge, d_nlarge, sizeof(int) * B, cudaMemcpyDeviceToHost));
-        FGR_CHECK_CUDA(g, cudaMemcpy(c.h_maxm, d_maxm, sizeof(int) * B, cudaMemcpyDeviceToHost));
-        FGR_CHECK_CUDA(g, cudaMemcpy(c.h_ntwo, d_ntwo, sizeof(int) * B, cudaMemcpyDeviceToHost));
-        FGR_CHECK_CUDA(g, cudaMemcpy(c.h_n9, d_n9, sizeof(int) * B, cudaMemcpyDeviceToHost));
-        FGR_CHECK_CUDA(g, cudaMemcpy(c.h_lsplit, d_ls, sizeof(int) * 5 * B, cudaMemcpyDeviceToHost));
-        FGR_CHECK_CUDA(g, cudaMemcpy(c.h_segb, segsum, sizeof(long long) * B, cudaMemcpyDeviceToHost));
+    FGR_CHECK_CUDA(g, fgr_mirrors_reserve(c, B));
+    if (B > 0) {   // pinned mirrors: the copies are queued, one synchronisation
+        FGR_CHECK_CUDA(g, cudaMemcpyAsync(c.h_off, batch_offset, sizeof(int) * (B + 1), cudaMemcpyDeviceToHost, st));
+        FGR_CHECK_CUDA(g, cudaMemcpyAsync(c.h_nlarge, d_nlarge, sizeof(int) * B, cudaMemcpyDeviceToHost, st));
+        FGR_CHECK_CUDA(g, cudaMemcpyAsync(c.h_maxm, d_maxm, sizeof(int) * B, cudaMemcpyDeviceToHost, st));
+        FGR_CHECK_CUDA(g, cudaMemcpyAsync(c.h_ntwo, d_ntwo, sizeof(int) * B, cudaMemcpyDeviceToHost, st));
+        FGR_CHECK_CUDA(g, cudaMemcpyAsync(c.h_n9, d_n9, sizeof(int) * B, cudaMemcpyDeviceToHost, st));
+        FGR_CHECK_CUDA(g, cudaMemcpyAsync(c.h_lsplit, d_ls, sizeof(int) * 5 * B, cudaMemcpyDeviceToHost, st));
+        FGR_CHECK_CUDA(g, cudaMemcpyAsync(c.h_segb, segsum, sizeof(long long) * B, cudaMemcpyDeviceToHost, st));
+        FGR_CHECK_CUDA(g, cudaStreamSynchronize(st));
     }
     c.valid = true;
     c.prep_valid = false;

@@ -272,18 +272,7 @@ static fgr_status batch_info(fgr_grid* g, const fgr_nets* nets, const int32_t* o
     int* d_n9 = d_n2 + B;
     int* d_ls = d_n9 + B;
     FGR_CHECK_CUDA(g, cudaMemsetAsync(p, 0, (size_t)B * 44, st));
-    if (c.cap < B + 1) {
-        free(c.h_off); free(c.h_nlarge); free(c.h_maxm); free(c.h_segb); free(c.h_ntwo); free(c.h_n9);
-        free(c.h_lsplit);
-        c.cap = B + 1;
-        c.h_lsplit = (int*)malloc(sizeof(int) * 5 * c.cap);
-        c.h_n9 = (int*)malloc(sizeof(int) * c.cap);
-        c.h_off = (int*)malloc(sizeof(int) * c.cap);
-        c.h_nlarge = (int*)malloc(sizeof(int) * c.cap);
-        c.h_maxm = (int*)malloc(sizeof(int) * c.cap);
-        c.h_segb = (long long*)malloc(sizeof(long long) * c.cap);
-        c.h_ntwo = (int*)malloc(sizeof(int) * c.cap);
-    }
+    FGR_CHECK_CUDA(g, fgr_mirrors_reserve(c, B));
     FGR_CHECK_CUDA(g, cudaMemcpyAsync(c.h_off, batch_offset, sizeof(int) * (B + 1), cudaMemcpyDeviceToHost, st));
     FGR_CHECK_CUDA(g, cudaStreamSynchronize(st));
     const int nb = B > 0 ? c.h_off[B] : 0;

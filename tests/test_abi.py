@@ -73,3 +73,11 @@ def test_no_cpu_fallback_without_gpu():
         pytest.skip("GPU present")
     with pytest.raises(RuntimeError):
         F.Router(gen.make_config("tiny", num_nets=5))
+
+
+def test_setters_reject_null_grid():
+    """Host-only setters validate their grid argument without a device (FGR_ERR_INVALID)."""
+    lib = F.lib()
+    assert lib.fgr_set_graph(None, 1) == F.FGR_ERR_INVALID
+    assert lib.fgr_set_exchange(None, 16, 0) == F.FGR_ERR_INVALID
+    assert lib.fgr_set_dp_policy(None, 0, 64) == F.FGR_ERR_INVALID

@@ -70,7 +70,7 @@ if os.path.exists(p):
         agg[k][0] += 1
         agg[k][1] += m.get("dram__bytes_read.sum", 0) + m.get("dram__bytes_write.sum", 0)
         agg[k][2] += m.get("gpu__time_duration.sum", 0)
-    cls = {"k_dp_large": "dp_large", "k_dp_walk": "dp_small", "k_dp_two": "dp_two", "k_refresh": "refresh",
+    cls = {"k_dp_tree": "dp_large", "k_dp_large": "dp_large_heavy", "k_dp_walk": "dp_small", "k_dp_two": "dp_two", "k_refresh": "refresh",
            "k_color": "plan_color", "k_dp_flow": "dp_flow"}
     out_md.append("## DRAM traffic per launch over one t9 step (ncu dram__bytes_read.sum + write.sum)\n")
     out_md.append("| kernel | launches | avg bytes/launch | avg us/launch (serialised) |\n|---|---|---|---|")
