@@ -207,15 +207,17 @@ __device__ __forceinline__ int refresh_chunk(const GridView& g, const DirView& d
         cur = nxt;
         q = q2;
     }
+    // hand-off to the line's last finisher: release this warp's P/ST stores, acquire the others'
+    // (acq_rel at GPU scope: the tasks of one line run in different CTAs)
     int last = 0;
+    __syncwarp();
     if (lane == 0) {
-        __threadfence();
-        const unsigned old = atomicAdd(&g.linedone[lidx], 1u);
+        unsigned old;
+        asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], 1;" : "=r"(old) : "l"(&g.linedone[lidx]) : "memory");
         last = (old + 1 == (unsigned)nd);
     }
     last = __shfl_sync(0xffffffffu, last, 0);
     if (last) {
-        __threadfence();
         rebase_line<W>(d, line);
         uint8_t* fw = g.dseg + d.seg_base + (size_t)line * d.nseg;
         for (int sg = lane; sg < d.nseg; sg += 32) fw[sg] = 0;
