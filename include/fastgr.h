@@ -79,7 +79,8 @@ typedef struct {
 FGR_API fgr_status fgr_cost_table(const fgr_grid_desc* desc, int64_t* table);
 
 /* Allocates the grid on `device` (demand = 0).  Errors: INVALID (desc), RANGE
- * ((len_cost + max W) * max(nx,ny) >= 2^32), OOM, CUDA.  Caller owns *out. */
+ * ((len_cost + max W) * max(nx,ny) >= 2^31 - 1, or the via costs sum to >= 2^24),
+ * OOM, CUDA.  Caller owns *out. */
 FGR_API fgr_status fgr_grid_create(const fgr_grid_desc* desc, int device, void* stream, fgr_grid** out);
 FGR_API fgr_status fgr_grid_destroy(fgr_grid* grid);
 
@@ -123,8 +124,11 @@ typedef struct {
  *   batch_offset [num_nets+1] DEVICE out: batch b = order[batch_offset[b] .. batch_offset[b+1])
  *   num_batches               HOST out
  * Errors: INVALID (malformed nets: the message names the first bad net), RANGE
- * (a net's worst-case cost could reach 2^31, or a net too large for the
- * on-chip DP tables), OOM, CUDA.  Synchronises `stream`.
+ * (a net's worst-case cost could reach 2^31, or a net of more than 65535 nodes),
+ * OOM, CUDA.  Synchronises `stream`.  The plan (host batch sizes, the tree
+ * decompositions of the large nets, the hybrid tables, a captured batch-loop
+ * graph) is cached by the identity of the nets and output buffers: after
+ * rewriting the nets' arrays in place, call fgr_plan again before routing.
  */
 FGR_API fgr_status fgr_plan(fgr_grid* grid, const fgr_nets* nets, int32_t* batch_of_net, int32_t* order,
                             int32_t* batch_offset, int32_t* num_batches, void* stream);

@@ -268,6 +268,9 @@ static cudaError_t launch_t(fgr_grid* g, cudaStream_t st, bool full, int blocks)
 }
 
 // One warp per (line, chunk) task; grid capped at 8 CTAs per SM (grid-stride beyond).
+// max_tasks (an upper bound on the segments the last batch dirtied) does not size the grid: the
+// grid covers every (line, chunk) task and clean lines exit after one flag load, which measured
+// faster than a bound-sized grid over a commit-built list.
 cudaError_t fgr_launch_refresh_sized(fgr_grid* g, cudaStream_t st, bool full, long long max_tasks) {
     (void)max_tasks;
     const GridView& v = g->view;
