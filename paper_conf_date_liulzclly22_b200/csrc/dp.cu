@@ -14,11 +14,17 @@
 // (S6) with dirty-segment marking for the next cost refresh.
 //
 // B200 mapping.  The layer count LT is a template parameter (every per-layer
-// loop is unrolled exactly).  A "group" of LT lanes evaluates one node: lane l
-// owns layer l of the node's vectors (F rows, B, E — the L parallel computation
-// flows of P:L754-756).  A warp holds G = min(4, 32/LT) groups:
-//   * k_dp_large: nets with > 32 nodes, one 256-thread CTA per net, level by
-//     level, 8*G nodes of a level in flight.
+// loop is unrolled exactly).  This file holds:
+//   * k_dp_two: 2-node nets (half of all nets), one thread per net, the whole DP
+//     in registers;
+//   * k_dp_large: the round-1 kernel for nets of 65..~1.3k nodes, one 512-thread
+//     CTA per net, heavy-path product form (the root path walked with transfer
+//     matrices precomputed by helper warps, other paths by path walks) — selected
+//     only by FGR_DP_HEAVY; the default large-net kernel is k_dp_tree (dp_tree.cu);
+//   * k_commit_records: the S6 commit from exchanged route records (multi-GPU);
+//   * launch_lt: the per-batch launcher (size classes on side streams, the
+//     kernel of each large-net bucket by fgr_set_dp_policy, one grid-wide commit
+//     of the tree-kernel nets after the join).
 // All prefix gathers of a net are issued up front (costs are fixed during the
 // DP); the per-node tables live in shared memory; each min-plus step is a DPX
 // VIADDMNMX (sat_add).  Tie-breaks follow reading R11 exactly.
