@@ -1321,7 +1321,13 @@ cudaError_t launch_lt(fgr_grid* g, cudaStream_t st, const NetsView& nv, const in
             e = fgr_launch_hld(g, su, nv, l, n, un.cap, os, commit, prep.hld, wsb ? wsb + wsoff[ui] : nullptr);
             if (e != cudaSuccess) return e;
         } else if (lk == 3) {
-            e = fgr_launch_tree(g, su, nv, l, n, un.cap, os, false, prep.hld);   // committed after the join
+            uint32_t* legs = nullptr;   // nets above 512 nodes: leg costs gathered by many SMs first
+            if (un.cap > 512) {
+                legs = (uint32_t*)fgr_scratch(g->s_tlegs, (size_t)n * 2 * un.cap * LT * 4 + 256, &e);
+                if (e != cudaSuccess) return e;
+                if ((e = fgr_launch_tree_legs(g, su, nv, l, n, un.cap, legs)) != cudaSuccess) return e;
+            }
+            e = fgr_launch_tree(g, su, nv, l, n, un.cap, os, false, prep.hld, legs, un.cap);   // committed after the join
             if (tree_n == 0) { tree_off = un.off; tree_cap = un.cap; }
             tree_n += n;
             if (e != cudaSuccess) return e;

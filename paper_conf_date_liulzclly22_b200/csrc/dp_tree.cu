@@ -324,7 +324,8 @@ __device__ __forceinline__ void tree_node_argmin(const GridView& g, const HybVie
 
 template <int LT, int NT, int CAP>
 __global__ void __launch_bounds__(NT, (NT >= 384 ? 1 : (NT >= 256 ? 2 : 4)))
-k_dp_tree(GridView g, NetsView nv, const int32_t* __restrict__ list, int count, Out o, HldPrep hp, HybView hy) {
+k_dp_tree(GridView g, NetsView nv, const int32_t* __restrict__ list, int count, Out o, HldPrep hp, HybView hy,
+          const uint32_t* __restrict__ legs, int legs_maxm) {
     using T = TL<LT, NT, CAP>;
     constexpr int NS = T::NS, GPW = T::GPW, NW = T::NW;
     extern __shared__ __align__(16) unsigned char sm[];
@@ -410,7 +411,7 @@ k_dp_tree(GridView g, NetsView nv, const int32_t* __restrict__ list, int count, 
             sPN[i] = hp.pn[a0 + i];
             sQ[i] = 0xFFFF;
             if (i < np) { sLF[i] = hp.lf[a0 + i]; sPO[i] = hp.po[a0 + i]; }
-            if (et == TE_SH || et == TE_SV) {   // the off-direction layers of a straight edge stay impossible (R6, R7)
+            if (!legs && (et == TE_SH || et == TE_SV)) {   // the off-direction layers of a straight edge stay impossible (R6, R7)
 #pragma unroll
                 for (int l = 0; l < LT; l++) sLG1[i * LT + l] = FGR_INF;
             }
@@ -427,37 +428,48 @@ k_dp_tree(GridView g, NetsView nv, const int32_t* __restrict__ list, int count, 
         if (!waited) { pdl_wait(); waited = true; }   // the refresh must be complete before the gathers
         cta_sync();
         TMARK(1);
-        // ---- P1: leg gathers, 4 tasks per edge:
-        //   0: leg 1 H on row y_v, 1: leg 1 V on col x_v, 2: leg 2 V on col x_u, 3: leg 2 H on row y_u
+        // ---- P1: leg costs.  Nets above 512 nodes: the rows k_tree_legs gathered with many SMs (LG1 |
+        // LG2 blocks of legs_maxm rows); otherwise gathered here, 4 tasks per edge.
+        if (legs) {
+            const uint32_t* L1 = legs + (size_t)idx * 2 * legs_maxm * LT;
+            const uint32_t* L2 = L1 + (size_t)legs_maxm * LT;
+            for (int i = LT + tid; i < m * LT; i += NT) {
+                sLG1[i] = __ldcg(L1 + i);
+                sLG2[i] = __ldcg(L2 + i);
+            }
+        } else {
+            // ---- P1: leg gathers, 4 tasks per edge:
+            //   0: leg 1 H on row y_v, 1: leg 1 V on col x_v, 2: leg 2 V on col x_u, 3: leg 2 H on row y_u
 #pragma unroll 4
-        for (int task = tid; task < 4 * (m - 1); task += NT) {
-            const int v = 1 + (task >> 2), type = task & 3;
-            const int et = sET[v];
-            if (et == TE_HYB || (et == TE_SH && type != 0) || (et == TE_SV && type != 1)) continue;
-            const int u = sPAR[v];
-            const int xv = nv.x[a0 + v], yv = nv.y[a0 + v], xu = nv.x[a0 + u], yu = nv.y[a0 + u];
-            const bool H = type == 0 || type == 3;
-            const int line = type == 0 ? yv : type == 1 ? xv : type == 2 ? xu : yu;
-            const int pa = H ? min(xv, xu) : min(yv, yu);
-            const int pb = H ? max(xv, xu) : max(yv, yu);
-            const uint32_t* P = H ? g.h.P : g.v.P;
-            const uint32_t* SB = H ? g.h.SB : g.v.SB;
-            const int len = H ? g.h.len : g.v.len, W = H ? g.h.W : g.v.W, nseg = H ? g.h.nseg : g.v.nseg;
-            const int cnt = H ? g.h.cnt : g.v.cnt;
-            uint32_t* dst = (type >= 2 ? sLG2 : sLG1) + v * LT;
-            const uint8_t* los = s_los[H ? 0 : 1];
-            const size_t ia = ((size_t)line * len + pa) * W, ib = ((size_t)line * len + pb) * W;
-            const size_t sa = ((size_t)line * nseg + (pa >> FGR_SEG_SHIFT)) * W;
-            const size_t sb = ((size_t)line * nseg + (pb >> FGR_SEG_SHIFT)) * W;
-            for (int q = 0; q < (W >> 2); q++) {
-                const uint4 Pa = __ldg(reinterpret_cast<const uint4*>(P + ia) + q);
-                const uint4 Pb = __ldg(reinterpret_cast<const uint4*>(P + ib) + q);
-                const uint4 Sa = __ldg(reinterpret_cast<const uint4*>(SB + sa) + q);
-                const uint4 Sb = __ldg(reinterpret_cast<const uint4*>(SB + sb) + q);
-                if (4 * q + 0 < cnt) dst[los[4 * q + 0]] = (Sb.x + Pb.x) - (Sa.x + Pa.x);
-                if (4 * q + 1 < cnt) dst[los[4 * q + 1]] = (Sb.y + Pb.y) - (Sa.y + Pa.y);
-                if (4 * q + 2 < cnt) dst[los[4 * q + 2]] = (Sb.z + Pb.z) - (Sa.z + Pa.z);
-                if (4 * q + 3 < cnt) dst[los[4 * q + 3]] = (Sb.w + Pb.w) - (Sa.w + Pa.w);
+            for (int task = tid; task < 4 * (m - 1); task += NT) {
+                const int v = 1 + (task >> 2), type = task & 3;
+                const int et = sET[v];
+                if (et == TE_HYB || (et == TE_SH && type != 0) || (et == TE_SV && type != 1)) continue;
+                const int u = sPAR[v];
+                const int xv = nv.x[a0 + v], yv = nv.y[a0 + v], xu = nv.x[a0 + u], yu = nv.y[a0 + u];
+                const bool H = type == 0 || type == 3;
+                const int line = type == 0 ? yv : type == 1 ? xv : type == 2 ? xu : yu;
+                const int pa = H ? min(xv, xu) : min(yv, yu);
+                const int pb = H ? max(xv, xu) : max(yv, yu);
+                const uint32_t* P = H ? g.h.P : g.v.P;
+                const uint32_t* SB = H ? g.h.SB : g.v.SB;
+                const int len = H ? g.h.len : g.v.len, W = H ? g.h.W : g.v.W, nseg = H ? g.h.nseg : g.v.nseg;
+                const int cnt = H ? g.h.cnt : g.v.cnt;
+                uint32_t* dst = (type >= 2 ? sLG2 : sLG1) + v * LT;
+                const uint8_t* los = s_los[H ? 0 : 1];
+                const size_t ia = ((size_t)line * len + pa) * W, ib = ((size_t)line * len + pb) * W;
+                const size_t sa = ((size_t)line * nseg + (pa >> FGR_SEG_SHIFT)) * W;
+                const size_t sb = ((size_t)line * nseg + (pb >> FGR_SEG_SHIFT)) * W;
+                for (int q = 0; q < (W >> 2); q++) {
+                    const uint4 Pa = __ldg(reinterpret_cast<const uint4*>(P + ia) + q);
+                    const uint4 Pb = __ldg(reinterpret_cast<const uint4*>(P + ib) + q);
+                    const uint4 Sa = __ldg(reinterpret_cast<const uint4*>(SB + sa) + q);
+                    const uint4 Sb = __ldg(reinterpret_cast<const uint4*>(SB + sb) + q);
+                    if (4 * q + 0 < cnt) dst[los[4 * q + 0]] = (Sb.x + Pb.x) - (Sa.x + Pa.x);
+                    if (4 * q + 1 < cnt) dst[los[4 * q + 1]] = (Sb.y + Pb.y) - (Sa.y + Pa.y);
+                    if (4 * q + 2 < cnt) dst[los[4 * q + 2]] = (Sb.z + Pb.z) - (Sa.z + Pa.z);
+                    if (4 * q + 3 < cnt) dst[los[4 * q + 3]] = (Sb.w + Pb.w) - (Sa.w + Pa.w);
+                }
             }
         }
         cta_sync();
@@ -727,6 +739,65 @@ k_dp_tree(GridView g, NetsView nv, const int32_t* __restrict__ list, int count, 
     }
 }
 
+// P1 for the tree-kernel nets above 512 nodes, done by many SMs: every edge's leg costs, one task
+// per thread (4 tasks per edge as in the kernel's own tables: 0 leg 1 H on row y_v, 1 leg 1 V on
+// col x_v, 2 leg 2 V on col x_u, 3 leg 2 H on row y_u), written as rows LG1 [maxm][LT] | LG2
+// [maxm][LT] per net, so that a lone large net does not pull its ~4000 prefix gathers through one
+// SM.  Straight edges get INF on the layers of the other direction (R6, R7); hybrid edges use
+// their transfer matrices instead.
+template <int LT>
+__global__ void __launch_bounds__(256) k_tree_legs(GridView g, NetsView nv, const int32_t* __restrict__ list, int count,
+                                                   int chunks, int maxm, uint32_t* __restrict__ out, HybView hy) {
+    pdl_trigger();   // the tree kernel may start its topology prologue
+    pdl_wait();      // the refresh must be complete
+    const int idx = blockIdx.x / chunks;
+    if (idx >= count) return;
+    const int net = list[idx];
+    const int a0 = nv.off[net], m = nv.off[net + 1] - a0;
+    const int task = (blockIdx.x % chunks) * 256 + threadIdx.x;
+    if (task >= 4 * (m - 1)) return;
+    const int hnet = hy.net ? hy.net[net] : -1;
+    uint32_t* const L1 = out + (size_t)idx * 2 * maxm * LT;
+    uint32_t* const L2 = L1 + (size_t)maxm * LT;
+    const int v = 1 + (task >> 2), type = task & 3;
+    const int u = nv.par[a0 + v];
+    const int xv = nv.x[a0 + v], yv = nv.y[a0 + v], xu = nv.x[a0 + u], yu = nv.y[a0 + u];
+    const int et = (yv == yu) ? TE_SH : (xv == xu) ? TE_SV : ((hnet >= 0 && hy.slot[a0 + v] >= 0) ? TE_HYB : TE_BENT);
+    if (et == TE_HYB || (et == TE_SH && type != 0) || (et == TE_SV && type != 1)) return;
+    const bool H = type == 0 || type == 3;
+    const int line = type == 0 ? yv : type == 1 ? xv : type == 2 ? xu : yu;
+    const int pa = H ? min(xv, xu) : min(yv, yu);
+    const int pb = H ? max(xv, xu) : max(yv, yu);
+    const uint32_t* P = H ? g.h.P : g.v.P;
+    const uint32_t* SB = H ? g.h.SB : g.v.SB;
+    const int len = H ? g.h.len : g.v.len, W = H ? g.h.W : g.v.W, nseg = H ? g.h.nseg : g.v.nseg;
+    const int cnt = H ? g.h.cnt : g.v.cnt;
+    uint32_t* dst = (type >= 2 ? L2 : L1) + (size_t)v * LT;
+    const uint8_t* los = g.layer_of_slot[H ? 0 : 1];
+    if (et != TE_BENT) {   // straight: the other direction's layers are impossible
+        const uint8_t* lo2 = g.layer_of_slot[H ? 1 : 0];
+        const int c2 = H ? g.v.cnt : g.h.cnt;
+        for (int k2 = 0; k2 < c2; k2++) dst[lo2[k2]] = FGR_INF;
+    }
+    const size_t ia = ((size_t)line * len + pa) * W, ib = ((size_t)line * len + pb) * W;
+    const size_t sa = ((size_t)line * nseg + (pa >> FGR_SEG_SHIFT)) * W;
+    const size_t sb = ((size_t)line * nseg + (pb >> FGR_SEG_SHIFT)) * W;
+    const bool oneseg = (pa >> FGR_SEG_SHIFT) == (pb >> FGR_SEG_SHIFT);   // segment bases cancel
+    for (int q = 0; q < (W >> 2); q++) {
+        const uint4 Pa = __ldg(reinterpret_cast<const uint4*>(P + ia) + q);
+        const uint4 Pb = __ldg(reinterpret_cast<const uint4*>(P + ib) + q);
+        uint4 Sa = make_uint4(0, 0, 0, 0), Sb = make_uint4(0, 0, 0, 0);
+        if (!oneseg) {
+            Sa = __ldg(reinterpret_cast<const uint4*>(SB + sa) + q);
+            Sb = __ldg(reinterpret_cast<const uint4*>(SB + sb) + q);
+        }
+        if (4 * q + 0 < cnt) dst[los[4 * q + 0]] = (Sb.x + Pb.x) - (Sa.x + Pa.x);
+        if (4 * q + 1 < cnt) dst[los[4 * q + 1]] = (Sb.y + Pb.y) - (Sa.y + Pa.y);
+        if (4 * q + 2 < cnt) dst[los[4 * q + 2]] = (Sb.z + Pb.z) - (Sa.z + Pa.z);
+        if (4 * q + 3 < cnt) dst[los[4 * q + 3]] = (Sb.w + Pb.w) - (Sa.w + Pa.w);
+    }
+}
+
 // S6 for the nets of a tree-kernel launch: one thread per tree edge, blocks of 256 edges.
 __global__ void __launch_bounds__(256) k_commit_nets(GridView g, NetsView nv, const int32_t* __restrict__ list, int count,
                                                      int chunks, Out o, HybView hy) {
@@ -755,7 +826,7 @@ int tree_grid(const fgr_grid* g, int n) {
 
 template <int LT, int NT, int CAP>
 cudaError_t launch_tree_v(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int n, const Out& o,
-                          const HldPrep& hp) {
+                          const HldPrep& hp, const uint32_t* legs, int legs_maxm) {
     using T = TL<LT, NT, CAP>;
     static int configured = 0;
     if (!configured) {
@@ -773,15 +844,31 @@ cudaError_t launch_tree_v(fgr_grid* g, cudaStream_t st, const NetsView& nv, cons
     at[0].val.programmaticStreamSerializationAllowed = 1;
     cfg.attrs = at;
     cfg.numAttrs = 1;
-    return cudaLaunchKernelEx(&cfg, k_dp_tree<LT, NT, CAP>, g->view, nv, list, n, o, hp, g->hy.view());
+    return cudaLaunchKernelEx(&cfg, k_dp_tree<LT, NT, CAP>, g->view, nv, list, n, o, hp, g->hy.view(), legs, legs_maxm);
 }
 
 template <int LT>
 cudaError_t launch_tree_lt(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int n, int maxm,
-                           const Out& o, const HldPrep& hp) {
-    if (maxm <= 128) return launch_tree_v<LT, 128, 128>(g, st, nv, list, n, o, hp);
-    if (maxm <= 512) return launch_tree_v<LT, 256, 512>(g, st, nv, list, n, o, hp);
-    return launch_tree_v<LT, kTreeBigNT, tree_cap512(LT)>(g, st, nv, list, n, o, hp);
+                           const Out& o, const HldPrep& hp, const uint32_t* legs, int legs_maxm) {
+    if (maxm <= 128) return launch_tree_v<LT, 128, 128>(g, st, nv, list, n, o, hp, legs, legs_maxm);
+    if (maxm <= 512) return launch_tree_v<LT, 256, 512>(g, st, nv, list, n, o, hp, legs, legs_maxm);
+    return launch_tree_v<LT, kTreeBigNT, tree_cap512(LT)>(g, st, nv, list, n, o, hp, legs, legs_maxm);
+}
+
+template <int LT>
+cudaError_t launch_legs_lt(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int n, int maxm,
+                           uint32_t* legs) {
+    const int chunks = (4 * (maxm - 1) + 255) / 256;
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)(n * chunks));
+    cfg.blockDim = dim3(256);
+    cfg.stream = st;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, k_tree_legs<LT>, g->view, nv, list, n, chunks, maxm, legs, g->hy.view());
 }
 
 }  // namespace
@@ -796,12 +883,25 @@ int fgr_tree_cap(const fgr_grid* g) {
     }
 }
 
+cudaError_t fgr_launch_tree_legs(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int n, int maxm,
+                                 uint32_t* legs) {
+    if (n <= 0) return cudaSuccess;
+    g->stats.kernel_launches++;
+    switch (g->L) {
+#define FGR_LT(k) case k: return launch_legs_lt<k>(g, st, nv, list, n, maxm, legs);
+        FGR_LT(2) FGR_LT(3) FGR_LT(4) FGR_LT(5) FGR_LT(6) FGR_LT(7) FGR_LT(8) FGR_LT(9) FGR_LT(10) FGR_LT(11)
+        FGR_LT(12) FGR_LT(13) FGR_LT(14) FGR_LT(15) FGR_LT(16)
+#undef FGR_LT
+        default: return cudaErrorInvalidValue;
+    }
+}
+
 cudaError_t fgr_launch_tree(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int n, int maxm,
-                            const Out& o, bool commit, const HldPrep& hp) {
+                            const Out& o, bool commit, const HldPrep& hp, const uint32_t* legs, int legs_maxm) {
     if (n <= 0) return cudaSuccess;
     cudaError_t e;
     switch (g->L) {
-#define FGR_LT(k) case k: e = launch_tree_lt<k>(g, st, nv, list, n, maxm, o, hp); break;
+#define FGR_LT(k) case k: e = launch_tree_lt<k>(g, st, nv, list, n, maxm, o, hp, legs, legs_maxm); break;
         FGR_LT(2) FGR_LT(3) FGR_LT(4) FGR_LT(5) FGR_LT(6) FGR_LT(7) FGR_LT(8) FGR_LT(9) FGR_LT(10) FGR_LT(11)
         FGR_LT(12) FGR_LT(13) FGR_LT(14) FGR_LT(15) FGR_LT(16)
 #undef FGR_LT

@@ -216,6 +216,7 @@ struct fgr_grid {
     Scratch s_hldp;             // k_hld_prep outputs (per stage)
     Scratch s_hldt;             // k_hld_prep temporaries for nets too large for shared memory
     Scratch s_hldw;             // k_dp_hld global workspaces (per CTA) for large nets
+    Scratch s_tlegs;            // leg rows of the tree-kernel nets above 512 nodes (k_tree_legs)
     fgr_stats stats{};
     int max_smem = 0;
     int num_sms = 0;
@@ -288,8 +289,12 @@ cudaError_t fgr_launch_hld_prep(fgr_grid* g, cudaStream_t st, const NetsView& nv
                                 int maxm, uint16_t* hv, uint16_t* cs, uint16_t* cl, uint16_t* pn, uint16_t* po,
                                 uint8_t* pr, int32_t* info, uint8_t* ld, uint16_t* lf);
 // k_dp_tree (dp_tree.cu): nets of FGR_SMALL_NET+1 .. fgr_tree_cap(g) nodes; commit = launch k_commit_nets after it
+// legs: NULL (the kernel gathers its legs) or the rows of fgr_launch_tree_legs (net i at legs + i * 2 * legs_maxm * L)
 cudaError_t fgr_launch_tree(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int n, int maxm,
-                            const Out& o, bool commit, const HldPrep& hp);
+                            const Out& o, bool commit, const HldPrep& hp, const uint32_t* legs, int legs_maxm);
+// k_tree_legs: leg rows of n nets (<= maxm nodes) into legs [n][2][maxm][L], one task per thread on many SMs
+cudaError_t fgr_launch_tree_legs(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int n, int maxm,
+                                 uint32_t* legs);
 // S6 for nets routed without an in-kernel commit: one thread per tree edge (reads seg or the route records)
 cudaError_t fgr_launch_commit_nets(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int n, int maxm,
                                    const Out& o);
