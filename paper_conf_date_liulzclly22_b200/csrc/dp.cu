@@ -1293,7 +1293,9 @@ cudaError_t launch_lt(fgr_grid* g, cudaStream_t st, const NetsView& nv, const in
         for (int ui = 0; ui < nu; ui++) {
             if (units[ui].kind != 0) continue;
             const int lk = large_kind(units[ui].cap);
-            const size_t b = lk == 0 ? fgr_hld_ws_bytes(g, units[ui].n, units[ui].cap) : 0;
+            // k_dp_hld: per-CTA workspaces; tree units above 128 nodes: their nets' leg rows (k_tree_legs)
+            const size_t b = lk == 0 ? fgr_hld_ws_bytes(g, units[ui].n, units[ui].cap)
+                             : (lk == 3 && units[ui].cap > 128) ? (size_t)units[ui].n * 2 * units[ui].cap * LT * 4 : 0;
             wsoff[ui] = wstot;
             wstot += (b + 255) & ~(size_t)255;
         }
@@ -1321,10 +1323,9 @@ cudaError_t launch_lt(fgr_grid* g, cudaStream_t st, const NetsView& nv, const in
             e = fgr_launch_hld(g, su, nv, l, n, un.cap, os, commit, prep.hld, wsb ? wsb + wsoff[ui] : nullptr);
             if (e != cudaSuccess) return e;
         } else if (lk == 3) {
-            uint32_t* legs = nullptr;   // nets above 512 nodes: leg costs gathered by many SMs first
-            if (un.cap > 512) {
-                legs = (uint32_t*)fgr_scratch(g->s_tlegs, (size_t)n * 2 * un.cap * LT * 4 + 256, &e);
-                if (e != cudaSuccess) return e;
+            uint32_t* legs = nullptr;   // nets above 128 nodes: leg costs gathered by many SMs first
+            if (un.cap > 128) {
+                legs = reinterpret_cast<uint32_t*>(wsb + wsoff[ui]);   // this unit's own region (units run concurrently)
                 if ((e = fgr_launch_tree_legs(g, su, nv, l, n, un.cap, legs)) != cudaSuccess) return e;
             }
             e = fgr_launch_tree(g, su, nv, l, n, un.cap, os, false, prep.hld, legs, un.cap);   // committed after the join

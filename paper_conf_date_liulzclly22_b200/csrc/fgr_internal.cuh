@@ -215,8 +215,7 @@ struct fgr_grid {
     Scratch s_prep;
     Scratch s_hldp;             // k_hld_prep outputs (per stage)
     Scratch s_hldt;             // k_hld_prep temporaries for nets too large for shared memory
-    Scratch s_hldw;             // k_dp_hld global workspaces (per CTA) for large nets
-    Scratch s_tlegs;            // leg rows of the tree-kernel nets above 512 nodes (k_tree_legs)
+    Scratch s_hldw;             // per large-net unit: k_dp_hld workspaces (per CTA), k_tree_legs leg rows
     fgr_stats stats{};
     int max_smem = 0;
     int num_sms = 0;
