@@ -14,11 +14,11 @@ ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpuru
 cp gpurun_out/${TAG}_launches.csv /tmp/ncu_$TAG/
 python tools/launch_batches.py gpurun_out/${TAG}_launches.csv > gpurun_out/${TAG}_batches.txt 2>&1
 full() {  # name regex skip [extra ncu args]
-  ncu --set full --import-source on --clock-control none --kernel-name-base demangled -k regex:"$2" -s $3 -c 1 ${4:-} \
+  ncu --set full --import-source on --clock-control none --kernel-name-base mangled -k regex:"$2" -s $3 -c 1 ${4:-} \
       -o /tmp/ncu_$TAG/${TAG}_full_$1 python tools/prof_step.py t9 > /dev/null 2>&1
 }
-full tree384 'k_dp_tree<9, 384' 30
-full tree256 'k_dp_tree<9, 256' 40
+full tree384 'k_dp_treeILi9ELi384' 30
+full tree256 'k_dp_treeILi9ELi256' 40
 full refresh 'k_refresh' 2
 full walk_tail 'k_dp_walk' 150
 full walk_warm 'k_dp_walk' 150 '--cache-control none'
