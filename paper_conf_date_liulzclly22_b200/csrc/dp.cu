@@ -1026,8 +1026,11 @@ __device__ __forceinline__ void leg_cost_col(const DirView& d, int line, int a, 
         if (q < nq) {
             const uint4 Pa = __ldg(reinterpret_cast<const uint4*>(d.P + pa) + q);
             const uint4 Pb = __ldg(reinterpret_cast<const uint4*>(d.P + pb) + q);
-            const uint4 Sa = __ldg(reinterpret_cast<const uint4*>(d.SB + sa) + q);
-            const uint4 Sb = __ldg(reinterpret_cast<const uint4*>(d.SB + sb) + q);
+            uint4 Sa = make_uint4(0, 0, 0, 0), Sb = Sa;
+            if (sa != sb) {   // inside one segment the bases cancel
+                Sa = __ldg(reinterpret_cast<const uint4*>(d.SB + sa) + q);
+                Sb = __ldg(reinterpret_cast<const uint4*>(d.SB + sb) + q);
+            }
             col[(4 * q + 0) * kTwoThreads] = (Sb.x + Pb.x) - (Sa.x + Pa.x);
             col[(4 * q + 1) * kTwoThreads] = (Sb.y + Pb.y) - (Sa.y + Pa.y);
             col[(4 * q + 2) * kTwoThreads] = (Sb.z + Pb.z) - (Sa.z + Pa.z);

@@ -353,7 +353,8 @@ __global__ void __launch_bounds__(32 * WARPS, MC <= 8 ? 8 : 4) k_dp_walk(GridVie
                 k[j] = wtask(g, wh, tabs_of(q), ES, i, ti - (i - 1) * TPE, qh_shift, qv_shift);
                 if (k[j].on) {
                     r[j][0] = __ldg(k[j].pa); r[j][1] = __ldg(k[j].pb);
-                    r[j][2] = __ldg(k[j].sa); r[j][3] = __ldg(k[j].sb);
+                    if (k[j].sa != k[j].sb) { r[j][2] = __ldg(k[j].sa); r[j][3] = __ldg(k[j].sb); }
+                    else { r[j][2] = make_uint4(0, 0, 0, 0); r[j][3] = r[j][2]; }   // one segment: bases cancel
                 }
             }
         }
@@ -675,7 +676,8 @@ __global__ void __launch_bounds__(32 * WARPS) k_dp_flow(GridView g, NetsView nv,
                     k[j] = wtask(g, wh, t, ES, i, it - (i - 1) * TPE, qh_shift, qv_shift);
                     if (k[j].on) {
                         r[j][0] = __ldg(k[j].pa); r[j][1] = __ldg(k[j].pb);
-                        r[j][2] = __ldg(k[j].sa); r[j][3] = __ldg(k[j].sb);
+                        if (k[j].sa != k[j].sb) { r[j][2] = __ldg(k[j].sa); r[j][3] = __ldg(k[j].sb); }
+                        else { r[j][2] = make_uint4(0, 0, 0, 0); r[j][3] = r[j][2]; }   // one segment: bases cancel
                     }
                 }
             }
