@@ -274,7 +274,7 @@ __device__ __forceinline__ GTask wtask(const GridView& g, const WHdr* wh, const 
 }
 
 template <int LT, int MC, int WARPS>
-__global__ void __launch_bounds__(32 * WARPS, MC <= 8 ? 8 : 4) k_dp_walk(GridView g, NetsView nv, const int32_t* __restrict__ list,
+__global__ void __launch_bounds__(32 * WARPS, MC <= 8 ? 5 : 4) k_dp_walk(GridView g, NetsView nv, const int32_t* __restrict__ list,
                                                          int count, Out o, int commit, HybView hy) {
     constexpr int G = WK<LT>::G, ES = WK<LT>::ES;
     extern __shared__ __align__(16) unsigned char smem[];
