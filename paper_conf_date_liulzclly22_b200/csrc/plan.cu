@@ -38,6 +38,28 @@ __device__ __forceinline__ void unpack_box(unsigned long long b, int& x0, int& y
     x0 = (int)(b & 0xFFFF); y0 = (int)((b >> 16) & 0xFFFF); x1 = (int)((b >> 32) & 0xFFFF); y1 = (int)(b >> 48);
 }
 
+// S0 outputs of one net: error flags, the R19 range bound, the (HPWL, id) sort key, the box.
+__device__ __forceinline__ void prep_finish(const PlanParams& p, int net, int m, int bad, int x0, int y0, int x1, int y1,
+                                            unsigned long long wl, int sb, unsigned long long* keys,
+                                            unsigned long long* box, int* msize, int* segb, int* counters) {
+    if (bad) {
+        atomicMin(&counters[1], net);
+        x0 = y0 = x1 = y1 = 0;
+    }
+    const bool trivial = (m == 1);
+    if (trivial) atomicAdd(&counters[0], 1);
+    if (!bad && !trivial) {
+        // R19: worst case of any route = every unit edge at max cost + every via stack at max
+        const unsigned long long bound = wl * p.max_ec + (unsigned long long)(3 * m) * p.vmax;   // Z: 2 bend stacks per edge
+        if (bound >= (unsigned long long)FGR_INF || m > p.max_nodes_large) atomicMin(&counters[2], net);
+    }
+    const unsigned hpwl = trivial ? 0xFFFFu : (unsigned)((x1 - x0) + (y1 - y0));
+    keys[net] = ((unsigned long long)hpwl << 32) | (unsigned)net;
+    box[net] = pack_box(x0, y0, x1, y1);
+    msize[net] = m;
+    segb[net] = sb;
+}
+
 // S0: one warp per net.
 __global__ void k_preprocess(PlanParams p, NetsView nv, unsigned long long* __restrict__ keys,
                              unsigned long long* __restrict__ box, int* __restrict__ msize, int* __restrict__ segb,
@@ -48,6 +70,7 @@ __global__ void k_preprocess(PlanParams p, NetsView nv, unsigned long long* __re
     const int net = warp;
     const int a0 = nv.off[net], a1 = nv.off[net + 1];
     const int m = a1 - a0;
+    if (m <= 32) return;   // k_preprocess_small
     int bad = (m <= 0);
     int x0 = 0x7FFF, y0 = 0x7FFF, x1 = -1, y1 = -1;
     unsigned long long wl = 0;
@@ -81,22 +104,42 @@ __global__ void k_preprocess(PlanParams p, NetsView nv, unsigned long long* __re
         sb += __shfl_xor_sync(0xffffffffu, sb, off);
     }
     if (lane) return;
-    if (bad) {
-        atomicMin(&counters[1], net);
-        x0 = y0 = x1 = y1 = 0;
+    prep_finish(p, net, m, bad, x0, y0, x1, y1, wl, sb, keys, box, msize, segb, counters);
+}
+
+// S0 for the nets of at most 32 nodes (almost all of them): one thread per net, the same checks
+// and outputs as the warp-per-net kernel above (which skips these nets).
+__global__ void __launch_bounds__(256) k_preprocess_small(PlanParams p, NetsView nv, unsigned long long* __restrict__ keys,
+                                                          unsigned long long* __restrict__ box, int* __restrict__ msize,
+                                                          int* __restrict__ segb, int* __restrict__ counters) {
+    const int net = (int)(blockIdx.x * (size_t)blockDim.x + threadIdx.x);
+    if (net >= p.N) return;
+    const int a0 = nv.off[net], a1 = nv.off[net + 1];
+    const int m = a1 - a0;
+    if (m > 32) return;
+    int bad = (m <= 0);
+    int x0 = 0x7FFF, y0 = 0x7FFF, x1 = -1, y1 = -1;
+    unsigned long long wl = 0;
+    int sb = 0;
+    for (int i = 0; i < m; i++) {
+        const int v = a0 + i;
+        const int x = nv.x[v], y = nv.y[v];
+        const int lo = nv.plo[v], hi = nv.phi[v];
+        if (x < 0 || x >= p.nx || y < 0 || y >= p.ny) bad = 1;
+        if (!((lo == -1 && hi == -1) || (lo >= 0 && lo <= hi && hi < p.L))) bad = 1;
+        x0 = min(x0, x); y0 = min(y0, y); x1 = max(x1, x); y1 = max(y1, y);
+        const int par = nv.par[v];
+        if (i == 0) { if (par != -1) bad = 1; }
+        else if (par < 0 || par >= i) bad = 1;
+        else {
+            const int xu = nv.x[a0 + par], yu = nv.y[a0 + par];
+            const int dx = abs(x - xu), dy = abs(y - yu);
+            if (dx == 0 && dy == 0) bad = 1;   // zero-length tree edge (R8)
+            wl += (unsigned long long)(dx + dy);
+            sb += (dx >> 5) + (dy >> 5) + 4;
+        }
     }
-    const bool trivial = (m == 1);
-    if (trivial) atomicAdd(&counters[0], 1);
-    if (!bad && !trivial) {
-        // R19: worst case of any route = every unit edge at max cost + every via stack at max
-        const unsigned long long bound = wl * p.max_ec + (unsigned long long)(3 * m) * p.vmax;   // Z: 2 bend stacks per edge
-        if (bound >= (unsigned long long)FGR_INF || m > p.max_nodes_large) atomicMin(&counters[2], net);
-    }
-    const unsigned hpwl = trivial ? 0xFFFFu : (unsigned)((x1 - x0) + (y1 - y0));
-    keys[net] = ((unsigned long long)hpwl << 32) | (unsigned)net;
-    box[net] = pack_box(x0, y0, x1, y1);
-    msize[net] = m;
-    segb[net] = sb;
+    prep_finish(p, net, m, bad, x0, y0, x1, y1, wl, sb, keys, box, msize, segb, counters);
 }
 
 __global__ void k_rank_boxes(int N, const int* __restrict__ counters, const unsigned long long* __restrict__ keys,
@@ -523,6 +566,7 @@ extern "C" FGR_API fgr_status fgr_plan(fgr_grid* g, const fgr_nets* nets, int32_
     FGR_CHECK_CUDA(g, cudaMemcpyAsync(counters, hc, sizeof(hc), cudaMemcpyHostToDevice, st));
     FGR_CHECK_CUDA(g, cudaMemsetAsync(tstart, 0, 2 * sizeof(int) * ntiles, st));
     int ps = fgr_prof_begin(g, PROF_PRE, st);
+    k_preprocess_small<<<(unsigned)(((size_t)N + 255) / 256), 256, 0, st>>>(p, nv, keys, box, msize, segb, counters);
     k_preprocess<<<(unsigned)(((size_t)N * 32 + 255) / 256), 256, 0, st>>>(p, nv, keys, box, msize, segb, counters);
     fgr_prof_end(g, ps, st);
     FGR_CHECK_CUDA(g, cudaGetLastError());
@@ -630,7 +674,7 @@ extern "C" FGR_API fgr_status fgr_plan(fgr_grid* g, const fgr_nets* nets, int32_
     k_finalize<<<(N + 255) / 256, 256, 0, st>>>(N, counters, keys_s, bkeys_s, msize, segb, order, batch_of_net,
                                                 d_nlarge, d_maxm, segsum, d_ntwo, d_n9, d_ls, fgr_top_limit(g));
     FGR_CHECK_CUDA(g, cudaGetLastError());
-    g->stats.kernel_launches += 6;
+    g->stats.kernel_launches += 7;
     int B = 0;
     FGR_CHECK_CUDA(g, cudaMemcpyAsync(&B, counters + 4, sizeof(int), cudaMemcpyDeviceToHost, st));
     FGR_CHECK_CUDA(g, cudaStreamSynchronize(st));  // sync 2 of 2
