@@ -850,8 +850,8 @@ cudaError_t launch_tree_v(fgr_grid* g, cudaStream_t st, const NetsView& nv, cons
 template <int LT>
 cudaError_t launch_tree_lt(fgr_grid* g, cudaStream_t st, const NetsView& nv, const int32_t* list, int n, int maxm,
                            const Out& o, const HldPrep& hp, const uint32_t* legs, int legs_maxm) {
-    if (maxm <= 128) return launch_tree_v<LT, 128, 128>(g, st, nv, list, n, o, hp, legs, legs_maxm);
-    if (maxm <= 512) return launch_tree_v<LT, 256, 512>(g, st, nv, list, n, o, hp, legs, legs_maxm);
+    if (maxm <= 128) return launch_tree_v<LT, 256, 128>(g, st, nv, list, n, o, hp, legs, legs_maxm);
+    if (maxm <= 512) return launch_tree_v<LT, 384, 512>(g, st, nv, list, n, o, hp, legs, legs_maxm);
     return launch_tree_v<LT, kTreeBigNT, tree_cap512(LT)>(g, st, nv, list, n, o, hp, legs, legs_maxm);
 }
 
